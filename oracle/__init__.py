@@ -1,0 +1,174 @@
+"""CPU oracle for the expander-walk PRNG (Banerjee, Bahl & Kothapalli, IPDPS-W 2012).
+
+TEST INFRASTRUCTURE ONLY.  Only ``tests/``, ``__graft_entry__.smoke()`` and the
+``cpu_baseline`` / ``--impl reference`` legs of ``bench.py`` may import this
+package.  The product package ``paper_conf_ipps_banerjeebk12_b200`` never
+imports it and shares no code with it.
+
+The arithmetic lives in plain single-threaded C (``gg_oracle.c``,
+``lr_oracle.c``, ``mc_oracle.c``); this module only compiles and loads it and
+marshals numpy arrays.  Every C function cites the PAPER.md passage it follows.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+import threading
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SOURCES = ["gg_oracle.c", "lr_oracle.c", "mc_oracle.c"]
+_LIB_PATH = os.path.join(_HERE, "libggoracle.so")
+_lock = threading.Lock()
+_lib = None
+
+u64 = ctypes.c_uint64
+u32 = ctypes.c_uint32
+i32 = ctypes.c_int32
+i64 = ctypes.c_int64
+f64 = ctypes.c_double
+P = ctypes.c_void_p
+
+
+def build(force: bool = False) -> str:
+    """Compile the oracle with gcc (plain -O2, no fast-math, no FP contraction)."""
+    srcs = [os.path.join(_HERE, s) for s in _SOURCES if os.path.exists(os.path.join(_HERE, s))]
+    newest = max(os.path.getmtime(s) for s in srcs)
+    if not force and os.path.exists(_LIB_PATH) and os.path.getmtime(_LIB_PATH) >= newest:
+        return _LIB_PATH
+    tmp = _LIB_PATH + f".tmp{os.getpid()}"
+    cmd = ["gcc", "-O2", "-std=c11", "-fPIC", "-shared", "-ffp-contract=off",
+           "-fno-fast-math", "-Wall", "-o", tmp] + srcs + ["-lm"]
+    subprocess.check_call(cmd)
+    os.replace(tmp, _LIB_PATH)
+    return _LIB_PATH
+
+
+def lib():
+    global _lib
+    with _lock:
+        if _lib is None:
+            build()
+            L = ctypes.CDLL(_LIB_PATH)
+            sig = {
+                "or_mix64": (u64, [u64]),
+                "or_stream_word64": (u64, [u64, u64, u64]),
+                "or_stream_word32": (u32, [u64, u64, u64]),
+                "or_words_per_walk": (u32, [u32]),
+                "or_bits3": (ctypes.c_int, [P, u32]),
+                "or_walk": (None, [u64, P, P, P, u32]),
+                "or_label": (u64, [u64, u64, u64]),
+                "or_draw_word_index": (u64, [u32, u32, u64, u32]),
+                "or_walker_init": (ctypes.c_int, [u64, u32, u64, u64, P, P]),
+                "or_walker_draw": (u64, [u64, u32, u32, u64, u64, u64, P, P]),
+                "or_bulk": (ctypes.c_int, [u64, u32, u32, u64, u64, u64, u64, P]),
+                "or_walker_draws": (ctypes.c_int, [u64, u32, u32, u64, u64, u64, u64, P]),
+                "or_sigma_array": (None, [u64, ctypes.c_int, P, P, P, P, u64]),
+                "or_stream_block": (None, [u64, u64, u64, u64, u32, P]),
+            }
+            for name, (res, args) in sig.items():
+                fn = getattr(L, name)
+                fn.restype = res
+                fn.argtypes = args
+            _bind_optional(L)
+            _lib = L
+    return _lib
+
+
+def _bind_optional(L):
+    """Signatures of the application oracles (list ranking, Monte Carlo)."""
+    opt = {
+        "or_lr_rank_seq": (ctypes.c_int, [i64, P, i64, P]),
+        "or_lr_run": (ctypes.c_int, [u64, u32, u32, u64, i64, P, P, i64, i64, P, P, P]),
+        "or_mc_run": (ctypes.c_int, [P, P, P, P]),
+    }
+    for name, (res, args) in opt.items():
+        fn = getattr(L, name, None)
+        if fn is not None:
+            fn.restype = res
+            fn.argtypes = args
+
+
+def _ptr(a: np.ndarray):
+    return ctypes.c_void_p(a.ctypes.data)
+
+
+# ----------------------------------------------------------------------------
+# Thin numpy wrappers (argument marshalling only).
+# ----------------------------------------------------------------------------
+
+def mix64(z: int) -> int:
+    return int(lib().or_mix64(z))
+
+
+def stream_word32(seed: int, t: int, k: int) -> int:
+    return int(lib().or_stream_word32(seed, t, k))
+
+
+def stream_word64(seed: int, t: int, c: int) -> int:
+    return int(lib().or_stream_word64(seed, t, c))
+
+
+def words_per_walk(nsteps: int) -> int:
+    return int(lib().or_words_per_walk(nsteps))
+
+
+def sigma(m: int, k: int, x, y):
+    """sigma_k applied elementwise to arrays x, y (uint64)."""
+    x = np.ascontiguousarray(x, dtype=np.uint64)
+    y = np.ascontiguousarray(y, dtype=np.uint64)
+    nx = np.empty_like(x)
+    ny = np.empty_like(y)
+    lib().or_sigma_array(m, k, _ptr(x), _ptr(y), _ptr(nx), _ptr(ny), x.size)
+    return nx, ny
+
+
+def bits3(rec, i: int) -> int:
+    rec = np.ascontiguousarray(rec, dtype=np.uint32)
+    return int(lib().or_bits3(_ptr(rec), i))
+
+
+def walk(m: int, x: int, y: int, rec, nsteps: int):
+    """One walk of nsteps with an explicit bit record (user-supplied bits)."""
+    rec = np.ascontiguousarray(rec, dtype=np.uint32)
+    xs = np.array([x], dtype=np.uint64)
+    ys = np.array([y], dtype=np.uint64)
+    lib().or_walk(m, _ptr(xs), _ptr(ys), _ptr(rec), nsteps)
+    return int(xs[0]), int(ys[0])
+
+
+def label(m: int, x: int, y: int) -> int:
+    return int(lib().or_label(m, x, y))
+
+
+def walker_init(m: int, l0: int, seed: int, t: int):
+    xs = np.zeros(1, dtype=np.uint64)
+    ys = np.zeros(1, dtype=np.uint64)
+    rc = lib().or_walker_init(m, l0, seed, t, _ptr(xs), _ptr(ys))
+    if rc != 0:
+        raise ValueError("or_walker_init failed")
+    return int(xs[0]), int(ys[0])
+
+
+def walker_draws(m: int, l: int, l0: int, seed: int, t: int, j0: int, nd: int) -> np.ndarray:
+    out = np.empty(nd, dtype=np.uint64)
+    rc = lib().or_walker_draws(m, l, l0, seed, t, j0, nd, _ptr(out))
+    if rc != 0:
+        raise ValueError("or_walker_draws failed")
+    return out
+
+
+def bulk(m: int, l: int, l0: int, seed: int, W: int, g0: int, n: int) -> np.ndarray:
+    out = np.empty(n, dtype=np.uint64)
+    rc = lib().or_bulk(m, l, l0, seed, W, g0, n, _ptr(out))
+    if rc != 0:
+        raise ValueError("or_bulk failed")
+    return out
+
+
+def stream_block(seed: int, t0: int, count: int, k0: int, nwords: int) -> np.ndarray:
+    out = np.empty((nwords, count), dtype=np.uint32)
+    lib().or_stream_block(seed, t0, count, k0, nwords, _ptr(out))
+    return out
