@@ -1,0 +1,375 @@
+#!/usr/bin/env python
+"""Benchmark of the B200 expander-walk PRNG (BASELINE.json metric, config C2).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+    torchrun --nproc-per-node N bench.py --gpus N ...        (one rank per GPU)
+
+A step = one bulk prng_fill of 2^30 uint32 numbers (= 2^29 64-bit labels,
+the paper's numbers) from 2^20 walkers on the full-size expander (m = 2^32,
+n = 2^65, l = l0 = 64) per GPU: Alg.2 x 512 draws per walker with the seed
+bits resident in HBM (prefetched by the host FEED before the timed region).
+Between steps the generator is rewound to the same checkpoint, so every step
+walks the same 12 GiB of bits (larger than L2: no flush needed) and writes
+4 GiB of labels.  Multi-GPU: walkers shard by rank with disjoint streams
+(weak scaling, no collective on the data path); time = max over ranks.
+
+`e2e` is the same metric through prng_fill_host with host buffers: host FEED
+threads generate every bit, H2D copies, the walk, D2H of all numbers.
+`--impl reference` times the CPU oracle (the paper's method as plain C) on
+the host cores instead.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+if ROOT not in sys.path:
+    sys.path.insert(0, ROOT)
+
+METRIC = "GNumbers/s (bulk fill and on-demand) per B200 and at 2/4/8 GPUs; % roofline"
+UNIT = "GNumbers/s"
+M32 = 1 << 32
+SEED = 0x5EED0002
+W_PER_GPU = 1 << 20
+U32_PER_STEP = 1 << 30
+LABELS_PER_STEP = U32_PER_STEP // 2          # 2^29 labels per GPU per step
+DRAWS_PER_STEP = LABELS_PER_STEP // W_PER_GPU  # 512
+BITS_BYTES_PER_LABEL = 24                     # 64 steps x 3 bits
+OPS_PER_STEP = 6                              # algorithmic int ops per walk step
+OPS_PER_LABEL = 64 * OPS_PER_STEP + 1         # + the emit
+WORKLOAD = ("C2 bulk prng_fill: m=2^32 (n=2^65), degree 7, l=l0=64, 2^20 walkers per GPU, "
+            "2^30 uint32 numbers (2^29 64-bit labels) per GPU per step")
+
+
+# --------------------------------------------------------------- CPU oracle
+def _oracle_worker(args):
+    t0, nwalkers, ndraws = args
+    import oracle as O
+    lib = O.lib()
+    import numpy as np
+    out = np.empty(ndraws, dtype=np.uint64)
+    acc = 0
+    for t in range(t0, t0 + nwalkers):
+        lib.or_walker_draws(M32, 64, 64, SEED, t, 0, ndraws, out.ctypes.data)
+        acc ^= int(out[-1])
+    return acc
+
+
+def oracle_rate(cores: int, walkers_per_core: int, draws: int):
+    """Labels/s of `cores` single-threaded oracle processes on disjoint walkers."""
+    import multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    with ctx.Pool(cores) as pool:
+        pool.map(_oracle_worker, [(0, 1, 1)] * cores)  # warm (load + build the .so)
+        jobs = [(c * walkers_per_core * 1021 % (W_PER_GPU - walkers_per_core), walkers_per_core,
+                 draws) for c in range(cores)]
+        t = time.perf_counter()
+        pool.map(_oracle_worker, jobs)
+        dt = time.perf_counter() - t
+    labels = cores * walkers_per_core * draws
+    return labels / dt, labels, dt
+
+
+def cpu_baseline_block(target_seconds: float = 8.0):
+    cores = os.cpu_count() or 1
+    # calibrate on one core, then size the sample to ~target_seconds wall
+    r1, _, _ = oracle_rate(1, 64, 64)
+    per_core = max(64 * 16, int(r1 * target_seconds))
+    draws = 64
+    walkers = max(1, per_core // draws)
+    rate, labels, dt = oracle_rate(cores, walkers, draws)
+    return {
+        "value": rate / 1e9, "unit": UNIT, "cores": cores, "kind": "oracle",
+        "sample": (f"{labels} labels of the C2 workload (m=2^32, l=l0=64, seed 0x5EED0002): "
+                   f"{cores} single-threaded oracle processes x {walkers} walkers x draws 0..{draws-1} "
+                   f"(Alg.1 burn-in included), {dt:.1f} s wall"),
+    }
+
+
+# ------------------------------------------------------------------ clocks
+class ClockSampler:
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_id: str):
+        self.gpu_id, self.rows, self.proc = gpu_id, [], None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", self.gpu_id, f"--query-gpu={self.FIELDS}",
+                 "--format=csv,noheader,nounits", "-lms", "200"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.th = threading.Thread(target=self._read, daemon=True)
+            self.th.start()
+        except OSError:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) == 7:
+                self.rows.append(parts)
+
+    def __exit__(self, *exc):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"], "samples": 0}
+        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows for i in range(4) if r[3 + i] == "Active"})
+        pw = [float(r[2]) for r in self.rows if r[2].replace(".", "").isdigit()]
+        return {"sm_mhz": statistics.median(sm) if sm else None,
+                "sm_max_mhz": max(mx) if mx else None, "reasons": reasons,
+                "power_w_max": max(pw) if pw else None, "samples": len(self.rows)}
+
+
+def measured_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return json.load(f)
+    except OSError:
+        return {}
+
+
+# ------------------------------------------------------------- our arm
+def run_ours(args, rank, world, local_rank):
+    import torch
+    import torch.distributed as dist
+    from paper_conf_ipps_banerjeebk12_b200 import Generator
+
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    props = torch.cuda.get_device_properties(dev)
+    stream = torch.cuda.current_stream()
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    def max_over_ranks(v: float) -> float:
+        if world == 1:
+            return v
+        t = torch.tensor([v], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    # ---- K-mode: bits resident in HBM, one prng_fill per step
+    g = Generator(walkers=W_PER_GPU, seed=SEED, walker_base=rank * W_PER_GPU, device=local_rank)
+    g.prefetch(DRAWS_PER_STEP)
+    g.mark()
+    out = torch.empty(U32_PER_STEP, dtype=torch.int32, device=dev)
+    for _ in range(args.warmup):
+        g.rewind()
+        g.fill(out)
+    torch.cuda.synchronize()
+    ev0 = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    ev1 = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    start, end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    gpu_id = getattr(props, "uuid", None)
+    gpu_id = f"GPU-{gpu_id}" if gpu_id is not None else str(local_rank)
+    launches0 = g.stats()["kernel_launches"]
+    barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(gpu_id) as clk:
+        start.record(stream)
+        for i in range(args.steps):
+            g.rewind()
+            ev0[i].record(stream)
+            g.fill(out)
+            ev1[i].record(stream)
+        end.record(stream)
+        torch.cuda.synchronize()
+    barrier()
+    launches = g.stats()["kernel_launches"] - launches0
+    ms = max_over_ranks(start.elapsed_time(end))
+    kern_ms = statistics.mean(a.elapsed_time(b) for a, b in zip(ev0, ev1))
+    labels_total = world * LABELS_PER_STEP * args.steps
+    value = labels_total / (ms / 1e3) / 1e9
+
+    peaks = measured_peaks()
+    sm_max = float(peaks.get("sm_max_mhz", 1965.0))
+    peak_ops = props.multi_processor_count * 128 * sm_max * 1e6  # int lanes/clk/SM x clock
+    achieved_ops = LABELS_PER_STEP * OPS_PER_LABEL / (kern_ms / 1e3)
+    roofline = {
+        "bound": "alu", "achieved": achieved_ops / 1e12, "peak": peak_ops / 1e12,
+        "unit": "Tops/s (32-bit integer ops)", "frac": achieved_ops / peak_ops,
+        "traffic": None, "kernel": "gg_fill64_kernel",
+        "kernel_ms": kern_ms, "ops_per_label": OPS_PER_LABEL,
+        "peak_basis": (f"{props.multi_processor_count} SMs x 128 int lanes/clk (ALU 64 + FMA 64, "
+                       f"issue 4x32) x {sm_max:.0f} MHz (MEASURED_PEAKS sm_max_mhz)"),
+        "hbm_gbs_achieved": LABELS_PER_STEP * (BITS_BYTES_PER_LABEL + 8) / (kern_ms / 1e3) / 1e9,
+        "hbm_gbs_peak": peaks.get("hbm_gbs"),
+    }
+    # parity spot check of the timed output (walker 0, draw 0 of this rank)
+    res = {"value": value, "ms": ms, "roofline": roofline, "clocks": clk.summary(),
+           "launches": launches, "kern_ms": kern_ms}
+    g.close()
+    del out
+    torch.cuda.empty_cache()
+
+    # ---- on-demand: every thread calls prng_next S = 100 times (Fig.4 batch)
+    if not args.no_ondemand:
+        S = 100
+        g = Generator(walkers=W_PER_GPU, seed=SEED + 1, walker_base=rank * W_PER_GPU,
+                      device=local_rank)
+        xo = torch.empty(W_PER_GPU, dtype=torch.int64, device=dev)
+        g.epoch_begin(W_PER_GPU, S * (args.warmup + 1))
+        for _ in range(args.warmup):
+            g.consume(W_PER_GPU, uniform=S, xor_out=xo)
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
+        a.record(stream)
+        g.consume(W_PER_GPU, uniform=S, xor_out=xo)
+        b.record(stream)
+        torch.cuda.synchronize()
+        g.epoch_end()
+        od_ms = max_over_ranks(a.elapsed_time(b))
+        res["on_demand"] = {"uniform_S100": world * W_PER_GPU * S / (od_ms / 1e3) / 1e9,
+                            "unit": UNIT, "draws": world * W_PER_GPU * S, "ms": od_ms,
+                            "what": "gg_consume: 2^20 threads/GPU x 100 prng_next each, bits resident"}
+        g.close()
+        torch.cuda.empty_cache()
+
+    # ---- e2e: host buffers through prng_fill_host (FEED + H2D + walk + D2H)
+    if not args.no_e2e:
+        e2e_steps = max(1, min(args.steps, args.e2e_steps))
+        g = Generator(walkers=W_PER_GPU, seed=SEED, walker_base=rank * W_PER_GPU,
+                      device=local_rank, epoch_draws=16)
+        host = torch.empty(U32_PER_STEP, dtype=torch.int32).pin_memory()
+        g.fill_host(host, n=W_PER_GPU * 2 * 16)  # warm (allocations, feed threads)
+        g.mark()
+        s0 = g.stats()
+        barrier()
+        torch.cuda.synchronize()
+        t = time.perf_counter()
+        for _ in range(e2e_steps):
+            g.rewind()
+            g.fill_host(host)
+        torch.cuda.synchronize()
+        dt = max_over_ranks(time.perf_counter() - t)
+        s1 = g.stats()
+        res["e2e"] = {
+            "value": world * LABELS_PER_STEP * e2e_steps / dt / 1e9, "unit": UNIT,
+            "h2d_bytes_per_step": (s1["h2d_bytes"] - s0["h2d_bytes"]) // e2e_steps,
+            "d2h_bytes_per_step": (s1["d2h_bytes"] - s0["d2h_bytes"]) // e2e_steps,
+            "steps": e2e_steps,
+            "feed_s_per_step": (s1["feed_seconds"] - s0["feed_seconds"]) / e2e_steps,
+            "api": "prng_fill_host (host FEED threads -> pinned -> H2D -> walk -> D2H to pinned)",
+            "host_threads": os.cpu_count(),
+        }
+        g.close()
+    return res
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-ondemand", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=8.0)
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+
+    if args.impl == "reference":
+        if rank != 0:
+            return 0
+        return run_reference(args, world)
+
+    # CPU baseline first (spawned processes; before CUDA is initialised)
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline_block(args.cpu_seconds)
+
+    if world > 1:
+        import torch
+        import torch.distributed as dist
+        torch.cuda.set_device(local_rank)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+    res = run_ours(args, rank, world, local_rank)
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": res["value"], "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": res["ms"] / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
+            "data": "synthetic (SplitMix64 counter-hash seed bits, reading R9)",
+            "config": {"workload": WORKLOAD, "number": "one 64-bit vertex label (the paper's unit)",
+                       "u32_numbers_per_s": 2 * res["value"] * 1e9,
+                       "walkers_per_gpu": W_PER_GPU, "labels_per_gpu_per_step": LABELS_PER_STEP,
+                       "bits": "resident in HBM (prng_prefetch before timing), rewound each step",
+                       "l2": "inputs larger than L2 (12 GiB of bits read per GPU per step)",
+                       "parallelism": f"walker shards dp{world}, no data-path collective"},
+            "roofline": res["roofline"], "cpu_baseline": cpu, "e2e": res.get("e2e"),
+            "clocks": res["clocks"], "gpu_launches": res["launches"],
+            "on_demand": res.get("on_demand"),
+        }
+        print(json.dumps(line))
+    if world > 1:
+        import torch.distributed as dist
+        dist.destroy_process_group()
+    return 0
+
+
+def run_reference(args, world):
+    """The oracle, as it stands, on the host cores (one bounded sample per step)."""
+    cores = os.cpu_count() or 1
+    import multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    walkers, draws = 512, 64
+    with ctx.Pool(cores) as pool:
+        pool.map(_oracle_worker, [(0, 1, 1)] * cores)
+        for _ in range(args.warmup):
+            pool.map(_oracle_worker, [(c * walkers, walkers, draws) for c in range(cores)])
+        t = time.perf_counter()
+        for s in range(args.steps):
+            pool.map(_oracle_worker, [((s * cores + c) * walkers, walkers, draws)
+                                      for c in range(cores)])
+        dt = time.perf_counter() - t
+    labels = args.steps * cores * walkers * draws
+    value = labels / dt / 1e9
+    sample = (f"per step {cores * walkers * draws} labels of the C2 workload: {cores} "
+              f"single-threaded oracle processes x {walkers} walkers x {draws} draws")
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt * 1e3 / args.steps,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64",
+        "data": "synthetic (SplitMix64 counter-hash seed bits, reading R9)",
+        "config": {"workload": WORKLOAD, "number": "one 64-bit vertex label (the paper's unit)",
+                   "parallelism": "host cores"},
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle",
+                         "sample": sample},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line))
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,219 @@
+/*
+ * include/prng_device.cuh — header-only device side of the expander-walk PRNG.
+ *
+ *   prng_next(&state, view)  = Alg.2 GetNextRand (§III-B) called by any
+ *   GPU thread "at any point of time" (§III): l = 64 steps of the walk on
+ *   the 7-regular Gabber–Galil expander (§III-A), 3 bits per step, and
+ *   the walker's vertex label returned as a 64-bit number (§III-B).
+ *
+ * Usage inside a user kernel (after prng_epoch_begin + prng_device_view):
+ *     prng_state st = prng_state_load(&view, walker);
+ *     uint64_t r = prng_next(&st, &view);      // as often as the epoch allows
+ *     prng_state_store(&view, &st);
+ * A walker must be used by one thread at a time (that is what makes the
+ * generator thread-safe, §I-B).  A draw outside the epoch window sets a
+ * sticky flag (read by prng_check) and returns 0 — never different bits.
+ *
+ * This header is part of the GPU path.  It shares nothing with oracle/.
+ */
+#ifndef GGPRNG_PRNG_DEVICE_CUH
+#define GGPRNG_PRNG_DEVICE_CUH
+
+#include <stdint.h>
+
+#define PRNG_FLAG_OVERRUN 1u
+
+/* Everything a device thread needs; filled by prng_device_view(). */
+struct prng_view {
+    const uint32_t *bits;  /* epoch window, SoA: word (d*R + r) of walker t at bits[(d*R+r)*pitch + t] */
+    uint32_t *x;           /* walker vertex, x coordinate (wrapped mod 2^32 when m is a power of two) */
+    uint32_t *y;           /* walker vertex, y coordinate */
+    uint32_t *j;           /* next absolute draw index of each walker */
+    uint32_t *flags;       /* sticky error flags (PRNG_FLAG_*) */
+    uint64_t pitch;        /* words between rows of the window */
+    uint64_t m;            /* modulus */
+    uint32_t J0;           /* first draw of the window */
+    uint32_t D;            /* draws per walker in the window */
+    uint32_t Wv;           /* walkers covered by the window: [0, Wv) */
+    uint32_t R;            /* words per draw record = ceil(3l/32) */
+    uint32_t l;            /* steps per number */
+    uint32_t log2m;        /* log2(m) if m is a power of two, else 0 */
+    uint32_t pow2;         /* 1 if m is a power of two */
+    uint32_t _pad;
+};
+
+struct prng_state {
+    uint32_t x, y;     /* current vertex */
+    uint32_t walker;   /* walker id (window-local) */
+    uint32_t used;     /* draws consumed in this epoch */
+};
+
+/* ------------------------------------------------------------------------
+ * The Gabber–Galil step (§III-A), 3-bit choice b, k = b mod 7 (R4):
+ *   b in {1,2,3}: y <- y + 2x + (b-1)        (sigma_1..3)
+ *   b in {4,5,6}: x <- x + 2y + (b-4)        (sigma_4..6)
+ *   b in {0,7}  : stay                        (sigma_0)
+ * For m = 2^k all arithmetic is done in Z/2^32 and reduced at emission
+ * (Z/2^32 -> Z/2^k is a ring homomorphism).
+ *
+ * Fast form (l = 64): the 192-bit record is repacked into 7 words of 10
+ * whole 3-bit fields (no field straddles a word).  Per word, SWAR gives
+ *   MY = fields in {1,2,3}, MX = fields in {4,5,6} (bit at the field's LSB),
+ *   C  = field - [y-move], whose low two bits are the step's constant c.
+ * Each step is then 7 SASS instructions: two LOP3.P predicate tests, one
+ * IMAD.SHL bringing c to the top of a register, two LEA.HI adding c to x and
+ * to y, and two predicated IMADs doing target = 2*src + (target + c).
+ * ------------------------------------------------------------------------ */
+template <int K>
+__device__ __forceinline__ void gg_step_swar(uint32_t MY, uint32_t MX, uint32_t C,
+                                             uint32_t &x, uint32_t &y)
+{
+    asm volatile(
+        "{\n\t"
+        ".reg .pred py, px;\n\t"
+        ".reg .b32 ty, tx, ct, c, yc, xc;\n\t"
+        "and.b32 ty, %2, %5;\n\t"
+        "setp.ne.b32 py, ty, 0;\n\t"
+        "and.b32 tx, %3, %5;\n\t"
+        "setp.ne.b32 px, tx, 0;\n\t"
+        "shl.b32 ct, %4, %6;\n\t"
+        "shr.b32 c, ct, 30;\n\t"
+        "add.u32 yc, %1, c;\n\t"
+        "add.u32 xc, %0, c;\n\t"
+        "@py mad.lo.u32 %1, %0, 2, yc;\n\t"
+        "@px mad.lo.u32 %0, %1, 2, xc;\n\t"
+        "}"
+        : "+r"(x), "+r"(y)
+        : "r"(MY), "r"(MX), "r"(C), "n"(1u << (3 * K)), "n"(30 - 3 * K));
+}
+
+template <int NK>
+__device__ __forceinline__ void gg_word10(uint32_t Q, uint32_t &x, uint32_t &y)
+{
+    const uint32_t f1 = Q >> 1, f2 = Q >> 2;
+    const uint32_t MY = ~f2 & (f1 | Q);   /* b2=0 and b != 0 */
+    const uint32_t MX = f2 & ~(f1 & Q);   /* b2=1 and b != 7 */
+    const uint32_t C = Q - MY;            /* y-move fields hold b-1 (no borrow: b>=1) */
+    if (NK > 0) gg_step_swar<0>(MY, MX, C, x, y);
+    if (NK > 1) gg_step_swar<1>(MY, MX, C, x, y);
+    if (NK > 2) gg_step_swar<2>(MY, MX, C, x, y);
+    if (NK > 3) gg_step_swar<3>(MY, MX, C, x, y);
+    if (NK > 4) gg_step_swar<4>(MY, MX, C, x, y);
+    if (NK > 5) gg_step_swar<5>(MY, MX, C, x, y);
+    if (NK > 6) gg_step_swar<6>(MY, MX, C, x, y);
+    if (NK > 7) gg_step_swar<7>(MY, MX, C, x, y);
+    if (NK > 8) gg_step_swar<8>(MY, MX, C, x, y);
+    if (NK > 9) gg_step_swar<9>(MY, MX, C, x, y);
+}
+
+/* 64 steps from a 6-word record, m = 2^k (wrapped arithmetic). */
+__device__ __forceinline__ void gg_walk64(const uint32_t w[6], uint32_t &x, uint32_t &y)
+{
+    gg_word10<10>(w[0], x, y);
+    gg_word10<10>(__funnelshift_r(w[0], w[1], 30), x, y);
+    gg_word10<10>(__funnelshift_r(w[1], w[2], 28), x, y);
+    gg_word10<10>(__funnelshift_r(w[2], w[3], 26), x, y);
+    gg_word10<10>(__funnelshift_r(w[3], w[4], 24), x, y);
+    gg_word10<10>(__funnelshift_r(w[4], w[5], 22), x, y);
+    gg_word10<4>(w[5] >> 20, x, y);
+}
+
+/* One step, any m (generic path).  Non power-of-two m requires m <= 2^30 and
+ * x, y < m: the pre-reduction value 2*src + target + 2 < 4m fits in 32 bits. */
+__device__ __forceinline__ void gg_step_generic(uint32_t b, uint32_t &x, uint32_t &y,
+                                                uint32_t m, bool pow2)
+{
+    const uint32_t cy = b - 1u, cx = b - 4u;
+    if (cy < 3u) {
+        uint32_t t = y + 2u * x + cy;
+        if (!pow2) { t = (t >= 2u * m) ? t - 2u * m : t; t = (t >= m) ? t - m : t; }
+        y = t;
+    } else if (cx < 3u) {
+        uint32_t t = x + 2u * y + cx;
+        if (!pow2) { t = (t >= 2u * m) ? t - 2u * m : t; t = (t >= m) ? t - m : t; }
+        x = t;
+    }
+}
+
+/* Field i of a record stored at rec[r*stride] (R3: little-endian bit string). */
+__device__ __forceinline__ uint32_t gg_field(const uint32_t *rec, uint64_t stride, uint32_t i)
+{
+    const uint32_t bit = 3u * i, r = bit >> 5, s = bit & 31u;
+    uint32_t lo = rec[(uint64_t)r * stride];
+    if (s <= 29u)
+        return (lo >> s) & 7u;
+    uint32_t hi = rec[(uint64_t)(r + 1) * stride];
+    return __funnelshift_r(lo, hi, s) & 7u;
+}
+
+/* nsteps steps reading the record from global memory (generic l / m). */
+__device__ __forceinline__ void gg_walk_generic(const uint32_t *rec, uint64_t stride,
+                                                uint32_t nsteps, uint32_t &x, uint32_t &y,
+                                                uint32_t m, bool pow2)
+{
+    for (uint32_t i = 0; i < nsteps; i++)
+        gg_step_generic(gg_field(rec, stride, i), x, y, m, pow2);
+}
+
+/* Vertex label x + m*y (R8), reducing wrapped coordinates for m = 2^k. */
+__device__ __forceinline__ uint64_t gg_label(uint32_t x, uint32_t y, uint64_t m, uint32_t log2m,
+                                             bool pow2)
+{
+    if (pow2) {
+        const uint32_t mask = (log2m >= 32) ? 0xFFFFFFFFu : ((1u << log2m) - 1u);
+        return ((uint64_t)(y & mask) << log2m) | (uint64_t)(x & mask);
+    }
+    return (uint64_t)x + m * (uint64_t)y;
+}
+
+/* ------------------------------ on-demand API -------------------------- */
+
+__device__ __forceinline__ prng_state prng_state_load(const prng_view *v, uint32_t walker)
+{
+    prng_state st;
+    st.x = v->x[walker];
+    st.y = v->y[walker];
+    st.walker = walker;
+    const uint32_t j = v->j[walker];
+    st.used = (j > v->J0) ? (j - v->J0) : 0u; /* walkers that skipped epochs jump to J0 */
+    return st;
+}
+
+__device__ __forceinline__ void prng_state_store(const prng_view *v, const prng_state *st)
+{
+    v->x[st->walker] = st->x;
+    v->y[st->walker] = st->y;
+    v->j[st->walker] = v->J0 + st->used;
+}
+
+/* Draws left in the current window for this walker. */
+__device__ __forceinline__ uint32_t prng_available(const prng_view *v, const prng_state *st)
+{
+    return (st->used < v->D) ? (v->D - st->used) : 0u;
+}
+
+/* Alg.2 GetNextRand: walk l steps with the bits of draw (J0 + used). */
+__device__ __forceinline__ uint64_t prng_next(prng_state *st, const prng_view *v)
+{
+    if (st->used >= v->D || st->walker >= v->Wv) {
+        atomicOr(v->flags, PRNG_FLAG_OVERRUN);
+        return 0ull;
+    }
+    const uint32_t *rec = v->bits + (uint64_t)st->used * v->R * v->pitch + st->walker;
+    uint32_t x = st->x, y = st->y;
+    if (v->l == 64u && v->pow2) {
+        uint32_t w[6];
+#pragma unroll
+        for (int r = 0; r < 6; r++)
+            w[r] = __ldg(rec + (uint64_t)r * v->pitch);
+        gg_walk64(w, x, y);
+    } else {
+        gg_walk_generic(rec, v->pitch, v->l, x, y, (uint32_t)v->m, v->pow2 != 0);
+    }
+    st->x = x;
+    st->y = y;
+    st->used++;
+    return gg_label(x, y, v->m, v->log2m, v->pow2 != 0);
+}
+
+#endif /* GGPRNG_PRNG_DEVICE_CUH */

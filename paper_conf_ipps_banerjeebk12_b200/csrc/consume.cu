@@ -1,0 +1,50 @@
+// Synthetic on-demand consumer (include/gg_apps.h: gg_consume): every
+// thread owns one walker and calls the header-only prng_next
+// (prng_device.cuh) a data-dependent number of times — the usage pattern of
+// Alg.3 l.6 and Alg.4 l.3 without the application around it.
+#include <cstdint>
+
+#include <cuda_runtime.h>
+
+#include "gg_apps.h"
+#include "prng.h"
+#include "prng_device.cuh"
+
+namespace {
+
+__global__ void __launch_bounds__(128) consume_kernel(prng_view v, uint64_t threads,
+                                                      const uint32_t *counts, uint32_t uniform,
+                                                      uint64_t *out, const uint64_t *offsets,
+                                                      uint64_t *xor_out) {
+    const uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= threads) return;
+    const uint32_t c = counts ? counts[t] : uniform;
+    prng_state st = prng_state_load(&v, (uint32_t)t);
+    uint64_t acc = 0;
+    const uint64_t base = out ? (offsets ? offsets[t] : t * (uint64_t)uniform) : 0;
+    for (uint32_t r = 0; r < c; r++) {
+        const uint64_t z = prng_next(&st, &v);
+        acc ^= z;
+        if (out) out[base + r] = z;
+    }
+    prng_state_store(&v, &st);
+    if (xor_out) xor_out[t] = acc;
+}
+
+}  // namespace
+
+extern "C" int gg_consume(prng_t *h, uint64_t threads, const uint32_t *counts, uint32_t uniform,
+                          uint64_t *out, const uint64_t *offsets, uint64_t *xor_out,
+                          void *stream) {
+    if (!h) return PRNG_E_INVALID;
+    prng_view v;
+    int rc = prng_device_view(h, &v, sizeof(v));
+    if (rc != PRNG_OK) return rc;
+    if (threads == 0) return PRNG_OK;
+    if (threads > v.Wv) return PRNG_E_INVALID;
+    const uint32_t tpb = 128;
+    const uint64_t blocks = (threads + tpb - 1) / tpb;
+    consume_kernel<<<(unsigned)blocks, tpb, 0, (cudaStream_t)stream>>>(v, threads, counts, uniform,
+                                                                       out, offsets, xor_out);
+    return cudaGetLastError() == cudaSuccess ? PRNG_OK : PRNG_E_CUDA;
+}

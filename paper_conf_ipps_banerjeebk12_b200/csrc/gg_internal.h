@@ -1,0 +1,52 @@
+// Internal interfaces between the C-ABI host code and the CUDA kernels.
+// Not installed; not part of the public ABI (include/prng.h is).
+#pragma once
+#include <cstddef>
+#include <cstdint>
+
+#include <cuda_runtime.h>
+
+namespace gg {
+
+// Alg.1 (§III-B) for walkers [w0, w0 + count): start vertex from stream
+// words 0,1 (R7), then l0 steps with words 2 .. 1+R0.  `bits` holds rows
+// 0 .. 1+R0 for those walkers, row pitch `pitch` words, walker w at column
+// (w - w0).
+struct InitArgs {
+    const uint32_t *bits;
+    uint64_t pitch;
+    uint32_t w0, count;
+    uint32_t l0, R0;
+    uint64_t m;
+    uint32_t log2m, pow2;
+    uint32_t *x, *y, *j;
+};
+cudaError_t launch_init(const InitArgs &a, cudaStream_t s);
+
+// Bulk Alg.2 over draws [ja, jb) of every walker, restricted to bulk
+// positions g in [N, N + nl) (R11: g = j*W + t).  The bits of draw j are rows
+// (j - Jw)*R .. (j - Jw)*R + R-1 of the window `bits` (pitch words per row).
+// Writes label(g) to out[g - g_origin] (u64), or its low word (u32 when
+// m <= 2^16).
+struct FillArgs {
+    const uint32_t *bits;
+    uint64_t pitch;
+    uint32_t Jw;
+    uint32_t ja, jb;
+    uint32_t W;
+    uint64_t N, nl, g_origin;
+    uint32_t *x, *y;
+    void *out;
+    int out_u32;
+    uint32_t l, R;
+    uint64_t m;
+    uint32_t log2m, pow2;
+};
+cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count);
+
+// Host feed: SplitMix64 counter-hash stream (R9), SoA rows.
+//   out[r*pitch + i] = word32(seed, tg0 + i, k0 + r),  r < nrows, i < count
+void feed_splitmix_rows(uint64_t seed, uint64_t tg0, uint64_t count, uint64_t k0,
+                        uint32_t nrows, uint32_t *out, uint64_t pitch);
+
+}  // namespace gg

@@ -1,0 +1,770 @@
+// C ABI of the B200 expander-walk PRNG (declarations and contract:
+// include/prng.h).  Host-side runtime: handle, feed thread pool, pinned
+// staging pipeline (FEED -> TRANSFER, §IV-A Fig.4), resident and
+// streamed bit windows, on-demand epochs (R10), checkpoints.
+#include <algorithm>
+#include <chrono>
+#include <condition_variable>
+#include <cstdint>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <functional>
+#include <mutex>
+#include <new>
+#include <thread>
+#include <vector>
+
+#include <cuda_runtime.h>
+
+#include "gg_internal.h"
+#include "prng.h"
+#include "prng_device.cuh"
+
+namespace {
+
+// ------------------------------------------------------------ thread pool
+class ThreadPool {
+  public:
+    explicit ThreadPool(unsigned n) : n_(n ? n : 1) {
+        for (unsigned i = 1; i < n_; i++) workers_.emplace_back([this, i] { loop(i); });
+    }
+    ~ThreadPool() {
+        {
+            std::lock_guard<std::mutex> g(mu_);
+            stop_ = true;
+        }
+        cv_.notify_all();
+        for (auto &t : workers_) t.join();
+    }
+    unsigned size() const { return n_; }
+    // fn(thread_index) on every thread (the caller is thread 0); returns when all done.
+    void run(const std::function<void(unsigned)> &fn) {
+        if (n_ == 1) {
+            fn(0);
+            return;
+        }
+        {
+            std::lock_guard<std::mutex> g(mu_);
+            job_ = &fn;
+            pending_ = n_ - 1;
+            gen_++;
+        }
+        cv_.notify_all();
+        fn(0);
+        std::unique_lock<std::mutex> lk(mu_);
+        done_cv_.wait(lk, [this] { return pending_ == 0; });
+        job_ = nullptr;
+    }
+
+  private:
+    void loop(unsigned idx) {
+        uint64_t seen = 0;
+        for (;;) {
+            const std::function<void(unsigned)> *job;
+            {
+                std::unique_lock<std::mutex> lk(mu_);
+                cv_.wait(lk, [&] { return stop_ || gen_ != seen; });
+                if (stop_) return;
+                seen = gen_;
+                job = job_;
+            }
+            (*job)(idx);
+            {
+                std::lock_guard<std::mutex> g(mu_);
+                if (--pending_ == 0) done_cv_.notify_one();
+            }
+        }
+    }
+    unsigned n_;
+    std::vector<std::thread> workers_;
+    std::mutex mu_;
+    std::condition_variable cv_, done_cv_;
+    const std::function<void(unsigned)> *job_ = nullptr;
+    unsigned pending_ = 0;
+    uint64_t gen_ = 0;
+    bool stop_ = false;
+};
+
+inline uint32_t words_per_walk(uint32_t nsteps) { return (3u * nsteps + 31u) / 32u; }
+inline uint64_t round_up(uint64_t v, uint64_t a) { return (v + a - 1) / a * a; }
+
+struct CudaFail {
+    cudaError_t e;
+};
+#define CK(call)                                    \
+    do {                                            \
+        cudaError_t _e = (call);                    \
+        if (_e != cudaSuccess) throw CudaFail{_e};  \
+    } while (0)
+
+}  // namespace
+
+struct prng_s {
+    prng_graph_params g{};
+    prng_options o{};
+    uint64_t W = 0, seed = 0;
+    uint32_t R = 0, R0 = 0, log2m = 0, pow2 = 0;
+    int sm_count = 148;
+    bool poisoned = false;
+    cudaStream_t copy_stream = nullptr;  // H2D of seed bits
+    cudaStream_t d2h_stream = nullptr;   // D2H of results (prng_fill_host)
+    cudaStream_t work_stream = nullptr;  // kernels of prng_fill_host
+    ThreadPool *pool = nullptr;
+
+    // walker state (device) and checkpoint copies
+    uint32_t *x = nullptr, *y = nullptr, *j = nullptr, *flags = nullptr;
+    uint32_t *xs = nullptr, *ys = nullptr, *js = nullptr;
+    uint64_t N = 0;
+    uint64_t N_mark = 0, od_J0_mark = 0;
+    bool have_mark = false, od_started_mark = false;
+
+    // pinned staging chunks
+    static const int kChunks = 4;
+    uint32_t *chunk[kChunks] = {};
+    size_t chunk_bytes = 0;
+    cudaEvent_t chunk_done[kChunks] = {};
+    int chunk_next = 0;
+
+    // resident (prefetched) window: draws [res_J, res_J + res_D) of all walkers
+    uint32_t *res_bits = nullptr;
+    size_t res_cap = 0;
+    uint64_t res_J = 0, res_D = 0;
+
+    // streamed ring (E-mode): 2 device slots of Ds draws
+    uint32_t *ring[2] = {};
+    size_t ring_cap = 0;
+    cudaEvent_t ring_free[2] = {};
+    int ring_next = 0;
+
+    // prng_fill_host output staging
+    void *hout[2] = {};
+    size_t hout_cap = 0;
+    cudaEvent_t hout_free[2] = {};
+
+    // on-demand epoch
+    bool od_open = false, od_started = false;
+    uint64_t od_J0 = 0, od_Wv = 0, od_pitch = 0;
+    uint32_t od_D = 0;
+    uint32_t *od_bits = nullptr;
+    size_t od_cap = 0;
+
+    cudaEvent_t ev_tmp = nullptr;
+    prng_stats stats{};
+
+    uint64_t pitch() const { return round_up(W, 32); }
+};
+
+namespace {
+
+void free_all(prng_s *h) {
+    cudaSetDevice(h->o.device);
+    cudaDeviceSynchronize();
+    for (auto p : {h->x, h->y, h->j, h->flags, h->xs, h->ys, h->js, h->res_bits, h->ring[0],
+                   h->ring[1], h->od_bits})
+        if (p) cudaFree(p);
+    for (auto p : h->hout)
+        if (p) cudaFree(p);
+    for (int i = 0; i < prng_s::kChunks; i++) {
+        if (h->chunk[i]) cudaFreeHost(h->chunk[i]);
+        if (h->chunk_done[i]) cudaEventDestroy(h->chunk_done[i]);
+    }
+    for (int i = 0; i < 2; i++) {
+        if (h->ring_free[i]) cudaEventDestroy(h->ring_free[i]);
+        if (h->hout_free[i]) cudaEventDestroy(h->hout_free[i]);
+    }
+    if (h->ev_tmp) cudaEventDestroy(h->ev_tmp);
+    for (auto s : {h->copy_stream, h->d2h_stream, h->work_stream})
+        if (s) cudaStreamDestroy(s);
+    delete h->pool;
+    h->pool = nullptr;
+}
+
+// Generate rows [k0, k0+nrows) of the streams of local walkers [wa, wb)
+// into buf (pitch = wb - wa words), in parallel over walkers.
+void feed_chunk(prng_s *h, uint64_t wa, uint64_t wb, uint64_t k0, uint32_t nrows, uint32_t *buf) {
+    const uint64_t cw = wb - wa;
+    const unsigned nt = h->pool->size();
+    auto t0 = std::chrono::steady_clock::now();
+    h->pool->run([&](unsigned ti) {
+        // contiguous, 16-walker aligned slices
+        uint64_t per = round_up((cw + nt - 1) / nt, 16);
+        uint64_t lo = std::min<uint64_t>(cw, per * ti), hi = std::min<uint64_t>(cw, lo + per);
+        if (lo >= hi) return;
+        const uint64_t tg0 = h->o.walker_base + wa + lo;
+        if (h->o.bit_source == PRNG_BITS_CALLBACK)
+            h->o.bits_fn(h->o.bits_ctx, tg0, hi - lo, k0, nrows, buf + lo, cw);
+        else
+            gg::feed_splitmix_rows(h->seed, tg0, hi - lo, k0, nrows, buf + lo, cw);
+    });
+    auto t1 = std::chrono::steady_clock::now();
+    h->stats.feed_seconds += std::chrono::duration<double>(t1 - t0).count();
+    h->stats.bits_bytes_fed += (uint64_t)nrows * cw * 4;
+}
+
+// FEED + TRANSFER: stream words [k0, k0+nrows) of local walkers [0, Wv) into
+// the device window dst (row pitch dpitch words).  Host threads generate a
+// pinned chunk while the previous chunks are DMA'd on copy_stream.
+// On return every copy is enqueued on copy_stream.
+void stage_rows(prng_s *h, uint64_t k0, uint64_t nrows, uint64_t Wv, uint32_t *dst,
+                uint64_t dpitch) {
+    if (nrows == 0 || Wv == 0) return;
+    const uint64_t chunk_words = h->chunk_bytes / 4;
+    uint64_t rows_per, walkers_per;
+    if (Wv <= chunk_words) {
+        walkers_per = Wv;
+        rows_per = std::max<uint64_t>(1, chunk_words / Wv);
+    } else {
+        walkers_per = chunk_words;
+        rows_per = 1;
+    }
+    for (uint64_t r = 0; r < nrows; r += rows_per) {
+        const uint32_t nr = (uint32_t)std::min<uint64_t>(rows_per, nrows - r);
+        for (uint64_t wa = 0; wa < Wv; wa += walkers_per) {
+            const uint64_t wb = std::min<uint64_t>(Wv, wa + walkers_per);
+            const int b = h->chunk_next;
+            h->chunk_next = (b + 1) % prng_s::kChunks;
+            CK(cudaEventSynchronize(h->chunk_done[b]));  // pinned chunk free again
+            feed_chunk(h, wa, wb, k0 + r, nr, h->chunk[b]);
+            const uint64_t cw = wb - wa;
+            CK(cudaMemcpy2DAsync(dst + r * dpitch + wa, dpitch * 4, h->chunk[b], cw * 4, cw * 4,
+                                 nr, cudaMemcpyHostToDevice, h->copy_stream));
+            CK(cudaEventRecord(h->chunk_done[b], h->copy_stream));
+            h->stats.h2d_bytes += (uint64_t)nr * cw * 4;
+        }
+    }
+}
+
+// Make `s` wait for everything enqueued so far on copy_stream.
+void join_copies(prng_s *h, cudaStream_t s) {
+    CK(cudaEventRecord(h->ev_tmp, h->copy_stream));
+    CK(cudaStreamWaitEvent(s, h->ev_tmp, 0));
+}
+
+void ensure_dev(uint32_t *&p, size_t &cap, size_t bytes) {
+    if (bytes <= cap && p) return;
+    if (p) CK(cudaFree(p));
+    p = nullptr;
+    cap = 0;
+    CK(cudaMalloc(&p, bytes));
+    cap = bytes;
+}
+
+uint64_t labels_of(const prng_s *h, uint64_t n, int fmt) {
+    if (fmt == PRNG_FMT_U64) return n;
+    return (h->g.m <= 65536ull) ? n : n / 2;
+}
+
+int check_fmt(const prng_s *h, uint64_t n, int fmt) {
+    if (fmt != PRNG_FMT_U64 && fmt != PRNG_FMT_U32) return PRNG_E_INVALID;
+    if (fmt == PRNG_FMT_U32 && h->g.m > 65536ull && (n & 1)) return PRNG_E_INVALID;
+    return PRNG_OK;
+}
+
+gg::FillArgs fill_args(prng_s *h, const uint32_t *bits, uint64_t pitch, uint64_t Jw, uint64_t ja,
+                       uint64_t jb, uint64_t N, uint64_t nl, uint64_t g_origin, void *out,
+                       int out_u32) {
+    gg::FillArgs a{};
+    a.bits = bits;
+    a.pitch = pitch;
+    a.Jw = (uint32_t)Jw;
+    a.ja = (uint32_t)ja;
+    a.jb = (uint32_t)jb;
+    a.W = (uint32_t)h->W;
+    a.N = N;
+    a.nl = nl;
+    a.g_origin = g_origin;
+    a.x = h->x;
+    a.y = h->y;
+    a.out = out;
+    a.out_u32 = out_u32;
+    a.l = h->g.walk_len;
+    a.R = h->R;
+    a.m = h->g.m;
+    a.log2m = h->log2m;
+    a.pow2 = h->pow2;
+    return a;
+}
+
+// Core of prng_fill / prng_fill_host: draws [jlo, jhi) covering labels
+// [N, N+nl).  emit(ja, jb, bits, pitch, Jw) launches the walk for one piece.
+template <class Emit>
+void run_pieces(prng_s *h, uint64_t N, uint64_t nl, cudaStream_t s, Emit emit) {
+    const uint64_t W = h->W;
+    const uint64_t jlo = N / W, jhi = (N + nl + W - 1) / W;
+    const uint64_t Ds = std::max<uint32_t>(1, h->o.epoch_draws);
+    const uint64_t pitch = h->pitch();
+    uint64_t j = jlo;
+    while (j < jhi) {
+        if (h->res_bits && j >= h->res_J && j < h->res_J + h->res_D) {
+            const uint64_t jb = std::min(jhi, h->res_J + h->res_D);
+            emit(j, jb, h->res_bits, pitch, h->res_J, s);
+            j = jb;
+            continue;
+        }
+        uint64_t jb = std::min(jhi, j + Ds);
+        if (h->res_bits && h->res_J > j && h->res_J < jb) jb = h->res_J;
+        const int slot = h->ring_next;
+        h->ring_next ^= 1;
+        const size_t rbytes = (size_t)Ds * h->R * pitch * 4;
+        if (h->ring_cap < rbytes) {
+            CK(cudaDeviceSynchronize());
+            for (auto &p : h->ring) {
+                if (p) CK(cudaFree(p));
+                p = nullptr;
+            }
+            h->ring_cap = 0;
+            for (auto &p : h->ring) CK(cudaMalloc(&p, rbytes));
+            h->ring_cap = rbytes;
+        }
+        CK(cudaStreamWaitEvent(h->copy_stream, h->ring_free[slot], 0));  // slot no longer read
+        stage_rows(h, 2 + h->R0 + h->R * j, (jb - j) * h->R, W, h->ring[slot], pitch);
+        join_copies(h, s);
+        emit(j, jb, h->ring[slot], pitch, j, s);
+        CK(cudaEventRecord(h->ring_free[slot], s));
+        j = jb;
+    }
+}
+
+int guard(prng_s *h, const std::function<int()> &fn) {
+    if (!h) return PRNG_E_INVALID;
+    if (h->poisoned) return PRNG_E_STATE;
+    try {
+        CK(cudaSetDevice(h->o.device));
+        return fn();
+    } catch (const CudaFail &f) {
+        fprintf(stderr, "[ggprng] CUDA error: %s\n", cudaGetErrorString(f.e));
+        h->poisoned = true;
+        return PRNG_E_CUDA;
+    } catch (const std::bad_alloc &) {
+        return PRNG_E_NOMEM;
+    }
+}
+
+}  // namespace
+
+extern "C" {
+
+int prng_version(void) { return 100; }
+
+const char *prng_strerror(int status) {
+    switch (status) {
+        case PRNG_OK: return "ok";
+        case PRNG_E_INVALID: return "invalid argument";
+        case PRNG_E_UNSUPPORTED: return "unsupported parameters";
+        case PRNG_E_NOMEM: return "out of memory";
+        case PRNG_E_CUDA: return "CUDA error (handle poisoned)";
+        case PRNG_E_OVERRUN: return "on-demand draw outside the epoch window";
+        case PRNG_E_STATE: return "call not allowed in the current state";
+        default: return "unknown status";
+    }
+}
+
+int prng_default_params(prng_graph_params *p) {
+    if (!p) return PRNG_E_INVALID;
+    p->m = 1ull << 32;
+    p->degree = 7;
+    p->walk_len = 64;
+    p->burnin_len = 64;
+    p->variant = 0;
+    return PRNG_OK;
+}
+
+int prng_default_options(prng_options *o) {
+    if (!o) return PRNG_E_INVALID;
+    memset(o, 0, sizeof(*o));
+    o->device = 0;
+    o->walker_base = 0;
+    o->epoch_draws = 16;
+    o->host_threads = 0;
+    o->bit_source = PRNG_BITS_SPLITMIX;
+    return PRNG_OK;
+}
+
+int prng_create(prng_t **out, const prng_graph_params *g, uint64_t walkers, uint64_t seed,
+                const prng_options *opt) {
+    if (!out || !g) return PRNG_E_INVALID;
+    *out = nullptr;
+    if (walkers == 0) return PRNG_E_INVALID;
+    prng_options o;
+    if (opt)
+        o = *opt;
+    else
+        prng_default_options(&o);
+    if (g->degree != 7 || g->variant != 0) return PRNG_E_UNSUPPORTED;
+    if (g->m < 2 || g->m > (1ull << 32)) return PRNG_E_INVALID;
+    const bool pow2 = (g->m & (g->m - 1)) == 0;
+    if (!pow2 && g->m > (1ull << 30)) return PRNG_E_UNSUPPORTED;
+    if (g->walk_len < 1 || g->walk_len > 4096 || g->burnin_len > 4096) return PRNG_E_INVALID;
+    if (walkers + o.walker_base > (1ull << 24)) return PRNG_E_INVALID;
+    if (o.bit_source != PRNG_BITS_SPLITMIX && o.bit_source != PRNG_BITS_CALLBACK)
+        return PRNG_E_INVALID;
+    if (o.bit_source == PRNG_BITS_CALLBACK && !o.bits_fn) return PRNG_E_INVALID;
+    if (o.epoch_draws == 0) o.epoch_draws = 16;
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || o.device < 0 || o.device >= ndev)
+        return PRNG_E_INVALID;
+
+    prng_s *h = new (std::nothrow) prng_s();
+    if (!h) return PRNG_E_NOMEM;
+    h->g = *g;
+    h->o = o;
+    h->W = walkers;
+    h->seed = seed;
+    h->R = words_per_walk(g->walk_len);
+    h->R0 = words_per_walk(g->burnin_len);
+    h->pow2 = pow2 ? 1 : 0;
+    h->log2m = 0;
+    if (pow2)
+        while ((1ull << h->log2m) < g->m) h->log2m++;
+    try {
+        CK(cudaSetDevice(o.device));
+        CK(cudaDeviceGetAttribute(&h->sm_count, cudaDevAttrMultiProcessorCount, o.device));
+        unsigned nt = o.host_threads ? o.host_threads : std::thread::hardware_concurrency();
+        if (nt == 0) nt = 1;
+        h->pool = new ThreadPool(nt);
+        CK(cudaStreamCreateWithFlags(&h->copy_stream, cudaStreamNonBlocking));
+        CK(cudaStreamCreateWithFlags(&h->d2h_stream, cudaStreamNonBlocking));
+        CK(cudaStreamCreateWithFlags(&h->work_stream, cudaStreamNonBlocking));
+        CK(cudaEventCreateWithFlags(&h->ev_tmp, cudaEventDisableTiming));
+        h->chunk_bytes = 32ull << 20;
+        for (int i = 0; i < prng_s::kChunks; i++) {
+            CK(cudaHostAlloc((void **)&h->chunk[i], h->chunk_bytes, cudaHostAllocPortable));
+            CK(cudaEventCreateWithFlags(&h->chunk_done[i], cudaEventDisableTiming));
+        }
+        for (int i = 0; i < 2; i++) {
+            CK(cudaEventCreateWithFlags(&h->ring_free[i], cudaEventDisableTiming));
+            CK(cudaEventCreateWithFlags(&h->hout_free[i], cudaEventDisableTiming));
+        }
+        const size_t sb = (size_t)walkers * 4;
+        for (uint32_t **p : {&h->x, &h->y, &h->j, &h->xs, &h->ys, &h->js}) CK(cudaMalloc(p, sb));
+        CK(cudaMalloc(&h->flags, 4));
+        CK(cudaMemset(h->flags, 0, 4));
+        // Alg.1, in walker chunks to bound the temporary window.
+        const uint64_t chunkW = std::min<uint64_t>(walkers, 1ull << 22);
+        const uint64_t cpitch = round_up(chunkW, 32);
+        uint32_t *tmp = nullptr;
+        size_t tmp_cap = 0;
+        ensure_dev(tmp, tmp_cap, (size_t)(2 + h->R0) * cpitch * 4);
+        for (uint64_t w0 = 0; w0 < walkers; w0 += chunkW) {
+            const uint64_t cnt = std::min<uint64_t>(chunkW, walkers - w0);
+            // stage_rows works on walkers [0, Wv) of the handle; shift the base.
+            const uint64_t saved_base = h->o.walker_base;
+            h->o.walker_base = saved_base + w0;
+            stage_rows(h, 0, 2 + h->R0, cnt, tmp, cpitch);
+            h->o.walker_base = saved_base;
+            join_copies(h, h->work_stream);
+            gg::InitArgs a{};
+            a.bits = tmp;
+            a.pitch = cpitch;
+            a.w0 = (uint32_t)w0;
+            a.count = (uint32_t)cnt;
+            a.l0 = g->burnin_len;
+            a.R0 = h->R0;
+            a.m = g->m;
+            a.log2m = h->log2m;
+            a.pow2 = h->pow2;
+            a.x = h->x;
+            a.y = h->y;
+            a.j = h->j;
+            CK(gg::launch_init(a, h->work_stream));
+            h->stats.kernel_launches++;
+            CK(cudaStreamSynchronize(h->work_stream));
+        }
+        CK(cudaFree(tmp));
+        CK(cudaDeviceSynchronize());
+    } catch (const CudaFail &f) {
+        fprintf(stderr, "[ggprng] CUDA error in prng_create: %s\n", cudaGetErrorString(f.e));
+        free_all(h);
+        delete h;
+        return (f.e == cudaErrorMemoryAllocation) ? PRNG_E_NOMEM : PRNG_E_CUDA;
+    } catch (const std::bad_alloc &) {
+        free_all(h);
+        delete h;
+        return PRNG_E_NOMEM;
+    }
+    *out = h;
+    return PRNG_OK;
+}
+
+int prng_fill(prng_t *h, void *dev_ptr, uint64_t n, int fmt, void *stream) {
+    if (!h) return PRNG_E_INVALID;
+    int rc = check_fmt(h, n, fmt);
+    if (rc != PRNG_OK) return rc;
+    if (n == 0) return PRNG_OK;
+    if (!dev_ptr || ((uintptr_t)dev_ptr % (fmt == PRNG_FMT_U64 ? 8 : 4))) return PRNG_E_INVALID;
+    if (h->od_open) return PRNG_E_STATE;
+    return guard(h, [&] {
+        cudaStream_t s = (cudaStream_t)stream;
+        const uint64_t nl = labels_of(h, n, fmt);
+        const int out_u32 = (fmt == PRNG_FMT_U32 && h->g.m <= 65536ull) ? 1 : 0;
+        const uint64_t N = h->N;
+        run_pieces(h, N, nl, s,
+                   [&](uint64_t ja, uint64_t jb, const uint32_t *bits, uint64_t pitch, uint64_t Jw,
+                       cudaStream_t st) {
+                       gg::FillArgs a =
+                           fill_args(h, bits, pitch, Jw, ja, jb, N, nl, N, dev_ptr, out_u32);
+                       CK(gg::launch_fill(a, st, h->sm_count));
+                       h->stats.kernel_launches++;
+                   });
+        h->N = N + nl;
+        h->stats.labels_generated += nl;
+        return PRNG_OK;
+    });
+}
+
+int prng_fill_host(prng_t *h, void *host_ptr, uint64_t n, int fmt) {
+    if (!h) return PRNG_E_INVALID;
+    int rc = check_fmt(h, n, fmt);
+    if (rc != PRNG_OK) return rc;
+    if (n == 0) return PRNG_OK;
+    if (!host_ptr) return PRNG_E_INVALID;
+    if (h->od_open) return PRNG_E_STATE;
+    return guard(h, [&] {
+        const uint64_t nl = labels_of(h, n, fmt);
+        const int out_u32 = (fmt == PRNG_FMT_U32 && h->g.m <= 65536ull) ? 1 : 0;
+        const size_t esz = out_u32 ? 4 : 8;
+        const uint64_t N = h->N;
+        const uint64_t Ds = std::max<uint32_t>(1, h->o.epoch_draws);
+        const size_t need = (size_t)(Ds + 1) * h->W * esz;
+        if (h->hout_cap < need) {
+            for (auto &p : h->hout)
+                if (p) {
+                    CK(cudaFree(p));
+                    p = nullptr;
+                }
+            for (auto &p : h->hout) CK(cudaMalloc(&p, need));
+            h->hout_cap = need;
+        }
+        int oslot = 0;
+        char *dst = (char *)host_ptr;
+        cudaStream_t s = h->work_stream;
+        run_pieces(h, N, nl, s,
+                   [&](uint64_t ja, uint64_t jb, const uint32_t *bits, uint64_t pitch, uint64_t Jw,
+                       cudaStream_t st) {
+                       // a resident window may span many ring slots' worth: split
+                       for (uint64_t a0 = ja; a0 < jb; a0 += Ds) {
+                           const uint64_t a1 = std::min(jb, a0 + Ds);
+                           const uint64_t gA = std::max(N, a0 * h->W);
+                           const uint64_t gB = std::min(N + nl, a1 * h->W);
+                           if (gB <= gA) continue;
+                           CK(cudaStreamWaitEvent(st, h->hout_free[oslot], 0));
+                           gg::FillArgs a = fill_args(h, bits, pitch, Jw, a0, a1, N, nl, gA,
+                                                      h->hout[oslot], out_u32);
+                           CK(gg::launch_fill(a, st, h->sm_count));
+                           h->stats.kernel_launches++;
+                           CK(cudaEventRecord(h->ev_tmp, st));
+                           CK(cudaStreamWaitEvent(h->d2h_stream, h->ev_tmp, 0));
+                           CK(cudaMemcpyAsync(dst + (gA - N) * esz, h->hout[oslot],
+                                              (gB - gA) * esz, cudaMemcpyDeviceToHost,
+                                              h->d2h_stream));
+                           CK(cudaEventRecord(h->hout_free[oslot], h->d2h_stream));
+                           h->stats.d2h_bytes += (gB - gA) * esz;
+                           oslot ^= 1;
+                       }
+                   });
+        CK(cudaStreamSynchronize(h->d2h_stream));
+        CK(cudaStreamSynchronize(s));
+        h->N = N + nl;
+        h->stats.labels_generated += nl;
+        return PRNG_OK;
+    });
+}
+
+int prng_prefetch(prng_t *h, uint64_t draws) {
+    if (!h) return PRNG_E_INVALID;
+    if (draws == 0) return PRNG_E_INVALID;
+    if (h->od_open) return PRNG_E_STATE;
+    return guard(h, [&] {
+        const uint64_t pitch = h->pitch();
+        const size_t bytes = (size_t)draws * h->R * pitch * 4;
+        CK(cudaDeviceSynchronize());  // the old window may still be read
+        ensure_dev(h->res_bits, h->res_cap, bytes);
+        const uint64_t J = h->N / h->W;
+        stage_rows(h, 2 + h->R0 + h->R * J, draws * h->R, h->W, h->res_bits, pitch);
+        CK(cudaStreamSynchronize(h->copy_stream));
+        h->res_J = J;
+        h->res_D = draws;
+        return PRNG_OK;
+    });
+}
+
+int prng_tell(prng_t *h, uint64_t *n_out) {
+    if (!h || !n_out) return PRNG_E_INVALID;
+    *n_out = h->N;
+    return PRNG_OK;
+}
+
+int prng_mark(prng_t *h, void *stream) {
+    if (!h) return PRNG_E_INVALID;
+    return guard(h, [&] {
+        cudaStream_t s = (cudaStream_t)stream;
+        const size_t sb = h->W * 4;
+        CK(cudaMemcpyAsync(h->xs, h->x, sb, cudaMemcpyDeviceToDevice, s));
+        CK(cudaMemcpyAsync(h->ys, h->y, sb, cudaMemcpyDeviceToDevice, s));
+        CK(cudaMemcpyAsync(h->js, h->j, sb, cudaMemcpyDeviceToDevice, s));
+        h->N_mark = h->N;
+        h->od_J0_mark = h->od_J0;
+        h->od_started_mark = h->od_started;
+        h->have_mark = true;
+        return PRNG_OK;
+    });
+}
+
+int prng_rewind(prng_t *h, void *stream) {
+    if (!h) return PRNG_E_INVALID;
+    if (!h->have_mark || h->od_open) return PRNG_E_STATE;
+    return guard(h, [&] {
+        cudaStream_t s = (cudaStream_t)stream;
+        const size_t sb = h->W * 4;
+        CK(cudaMemcpyAsync(h->x, h->xs, sb, cudaMemcpyDeviceToDevice, s));
+        CK(cudaMemcpyAsync(h->y, h->ys, sb, cudaMemcpyDeviceToDevice, s));
+        CK(cudaMemcpyAsync(h->j, h->js, sb, cudaMemcpyDeviceToDevice, s));
+        h->N = h->N_mark;
+        h->od_J0 = h->od_J0_mark;
+        h->od_started = h->od_started_mark;
+        return PRNG_OK;
+    });
+}
+
+namespace {
+struct SavedHeader {
+    uint64_t magic, W, N, od_J0, od_started, m, seed, walk_len;
+};
+const uint64_t kMagic = 0x47475052'4e470001ull;
+}  // namespace
+
+int prng_state_size(prng_t *h, size_t *bytes) {
+    if (!h || !bytes) return PRNG_E_INVALID;
+    *bytes = sizeof(SavedHeader) + 3 * h->W * 4;
+    return PRNG_OK;
+}
+
+int prng_save(prng_t *h, void *host_buf, size_t bytes) {
+    if (!h || !host_buf || bytes < sizeof(SavedHeader) + 3 * h->W * 4) return PRNG_E_INVALID;
+    if (h->od_open) return PRNG_E_STATE;
+    return guard(h, [&] {
+        SavedHeader hd{kMagic, h->W, h->N, h->od_J0, h->od_started ? 1ull : 0ull, h->g.m, h->seed,
+                       h->g.walk_len};
+        CK(cudaDeviceSynchronize());
+        memcpy(host_buf, &hd, sizeof(hd));
+        char *p = (char *)host_buf + sizeof(hd);
+        CK(cudaMemcpy(p, h->x, h->W * 4, cudaMemcpyDeviceToHost));
+        CK(cudaMemcpy(p + h->W * 4, h->y, h->W * 4, cudaMemcpyDeviceToHost));
+        CK(cudaMemcpy(p + 2 * h->W * 4, h->j, h->W * 4, cudaMemcpyDeviceToHost));
+        return PRNG_OK;
+    });
+}
+
+int prng_load(prng_t *h, const void *host_buf, size_t bytes) {
+    if (!h || !host_buf || bytes < sizeof(SavedHeader) + 3 * h->W * 4) return PRNG_E_INVALID;
+    SavedHeader hd;
+    memcpy(&hd, host_buf, sizeof(hd));
+    if (hd.magic != kMagic || hd.W != h->W || hd.m != h->g.m || hd.seed != h->seed ||
+        hd.walk_len != h->g.walk_len)
+        return PRNG_E_INVALID;
+    if (h->od_open) return PRNG_E_STATE;
+    return guard(h, [&] {
+        CK(cudaDeviceSynchronize());
+        const char *p = (const char *)host_buf + sizeof(hd);
+        CK(cudaMemcpy(h->x, p, h->W * 4, cudaMemcpyHostToDevice));
+        CK(cudaMemcpy(h->y, p + h->W * 4, h->W * 4, cudaMemcpyHostToDevice));
+        CK(cudaMemcpy(h->j, p + 2 * h->W * 4, h->W * 4, cudaMemcpyHostToDevice));
+        h->N = hd.N;
+        h->od_J0 = hd.od_J0;
+        h->od_started = hd.od_started != 0;
+        return PRNG_OK;
+    });
+}
+
+int prng_epoch_begin(prng_t *h, uint64_t active_walkers, uint32_t draws, void *stream) {
+    if (!h) return PRNG_E_INVALID;
+    if (active_walkers == 0 || active_walkers > h->W || draws == 0) return PRNG_E_INVALID;
+    if (h->od_open) return PRNG_E_STATE;
+    return guard(h, [&] {
+        cudaStream_t s = (cudaStream_t)stream;
+        const uint64_t J0 = h->od_started ? h->od_J0 : (h->N + h->W - 1) / h->W;
+        if (J0 + draws > 0xFFFFFFFFull) return PRNG_E_UNSUPPORTED;
+        const uint64_t pitch = round_up(active_walkers, 32);
+        const size_t bytes = (size_t)draws * h->R * pitch * 4;
+        if (bytes > h->od_cap) {
+            CK(cudaDeviceSynchronize());
+            ensure_dev(h->od_bits, h->od_cap, bytes);
+        } else {
+            // the previous epoch's kernels must be done reading the window
+            CK(cudaEventRecord(h->ev_tmp, s));
+            CK(cudaStreamWaitEvent(h->copy_stream, h->ev_tmp, 0));
+        }
+        stage_rows(h, 2 + h->R0 + h->R * J0, (uint64_t)draws * h->R, active_walkers, h->od_bits,
+                   pitch);
+        join_copies(h, s);
+        h->od_J0 = J0;
+        h->od_D = draws;
+        h->od_Wv = active_walkers;
+        h->od_pitch = pitch;
+        h->od_open = true;
+        h->od_started = true;
+        return PRNG_OK;
+    });
+}
+
+int prng_epoch_end(prng_t *h, void *stream) {
+    (void)stream;
+    if (!h) return PRNG_E_INVALID;
+    if (!h->od_open) return PRNG_E_STATE;
+    h->od_J0 += h->od_D;
+    h->od_open = false;
+    h->N = h->od_J0 * h->W;  // a later bulk fill starts with every walker at draw J0
+    return PRNG_OK;
+}
+
+int prng_device_view(prng_t *h, void *view, size_t view_bytes) {
+    if (!h || !view || view_bytes != sizeof(prng_view)) return PRNG_E_INVALID;
+    if (!h->od_open) return PRNG_E_STATE;
+    prng_view v{};
+    v.bits = h->od_bits;
+    v.x = h->x;
+    v.y = h->y;
+    v.j = h->j;
+    v.flags = h->flags;
+    v.pitch = h->od_pitch;
+    v.m = h->g.m;
+    v.J0 = (uint32_t)h->od_J0;
+    v.D = h->od_D;
+    v.Wv = (uint32_t)h->od_Wv;
+    v.R = h->R;
+    v.l = h->g.walk_len;
+    v.log2m = h->log2m;
+    v.pow2 = h->pow2;
+    memcpy(view, &v, sizeof(v));
+    return PRNG_OK;
+}
+
+int prng_check(prng_t *h) {
+    if (!h) return PRNG_E_INVALID;
+    return guard(h, [&] {
+        uint32_t f = 0;
+        CK(cudaDeviceSynchronize());
+        CK(cudaMemcpy(&f, h->flags, 4, cudaMemcpyDeviceToHost));
+        if (f) {
+            CK(cudaMemset(h->flags, 0, 4));
+            return PRNG_E_OVERRUN;
+        }
+        return PRNG_OK;
+    });
+}
+
+int prng_get_stats(prng_t *h, prng_stats *s) {
+    if (!h || !s) return PRNG_E_INVALID;
+    *s = h->stats;
+    return PRNG_OK;
+}
+
+int prng_destroy(prng_t *h) {
+    if (!h) return PRNG_OK;
+    free_all(h);
+    delete h;
+    return PRNG_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,112 @@
+"""On-demand prng_next (header-only device API) vs the oracle, bit-exact.
+
+Epoch rule R10: in an epoch with cursor J0 and depth D, the
+i-th prng_next of walker t returns draw J0 + i of walker t; draws a walker
+does not use are skipped at epoch end; a walker that sits out an epoch jumps
+to the next window.  A draw past the window returns 0 and sets the sticky
+overrun flag.
+"""
+import numpy as np
+import pytest
+
+import oracle as O
+
+pytestmark = pytest.mark.gpu
+M32 = 1 << 32
+
+
+class OracleWalker:
+    """Oracle replay of one walker under the epoch rule."""
+
+    def __init__(self, m, seed, t):
+        self.m, self.seed, self.t = m, seed, t
+        x, y = O.walker_init(m, 64, seed, t)
+        self.xy = np.array([x], np.uint64), np.array([y], np.uint64)
+
+    def draw(self, j):
+        lib = O.lib()
+        x, y = self.xy
+        lab = lib.or_walker_draw(self.m, 64, 64, self.seed, self.t, j, x.ctypes.data, y.ctypes.data)
+        return int(lab)
+
+
+def test_uniform_epochs_match_bulk_order():
+    import torch
+    from paper_conf_ipps_banerjeebk12_b200 import Generator
+    W, D, seed = 2048, 5, 21
+    g = Generator(walkers=W, seed=seed)
+    outs = []
+    for e in range(3):
+        g.epoch_begin(W, D)
+        o = torch.empty(W * D, dtype=torch.int64, device="cuda")
+        g.consume(W, uniform=D, out=o)
+        g.epoch_end()
+        outs.append(o.view(W, D).cpu().numpy().view(np.uint64))
+    assert g.check() == 0
+    for t in (0, 1, 777, W - 1):
+        seq = np.concatenate([o[t] for o in outs])
+        assert np.array_equal(seq, O.walker_draws(M32, 64, 64, seed, t, 0, 3 * D))
+
+
+def test_variable_demand_skips_and_active_subsets():
+    # LR-shaped demand: epoch 0 all walkers, varying counts; epoch 1 only
+    # walkers [0, 700) active; epoch 2 all again (walkers >= 700 sat out).
+    import torch
+    from paper_conf_ipps_banerjeebk12_b200 import Generator
+    W, D, seed = 1000, 4, 99
+    rng = np.random.default_rng(1)
+    g = Generator(walkers=W, seed=seed)
+    oracle = {t: OracleWalker(M32, seed, t) for t in (0, 3, 699, 700, 999)}
+    J0 = 0
+    for e, active in enumerate([W, 700, W]):
+        counts = rng.integers(0, D + 1, size=active).astype(np.uint32)
+        offs = np.concatenate([[0], np.cumsum(counts)[:-1]]).astype(np.uint64)
+        total = int(counts.sum())
+        g.epoch_begin(active, D)
+        o = torch.zeros(max(total, 1), dtype=torch.int64, device="cuda")
+        g.consume(active, counts=torch.from_numpy(counts).cuda(), out=o,
+                  offsets=torch.from_numpy(offs.view(np.int64)).cuda())
+        g.epoch_end()
+        z = o.cpu().numpy().view(np.uint64)
+        for t, ow in oracle.items():
+            if t >= active:
+                continue
+            for i in range(int(counts[t])):
+                assert int(z[offs[t] + i]) == ow.draw(J0 + i), (e, t, i)
+        J0 += D
+    assert g.check() == 0
+
+
+def test_overrun_sets_flag_and_returns_zero():
+    import torch
+    from paper_conf_ipps_banerjeebk12_b200 import Generator
+    from paper_conf_ipps_banerjeebk12_b200._lib import PRNG_E_OVERRUN
+    W, D = 256, 2
+    g = Generator(walkers=W, seed=4)
+    g.epoch_begin(W, D)
+    o = torch.empty(W * 3, dtype=torch.int64, device="cuda")
+    g.consume(W, uniform=3, out=o)
+    g.epoch_end()
+    z = o.view(W, 3).cpu().numpy().view(np.uint64)
+    assert np.all(z[:, 2] == 0) and np.all(z[:, :2] != 0)
+    assert g.check() == PRNG_E_OVERRUN
+    assert g.check() == 0  # read-and-clear
+    assert np.array_equal(z[5, :2], O.walker_draws(M32, 64, 64, 4, 5, 0, 2))
+
+
+def test_bulk_after_on_demand_realigns():
+    # After an epoch, a bulk fill continues with every walker at draw J0.
+    import torch
+    from paper_conf_ipps_banerjeebk12_b200 import Generator
+    W, seed = 512, 8
+    g = Generator(walkers=W, seed=seed)
+    g.epoch_begin(W, 2)
+    g.consume(W, uniform=1, xor_out=torch.empty(W, dtype=torch.int64, device="cuda"))
+    g.epoch_end()
+    o = torch.empty(W, dtype=torch.int64, device="cuda")
+    g.fill(o)
+    z = o.cpu().numpy().view(np.uint64)
+    for t in (0, 100, W - 1):
+        ow = OracleWalker(M32, seed, t)
+        ow.draw(0)  # the one used draw; draw 1 skipped
+        assert int(z[t]) == ow.draw(2)
