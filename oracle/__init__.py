@@ -81,7 +81,7 @@ def _bind_optional(L):
     """Signatures of the application oracles (list ranking, Monte Carlo)."""
     opt = {
         "or_lr_rank_seq": (ctypes.c_int, [i64, P, i64, P]),
-        "or_lr_run": (ctypes.c_int, [u64, u32, u32, u64, i64, P, P, i64, i64, P, P, P]),
+        "or_lr_run": (ctypes.c_int, [u64, u32, u32, u64, i64, P, P, i64, i64, P, P, P, P]),
         "or_mc_run": (ctypes.c_int, [P, P, P, P]),
     }
     for name, (res, args) in opt.items():
@@ -172,3 +172,32 @@ def stream_block(seed: int, t0: int, count: int, k0: int, nwords: int) -> np.nda
     out = np.empty((nwords, count), dtype=np.uint32)
     lib().or_stream_block(seed, t0, count, k0, nwords, _ptr(out))
     return out
+
+
+def lr_rank_seq(succ, head: int) -> np.ndarray:
+    """Ranks by walking the list from the head (the definition, R17)."""
+    succ = np.ascontiguousarray(succ, dtype=np.int32)
+    rank = np.full(succ.size, -1, dtype=np.int32)
+    reached = lib().or_lr_rank_seq(succ.size, _ptr(succ), head, _ptr(rank))
+    if reached != succ.size:
+        raise ValueError("not a single list")
+    return rank
+
+
+def lr_run(succ, pred, head: int, seed: int, m: int = 1 << 32, l: int = 64, l0: int = 64,
+           max_rounds: int = 1000):
+    """Sequential replica of Alg.3 + Helman-JaJa + re-insertion (lr_oracle.c)."""
+    succ = np.ascontiguousarray(succ, dtype=np.int32)
+    pred = np.ascontiguousarray(pred, dtype=np.int32)
+    n = succ.size
+    rank = np.full(n, -1, dtype=np.int32)
+    removed = np.empty(n, dtype=np.int32)
+    spl = np.empty(n, dtype=np.int32)
+    info = np.zeros(4, dtype=np.int64)
+    rc = lib().or_lr_run(m, l, l0, seed, n, _ptr(succ), _ptr(pred), head, max_rounds,
+                         _ptr(rank), _ptr(removed), _ptr(spl), _ptr(info))
+    if rc != 0:
+        raise MemoryError("or_lr_run")
+    return {"rank": rank, "removed_round": removed, "is_splitter": spl.astype(bool),
+            "rounds": int(info[0]), "reduced": int(info[1]), "splitters": int(info[2]),
+            "draws": int(info[3])}
