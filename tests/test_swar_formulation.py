@@ -1,0 +1,66 @@
+"""Host-side check of the kernel's SWAR step formulation (no GPU).
+
+gg_walk64 (include/prng_device.cuh) does not evaluate the Gabber-Galil step
+the way the paper writes it; it repacks the 192-bit record into 10-field
+words, derives move masks and constants with word-parallel logic and uses
+u = x + y + c so that either move is one add.  This test re-expresses that
+exact instruction-level recipe in Python (32-bit wrap-around, the same
+shifts, masks and multiply-high) and checks it against the oracle's plain
+step-by-step walk on random records — including the masking bug class where
+garbage bits of MY leak into C.  The GPU parity tests then check that the
+CUDA code implements this recipe.
+"""
+import numpy as np
+
+import oracle as O
+
+M = 0xFFFFFFFF
+
+
+def _word10(Q, nk, x, y):
+    f1, f2 = Q >> 1, Q >> 2
+    MY = (~f2 & (f1 | Q)) & M
+    MX = (f2 & ~(f1 & Q)) & M
+    C = (Q - (MY & 0x09249249)) & M
+    for k in range(nk):
+        py, px = MY & (1 << 3 * k), MX & (1 << 3 * k)
+        ct = (C << (30 - 3 * k)) & M          # IMAD.SHL
+        c = (ct * 4) >> 32                   # IMAD.HI with c_mul = 4
+        u = (x + y + c) & M
+        if py:
+            y = (u + x) & M
+        if px:
+            x = (u + y) & M
+    return x, y
+
+
+def _fsr(lo, hi, s):
+    return ((hi << 32 | lo) >> s) & M
+
+
+def walk64_swar(w, x, y):
+    x, y = _word10(w[0], 10, x, y)
+    for a, s in [(0, 30), (1, 28), (2, 26), (3, 24), (4, 22)]:
+        x, y = _word10(_fsr(w[a], w[a + 1], s), 10, x, y)
+    return _word10(w[5] >> 20, 4, x, y)
+
+
+def test_swar_recipe_equals_definition_random():
+    rng = np.random.default_rng(2024)
+    for _ in range(2000):
+        w = [int(v) for v in rng.integers(0, 2 ** 32, 6, dtype=np.uint64)]
+        x0, y0 = (int(v) for v in rng.integers(0, 2 ** 32, 2, dtype=np.uint64))
+        assert walk64_swar(w, x0, y0) == O.walk(1 << 32, x0, y0, np.array(w, np.uint32), 64)
+
+
+def test_swar_recipe_every_field_value_at_every_position():
+    # each 3-bit value 0..7 at each of the 64 field positions, others random
+    rng = np.random.default_rng(5)
+    for i in range(64):
+        for b in range(8):
+            bits = int.from_bytes(rng.bytes(24), "little")
+            bits &= ~(7 << (3 * i))
+            bits |= b << (3 * i)
+            w = [(bits >> (32 * r)) & M for r in range(6)]
+            x0, y0 = (int(v) for v in rng.integers(0, 2 ** 32, 2, dtype=np.uint64))
+            assert walk64_swar(w, x0, y0) == O.walk(1 << 32, x0, y0, np.array(w, np.uint32), 64)
