@@ -39,7 +39,7 @@ struct prng_view {
     uint32_t l;            /* steps per number */
     uint32_t log2m;        /* log2(m) if m is a power of two, else 0 */
     uint32_t pow2;         /* 1 if m is a power of two */
-    uint32_t c_mul;        /* = 4 (see gg_step_swar); set by prng_device_view */
+    uint32_t _pad;
 };
 
 struct prng_state {
@@ -61,71 +61,68 @@ struct prng_state {
  *   MY = fields in {1,2,3}, MX = fields in {4,5,6} (bit at the field's LSB),
  *   C  = field - [y-move], whose low two bits are the step's constant c.
  * With u = x + y + c both moves are one add:  y-move y' = u + x,
- * x-move x' = u + y.  Per step (7 SASS, 3 ALU-pipe + 4 FMA-pipe, which is
- * the split that fits sm_100a: the ALU pipe issues every other cycle, the
- * FMA pipe every cycle):
- *   LOP3.P py, LOP3.P px          predicates from MY / MX           (ALU)
- *   IMAD.SHL ct = C << (30-3k)    c to the top two bits             (FMA)
- *   IMAD.IADD s = x + y; IMAD.HI u = hi(ct*4 + (s<<32)) = s + c     (FMA)
- *   @py y = u + x ; @px x = u + y                                   (ALU / FMA)
- * `c_mul` must be 4; it is passed opaquely (kernel argument / view field)
- * so that ptxas keeps the multiply-high on the FMA pipe instead of turning
- * it into an ALU shift.
+ * x-move x' = u + y.  Per step 7 SASS, which ptxas splits evenly between
+ * the ALU pipe and the FMA-heavy pipe (IMAD.*); on sm_100a each accepts a
+ * warp instruction every other cycle per SMSP, so a 50/50 split is what lets
+ * the scheduler issue every cycle:
+ *   LOP3.P py, LOP3.P px        predicates from MY / MX              (ALU)
+ *   IMAD.SHL ct = C << (30-3k)  c to the top two bits                (FMA)
+ *   s = x + y ; LEA.HI u = s + (ct >> 30)                            (FMA, ALU)
+ *   @py y = u + x ; @px x = u + y                                    (ALU / FMA)
  * ------------------------------------------------------------------------ */
 template <int K>
 __device__ __forceinline__ void gg_step_swar(uint32_t MY, uint32_t MX, uint32_t C,
-                                             uint32_t &x, uint32_t &y, uint32_t c_mul)
+                                             uint32_t &x, uint32_t &y)
 {
     asm volatile(
         "{\n\t"
         ".reg .pred py, px;\n\t"
-        ".reg .b32 ty, tx, ct, c, u;\n\t"
+        ".reg .b32 ty, tx, ct, c, s, u;\n\t"
         "and.b32 ty, %2, %5;\n\t"
         "setp.ne.b32 py, ty, 0;\n\t"
         "and.b32 tx, %3, %5;\n\t"
         "setp.ne.b32 px, tx, 0;\n\t"
         "shl.b32 ct, %4, %6;\n\t"
-        "mul.hi.u32 c, ct, %7;\n\t"
-        "add.u32 u, %0, %1;\n\t"
-        "add.u32 u, u, c;\n\t"
+        "shr.b32 c, ct, 30;\n\t"
+        "add.u32 s, %0, %1;\n\t"
+        "add.u32 u, s, c;\n\t"
         "@py add.u32 %1, u, %0;\n\t"
         "@px add.u32 %0, u, %1;\n\t"
         "}"
         : "+r"(x), "+r"(y)
-        : "r"(MY), "r"(MX), "r"(C), "n"(1u << (3 * K)), "n"(30 - 3 * K), "r"(c_mul));
+        : "r"(MY), "r"(MX), "r"(C), "n"(1u << (3 * K)), "n"(30 - 3 * K));
 }
 
 template <int NK>
-__device__ __forceinline__ void gg_word10(uint32_t Q, uint32_t &x, uint32_t &y, uint32_t c_mul)
+__device__ __forceinline__ void gg_word10(uint32_t Q, uint32_t &x, uint32_t &y)
 {
     const uint32_t f1 = Q >> 1, f2 = Q >> 2;
     const uint32_t MY = ~f2 & (f1 | Q);   /* b2=0 and b != 0 */
     const uint32_t MX = f2 & ~(f1 & Q);   /* b2=1 and b != 7 */
     /* y-move fields hold b-1 (no borrow: b>=1); MY is masked to the fields' LSBs */
     const uint32_t C = Q - (MY & 0x09249249u);
-    if (NK > 0) gg_step_swar<0>(MY, MX, C, x, y, c_mul);
-    if (NK > 1) gg_step_swar<1>(MY, MX, C, x, y, c_mul);
-    if (NK > 2) gg_step_swar<2>(MY, MX, C, x, y, c_mul);
-    if (NK > 3) gg_step_swar<3>(MY, MX, C, x, y, c_mul);
-    if (NK > 4) gg_step_swar<4>(MY, MX, C, x, y, c_mul);
-    if (NK > 5) gg_step_swar<5>(MY, MX, C, x, y, c_mul);
-    if (NK > 6) gg_step_swar<6>(MY, MX, C, x, y, c_mul);
-    if (NK > 7) gg_step_swar<7>(MY, MX, C, x, y, c_mul);
-    if (NK > 8) gg_step_swar<8>(MY, MX, C, x, y, c_mul);
-    if (NK > 9) gg_step_swar<9>(MY, MX, C, x, y, c_mul);
+    if (NK > 0) gg_step_swar<0>(MY, MX, C, x, y);
+    if (NK > 1) gg_step_swar<1>(MY, MX, C, x, y);
+    if (NK > 2) gg_step_swar<2>(MY, MX, C, x, y);
+    if (NK > 3) gg_step_swar<3>(MY, MX, C, x, y);
+    if (NK > 4) gg_step_swar<4>(MY, MX, C, x, y);
+    if (NK > 5) gg_step_swar<5>(MY, MX, C, x, y);
+    if (NK > 6) gg_step_swar<6>(MY, MX, C, x, y);
+    if (NK > 7) gg_step_swar<7>(MY, MX, C, x, y);
+    if (NK > 8) gg_step_swar<8>(MY, MX, C, x, y);
+    if (NK > 9) gg_step_swar<9>(MY, MX, C, x, y);
 }
 
 /* 64 steps from a 6-word record, m = 2^k (wrapped arithmetic). */
-__device__ __forceinline__ void gg_walk64(const uint32_t w[6], uint32_t &x, uint32_t &y,
-                                          uint32_t c_mul)
+__device__ __forceinline__ void gg_walk64(const uint32_t w[6], uint32_t &x, uint32_t &y)
 {
-    gg_word10<10>(w[0], x, y, c_mul);
-    gg_word10<10>(__funnelshift_r(w[0], w[1], 30), x, y, c_mul);
-    gg_word10<10>(__funnelshift_r(w[1], w[2], 28), x, y, c_mul);
-    gg_word10<10>(__funnelshift_r(w[2], w[3], 26), x, y, c_mul);
-    gg_word10<10>(__funnelshift_r(w[3], w[4], 24), x, y, c_mul);
-    gg_word10<10>(__funnelshift_r(w[4], w[5], 22), x, y, c_mul);
-    gg_word10<4>(w[5] >> 20, x, y, c_mul);
+    gg_word10<10>(w[0], x, y);
+    gg_word10<10>(__funnelshift_r(w[0], w[1], 30), x, y);
+    gg_word10<10>(__funnelshift_r(w[1], w[2], 28), x, y);
+    gg_word10<10>(__funnelshift_r(w[2], w[3], 26), x, y);
+    gg_word10<10>(__funnelshift_r(w[3], w[4], 24), x, y);
+    gg_word10<10>(__funnelshift_r(w[4], w[5], 22), x, y);
+    gg_word10<4>(w[5] >> 20, x, y);
 }
 
 /* One step, any m (generic path).  Non power-of-two m requires m <= 2^30 and
@@ -216,7 +213,7 @@ __device__ __forceinline__ uint64_t prng_next(prng_state *st, const prng_view *v
 #pragma unroll
         for (int r = 0; r < 6; r++)
             w[r] = __ldg(rec + (uint64_t)r * v->pitch);
-        gg_walk64(w, x, y, v->c_mul);
+        gg_walk64(w, x, y);
     } else {
         gg_walk_generic(rec, v->pitch, v->l, x, y, (uint32_t)v->m, v->pow2 != 0);
     }

@@ -153,6 +153,22 @@ class Generator:
         check(_lib.gg_consume(self._h, threads, ptr(counts), uniform, ptr(out), ptr(offsets),
                               ptr(xor_out), _stream_handle(stream)), "gg_consume")
 
+    def list_rank(self, succ, pred, head: int, removed_round=None, is_splitter=None, stream=None):
+        """gg_list_rank: ranks (distance from head) of a linked list given as CUDA int32 arrays.
+
+        Returns (rank tensor, info dict)."""
+        import torch
+        n = succ.numel()
+        rank = torch.empty(n, dtype=torch.int32, device=succ.device)
+        info = (ctypes.c_int64 * 8)()
+        ptr = lambda t: None if t is None else t.data_ptr()
+        check(_lib.gg_list_rank(self._h, n, succ.data_ptr(), pred.data_ptr(), head, rank.data_ptr(),
+                                ptr(removed_round), ptr(is_splitter), info, _stream_handle(stream)),
+              "gg_list_rank")
+        keys = ("rounds", "reduced", "splitters", "draws", "phase1_us", "phase2_us", "phase3_us",
+                "rounds2")
+        return rank, {k: info[i] for i, k in enumerate(keys)}
+
     def view(self) -> _lib.prng_view:
         v = _lib.prng_view()
         check(_lib.prng_device_view(self._h, ctypes.byref(v), ctypes.sizeof(v)), "prng_device_view")

@@ -59,7 +59,7 @@ class prng_view(ctypes.Structure):
     """Mirror of struct prng_view (include/prng_device.cuh)."""
     _fields_ = [("bits", vp), ("x", vp), ("y", vp), ("j", vp), ("flags", vp), ("pitch", u64),
                 ("m", u64), ("J0", u32), ("D", u32), ("Wv", u32), ("R", u32), ("l", u32),
-                ("log2m", u32), ("pow2", u32), ("c_mul", u32)]
+                ("log2m", u32), ("pow2", u32), ("_pad", u32)]
 
 
 _SIGS = {
@@ -86,6 +86,7 @@ _SIGS = {
     "prng_destroy": (c_int, [vp]),
     # include/gg_apps.h
     "gg_consume": (c_int, [vp, u64, vp, u32, vp, vp, vp, vp]),
+    "gg_list_rank": (c_int, [vp, ctypes.c_int64, vp, vp, ctypes.c_int64, vp, vp, vp, vp, vp]),
 }
 
 for _name, (_res, _args) in _SIGS.items():

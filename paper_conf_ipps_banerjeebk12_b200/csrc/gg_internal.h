@@ -20,7 +20,6 @@ struct InitArgs {
     uint64_t m;
     uint32_t log2m, pow2;
     uint32_t *x, *y, *j;
-    uint32_t c_mul;  // = 4, opaque to ptxas (see gg_step_swar)
 };
 cudaError_t launch_init(const InitArgs &a, cudaStream_t s);
 
@@ -42,7 +41,6 @@ struct FillArgs {
     uint32_t l, R;
     uint64_t m;
     uint32_t log2m, pow2;
-    uint32_t c_mul;  // = 4
 };
 cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count);
 

@@ -31,7 +31,7 @@ __global__ void __launch_bounds__(128) gg_init_kernel(InitArgs a) {
         uint32_t w[6];
 #pragma unroll
         for (int r = 0; r < 6; r++) w[r] = rec[(uint64_t)(2 + r) * a.pitch];
-        gg_walk64(w, x, y, a.c_mul);
+        gg_walk64(w, x, y);
     } else {
         gg_walk_generic(rec + 2 * a.pitch, a.pitch, a.l0, x, y, (uint32_t)a.m, a.pow2 != 0);
     }
@@ -86,7 +86,7 @@ __global__ void __launch_bounds__(64) gg_fill64_kernel(FillArgs a, uint32_t unit
 #pragma unroll
                 for (int r = 0; r < 6; r++) wn[r] = __ldg(rec + (uint64_t)r * a.pitch);
             }
-            gg_walk64(w, x, y, a.c_mul);
+            gg_walk64(w, x, y);
             const uint64_t lab = gg_label(x, y, a.m, a.log2m, true);
             const uint64_t g = (uint64_t)j * a.W + t;
             if (OUT32)

@@ -1,0 +1,311 @@
+// Randomised list ranking with on-demand random numbers (§V,
+// Alg.3 + Phases II/III of [3]).  C ABI: gg_list_rank (include/gg_apps.h).
+//
+// Phase I (Alg.3 ReduceList), one round per on-demand epoch:
+//   lr_draw   : active slot i (walker i) calls prng_next; b(u) = bit 63 (R13)
+//   lr_decide : u leaves iff b(u)=1, b(pred)=0, b(succ)=0, u not head/tail (R14)
+//   lr_splice : splice u out; remember (pred, distance) for Phase III
+//   cub::DevicePartition::Flagged : stable compaction of the survivors; the
+//               removed nodes of the round go to the re-insertion log
+//   repeat until active <= ceil(n / floor(log2 n)) (R15).  The host learns the
+//   new active count each round and the feed supplies exactly that many draws
+//   (on demand, instead of [3]'s upper-bound pre-generation).
+// Phase II (Helman-JaJa [10]): splitters = head + nodes whose next draw is
+//   < 2^64/64 (R18); each splitter walks its sublist (local offsets); suffix
+//   sums over the splitter chain by pointer jumping; rank = prefix + local.
+// Phase III: re-insert removed nodes in reverse round order,
+//   rank(u) = rank(pred at removal) + distance at removal.
+#include <cstdint>
+#include <vector>
+
+#include <cub/cub.cuh>
+#include <cuda_runtime.h>
+
+#include "gg_apps.h"
+#include "prng.h"
+#include "prng_device.cuh"
+
+namespace {
+
+struct Fail {
+    int rc;
+};
+#define LCK(call)                                              \
+    do {                                                       \
+        cudaError_t _e = (call);                               \
+        if (_e != cudaSuccess) throw Fail{PRNG_E_CUDA};        \
+    } while (0)
+#define LRC(call)                                              \
+    do {                                                       \
+        int _r = (call);                                       \
+        if (_r != PRNG_OK) throw Fail{_r};                     \
+    } while (0)
+
+__global__ void lr_init(int64_t n, int32_t *act, int32_t *w, int32_t *rr, int32_t *spl) {
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    act[i] = (int32_t)i;  // A_0 = node ids in order
+    w[i] = 1;             // links from i to succ(i)
+    if (rr) rr[i] = -1;
+    if (spl) spl[i] = 0;
+}
+
+__global__ void lr_find_tail(int64_t n, const int32_t *succ, int32_t *tail) {
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < n && succ[i] < 0) *tail = (int32_t)i;
+}
+
+// Alg.3 l.6-7: temp = getnextrand(); b(u) = bit 63 of temp.
+__global__ void __launch_bounds__(128) lr_draw(prng_view v, const int32_t *act, int64_t A,
+                                               uint8_t *bit) {
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= A) return;
+    prng_state st = prng_state_load(&v, (uint32_t)i);
+    const uint64_t z = prng_next(&st, &v);
+    prng_state_store(&v, &st);
+    bit[act[i]] = (uint8_t)(z >> 63);
+}
+
+// Alg.3 l.8-9 on the bits of this round (no list change yet).
+__global__ void lr_decide(const int32_t *act, int64_t A, const uint8_t *bit, const int32_t *pred,
+                          const int32_t *succ, int32_t head, int32_t tail, uint8_t *keep) {
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= A) return;
+    const int32_t u = act[i];
+    bool rm = false;
+    if (u != head && u != tail) rm = bit[u] && !bit[pred[u]] && !bit[succ[u]];
+    keep[i] = rm ? 0 : 1;
+}
+
+// Alg.3 l.10: remove with book-keeping.  No two removed nodes are adjacent,
+// so every written field has exactly one writer.
+__global__ void lr_splice(const int32_t *act, int64_t A, const uint8_t *keep, int32_t *pred,
+                          int32_t *succ, int32_t *w, int32_t *rem_pred, int32_t *rem_dist,
+                          int32_t *rr, int32_t round) {
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= A || keep[i]) return;
+    const int32_t u = act[i], p = pred[u], s = succ[u];
+    rem_pred[u] = p;
+    rem_dist[u] = w[p];
+    w[p] += w[u];
+    succ[p] = s;
+    pred[s] = p;
+    if (rr) rr[u] = round;
+}
+
+// Phase II splitter choice (R18).
+__global__ void __launch_bounds__(128) lr_splitter_draw(prng_view v, const int32_t *act, int64_t A,
+                                                        int32_t head, uint8_t *spl_node,
+                                                        uint8_t *spl_slot, int32_t *spl_out) {
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= A) return;
+    prng_state st = prng_state_load(&v, (uint32_t)i);
+    const uint64_t z = prng_next(&st, &v);
+    prng_state_store(&v, &st);
+    const int32_t u = act[i];
+    const uint8_t s = (u == head || (z >> 58) == 0) ? 1 : 0;
+    spl_node[u] = s;
+    spl_slot[i] = s;
+    if (spl_out) spl_out[u] = s;
+}
+
+__global__ void lr_splitter_index(const int32_t *spl, int64_t ns, int32_t *spl_idx) {
+    const int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (k < ns) spl_idx[spl[k]] = (int32_t)k;
+}
+
+// Sublist walk: splitter k follows succ to the next splitter.
+__global__ void lr_sublist(const int32_t *spl, int64_t ns, const int32_t *succ, const int32_t *w,
+                           const uint8_t *spl_node, const int32_t *spl_idx, int32_t *local,
+                           int32_t *sub, int32_t *len, int32_t *nextk) {
+    const int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (k >= ns) return;
+    int32_t v = spl[k], off = 0;
+    for (;;) {
+        local[v] = off;
+        sub[v] = (int32_t)k;
+        off += w[v];
+        const int32_t nx = succ[v];
+        if (nx < 0 || spl_node[nx]) {
+            len[k] = off;
+            nextk[k] = nx < 0 ? -1 : spl_idx[nx];
+            return;
+        }
+        v = nx;
+    }
+}
+
+// One pointer-jumping step of suffix sums over the splitter chain (Wyllie).
+__global__ void lr_jump(int64_t ns, const int32_t *val_in, const int32_t *nxt_in, int32_t *val_out,
+                        int32_t *nxt_out) {
+    const int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (k >= ns) return;
+    const int32_t nx = nxt_in[k];
+    if (nx >= 0) {
+        val_out[k] = val_in[k] + val_in[nx];
+        nxt_out[k] = nxt_in[nx];
+    } else {
+        val_out[k] = val_in[k];
+        nxt_out[k] = -1;
+    }
+}
+
+// rank = (total - suffix of own sublist) + local offset.
+__global__ void lr_fixup(const int32_t *act, int64_t A, const int32_t *sub, const int32_t *local,
+                         const int32_t *suffix, const int32_t *spl_idx, int32_t head,
+                         int32_t *rank) {
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= A) return;
+    const int32_t v = act[i];
+    const int32_t total = suffix[spl_idx[head]];
+    rank[v] = total - suffix[sub[v]] + local[v];
+}
+
+__global__ void lr_reinsert(const int32_t *list, int64_t cnt, const int32_t *rem_pred,
+                            const int32_t *rem_dist, int32_t *rank) {
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= cnt) return;
+    const int32_t u = list[i];
+    rank[u] = rank[rem_pred[u]] + rem_dist[u];
+}
+
+inline unsigned nblk(int64_t n, int t = 256) { return (unsigned)((n + t - 1) / t); }
+
+}  // namespace
+
+extern "C" int gg_list_rank(prng_t *h, int64_t n, const int32_t *succ, const int32_t *pred,
+                            int64_t head, int32_t *rank, int32_t *removed_round,
+                            int32_t *is_splitter, int64_t *info, void *stream) {
+    if (!h || n <= 0 || !succ || !pred || !rank || head < 0 || head >= n) return PRNG_E_INVALID;
+    if (n > (1ll << 24)) return PRNG_E_UNSUPPORTED;
+    cudaStream_t s = (cudaStream_t)stream;
+    std::vector<void *> bufs;
+    auto alloc = [&](size_t bytes) -> void * {
+        void *p = nullptr;
+        LCK(cudaMallocAsync(&p, bytes ? bytes : 1, s));
+        bufs.push_back(p);
+        return p;
+    };
+    int rc = PRNG_OK;
+    try {
+        cudaEvent_t ev[4];
+        for (auto &e : ev) LCK(cudaEventCreate(&e));
+        LCK(cudaEventRecord(ev[0], s));
+        const size_t n4 = (size_t)n * 4;
+        int32_t *d_succ = (int32_t *)alloc(n4), *d_pred = (int32_t *)alloc(n4);
+        int32_t *w = (int32_t *)alloc(n4), *rem_pred = (int32_t *)alloc(n4);
+        int32_t *rem_dist = (int32_t *)alloc(n4), *act = (int32_t *)alloc(n4);
+        int32_t *act2 = (int32_t *)alloc(n4), *rem_log = (int32_t *)alloc(n4);
+        uint8_t *bit = (uint8_t *)alloc(n), *keep = (uint8_t *)alloc(n);
+        int32_t *d_num = (int32_t *)alloc(8);
+        LCK(cudaMemcpyAsync(d_succ, succ, n4, cudaMemcpyDeviceToDevice, s));
+        LCK(cudaMemcpyAsync(d_pred, pred, n4, cudaMemcpyDeviceToDevice, s));
+        lr_init<<<nblk(n), 256, 0, s>>>(n, act, w, removed_round, is_splitter);
+        // the tail is the node whose succ is -1
+        LCK(cudaMemsetAsync(d_num, 0xFF, 8, s));
+        lr_find_tail<<<nblk(n), 256, 0, s>>>(n, d_succ, d_num + 1);
+        int32_t tail = -1;
+        LCK(cudaMemcpyAsync(&tail, d_num + 1, 4, cudaMemcpyDeviceToHost, s));
+        size_t tmp_bytes = 0;
+        LCK(cub::DevicePartition::Flagged(nullptr, tmp_bytes, act, keep, act2, d_num, (int)n, s));
+        size_t tmp2 = 0;
+        LCK(cub::DeviceSelect::Flagged(nullptr, tmp2, act, keep, act2, d_num, (int)n, s));
+        if (tmp2 > tmp_bytes) tmp_bytes = tmp2;
+        void *tmp = alloc(tmp_bytes);
+        LCK(cudaStreamSynchronize(s));
+        if (tail < 0) throw Fail{PRNG_E_INVALID};
+
+        int64_t L = 0;
+        while ((1ll << (L + 1)) <= n) L++;
+        if (L == 0) L = 1;
+        const int64_t target = (n + L - 1) / L;
+        int64_t A = n, rounds = 0, draws = 0, log_off = 0;
+        std::vector<int64_t> round_off, round_cnt;
+        prng_view view;
+        // ---------------- Phase I
+        while (A > target && rounds < 1000) {
+            LRC(prng_epoch_begin(h, (uint64_t)A, 1, s));
+            LRC(prng_device_view(h, &view, sizeof(view)));
+            lr_draw<<<nblk(A, 128), 128, 0, s>>>(view, act, A, bit);
+            LRC(prng_epoch_end(h, s));
+            draws += A;
+            lr_decide<<<nblk(A), 256, 0, s>>>(act, A, bit, d_pred, d_succ, (int32_t)head, tail, keep);
+            lr_splice<<<nblk(A), 256, 0, s>>>(act, A, keep, d_pred, d_succ, w, rem_pred, rem_dist,
+                                              removed_round, (int32_t)rounds);
+            LCK(cub::DevicePartition::Flagged(tmp, tmp_bytes, act, keep, act2, d_num, (int)A, s));
+            int32_t kept = 0;
+            LCK(cudaMemcpyAsync(&kept, d_num, 4, cudaMemcpyDeviceToHost, s));
+            LCK(cudaStreamSynchronize(s));
+            const int64_t gone = A - kept;
+            LCK(cudaMemcpyAsync(rem_log + log_off, act2 + kept, (size_t)gone * 4,
+                                cudaMemcpyDeviceToDevice, s));
+            round_off.push_back(log_off);
+            round_cnt.push_back(gone);
+            log_off += gone;
+            std::swap(act, act2);
+            A = kept;
+            rounds++;
+        }
+        LCK(cudaEventRecord(ev[1], s));
+        // ---------------- Phase II
+        uint8_t *spl_node = bit;  // reuse: bits of Phase I are dead
+        LRC(prng_epoch_begin(h, (uint64_t)A, 1, s));
+        LRC(prng_device_view(h, &view, sizeof(view)));
+        LCK(cudaMemsetAsync(spl_node, 0, n, s));
+        lr_splitter_draw<<<nblk(A, 128), 128, 0, s>>>(view, act, A, (int32_t)head, spl_node, keep,
+                                                      is_splitter);
+        LRC(prng_epoch_end(h, s));
+        draws += A;
+        LCK(cub::DeviceSelect::Flagged(tmp, tmp_bytes, act, keep, act2, d_num, (int)A, s));
+        int32_t ns = 0;
+        LCK(cudaMemcpyAsync(&ns, d_num, 4, cudaMemcpyDeviceToHost, s));
+        LCK(cudaStreamSynchronize(s));
+        int32_t *spl = act2;
+        int32_t *spl_idx = (int32_t *)alloc(n4);
+        int32_t *local = (int32_t *)alloc(n4), *sub = (int32_t *)alloc(n4);
+        int32_t *va = (int32_t *)alloc((size_t)ns * 4), *na = (int32_t *)alloc((size_t)ns * 4);
+        int32_t *vb = (int32_t *)alloc((size_t)ns * 4), *nb = (int32_t *)alloc((size_t)ns * 4);
+        lr_splitter_index<<<nblk(ns), 256, 0, s>>>(spl, ns, spl_idx);
+        lr_sublist<<<nblk(ns, 128), 128, 0, s>>>(spl, ns, d_succ, w, spl_node, spl_idx, local, sub,
+                                                va, na);
+        int iters = 0;
+        while ((1ll << iters) < (int64_t)ns) iters++;
+        for (int it = 0; it <= iters; it++) {
+            lr_jump<<<nblk(ns), 256, 0, s>>>(ns, va, na, vb, nb);
+            std::swap(va, vb);
+            std::swap(na, nb);
+        }
+        lr_fixup<<<nblk(A), 256, 0, s>>>(act, A, sub, local, va, spl_idx, (int32_t)head, rank);
+        LCK(cudaEventRecord(ev[2], s));
+        // ---------------- Phase III
+        for (int64_t r = rounds - 1; r >= 0; r--) {
+            const int64_t cnt = round_cnt[r];
+            if (cnt)
+                lr_reinsert<<<nblk(cnt), 256, 0, s>>>(rem_log + round_off[r], cnt, rem_pred,
+                                                      rem_dist, rank);
+        }
+        LCK(cudaEventRecord(ev[3], s));
+        LCK(cudaGetLastError());
+        LCK(cudaEventSynchronize(ev[3]));
+        if (info) {
+            float t1, t2, t3;
+            LCK(cudaEventElapsedTime(&t1, ev[0], ev[1]));
+            LCK(cudaEventElapsedTime(&t2, ev[1], ev[2]));
+            LCK(cudaEventElapsedTime(&t3, ev[2], ev[3]));
+            info[0] = rounds;
+            info[1] = A;
+            info[2] = ns;
+            info[3] = draws;
+            info[4] = (int64_t)(t1 * 1000.0f);
+            info[5] = (int64_t)(t2 * 1000.0f);
+            info[6] = (int64_t)(t3 * 1000.0f);
+            info[7] = (int64_t)round_cnt.size();
+        }
+        for (auto &e : ev) cudaEventDestroy(e);
+    } catch (const Fail &f) {
+        rc = f.rc;
+    }
+    for (void *p : bufs) cudaFreeAsync(p, s);
+    if (rc == PRNG_OK && cudaStreamSynchronize(s) != cudaSuccess) rc = PRNG_E_CUDA;
+    return rc;
+}

@@ -283,7 +283,6 @@ gg::FillArgs fill_args(prng_s *h, const uint32_t *bits, uint64_t pitch, uint64_t
     a.m = h->g.m;
     a.log2m = h->log2m;
     a.pow2 = h->pow2;
-    a.c_mul = 4;
     return a;
 }
 
@@ -465,8 +464,7 @@ int prng_create(prng_t **out, const prng_graph_params *g, uint64_t walkers, uint
             a.m = g->m;
             a.log2m = h->log2m;
             a.pow2 = h->pow2;
-            a.c_mul = 4;
-            a.x = h->x;
+                    a.x = h->x;
             a.y = h->y;
             a.j = h->j;
             CK(gg::launch_init(a, h->work_stream));
@@ -738,7 +736,6 @@ int prng_device_view(prng_t *h, void *view, size_t view_bytes) {
     v.l = h->g.walk_len;
     v.log2m = h->log2m;
     v.pow2 = h->pow2;
-    v.c_mul = 4;
     memcpy(view, &v, sizeof(v));
     return PRNG_OK;
 }

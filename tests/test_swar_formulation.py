@@ -25,7 +25,7 @@ def _word10(Q, nk, x, y):
     for k in range(nk):
         py, px = MY & (1 << 3 * k), MX & (1 << 3 * k)
         ct = (C << (30 - 3 * k)) & M          # IMAD.SHL
-        c = (ct * 4) >> 32                   # IMAD.HI with c_mul = 4
+        c = ct >> 30                         # LEA.HI operand
         u = (x + y + c) & M
         if py:
             y = (u + x) & M

@@ -41,6 +41,26 @@ __device__ __forceinline__ void step(uint32_t MY, uint32_t MX, uint32_t C, uint3
       "shl.b32 ct, %4, %6;\n\tmul.hi.u32 c, ct, %7;\n\tadd.u32 u, %0, %1;\n\tadd.u32 u, u, c;\n\t"
       "@py add.u32 %1, u, %0;\n\t@px add.u32 %0, u, %1;\n\t}"
       : "+r"(x), "+r"(y) : "r"(MY), "r"(MX), "r"(C), "n"(1u << (3*K)), "n"(30 - 3*K), "r"(four));
+  } else if (V == 6) {  // u = (x + y) + c with c via LEA.HI; adds left to ptxas balancing
+    asm volatile("{\n\t.reg .pred py, px;\n\t.reg .b32 ty, tx, ct, c, u, s;\n\t"
+      "and.b32 ty, %2, %5;\n\tsetp.ne.b32 py, ty, 0;\n\tand.b32 tx, %3, %5;\n\tsetp.ne.b32 px, tx, 0;\n\t"
+      "shl.b32 ct, %4, %6;\n\tshr.b32 c, ct, 30;\n\tadd.u32 s, %0, %1;\n\tadd.u32 u, s, c;\n\t"
+      "@py add.u32 %1, u, %0;\n\t@px add.u32 %0, u, %1;\n\t}"
+      : "+r"(x), "+r"(y) : "r"(MY), "r"(MX), "r"(C), "n"(1u << (3*K)), "n"(30 - 3*K));
+  } else if (V == 7) {  // V6 with the shift alternating ALU (odd K) / FMA-heavy (even K)
+    if (K & 1) {
+      asm volatile("{\n\t.reg .pred py, px;\n\t.reg .b32 ty, tx, ct, c, u, s;\n\t"
+        "and.b32 ty, %2, %5;\n\tsetp.ne.b32 py, ty, 0;\n\tand.b32 tx, %3, %5;\n\tsetp.ne.b32 px, tx, 0;\n\t"
+        "shf.l.wrap.b32 ct, %7, %4, %6;\n\tshr.b32 c, ct, 30;\n\tmad.lo.u32 s, %0, %8, %1;\n\tadd.u32 u, s, c;\n\t"
+        "@py mad.lo.u32 %1, %0, %8, u;\n\t@px add.u32 %0, u, %1;\n\t}"
+        : "+r"(x), "+r"(y) : "r"(MY), "r"(MX), "r"(C), "n"(1u << (3*K)), "n"(30 - 3*K), "r"(0u), "r"(four >> 2));
+    } else {
+      asm volatile("{\n\t.reg .pred py, px;\n\t.reg .b32 ty, tx, ct, c, u, s;\n\t"
+        "and.b32 ty, %2, %5;\n\tsetp.ne.b32 py, ty, 0;\n\tand.b32 tx, %3, %5;\n\tsetp.ne.b32 px, tx, 0;\n\t"
+        "shl.b32 ct, %4, %6;\n\tshr.b32 c, ct, 30;\n\tmad.lo.u32 s, %0, %7, %1;\n\tadd.u32 u, s, c;\n\t"
+        "@py mad.lo.u32 %1, %0, %7, u;\n\t@px add.u32 %0, u, %1;\n\t}"
+        : "+r"(x), "+r"(y) : "r"(MY), "r"(MX), "r"(C), "n"(1u << (3*K)), "n"(30 - 3*K), "r"(four >> 2));
+    }
   } else {  // V3: c via shr (ALU) then adds as IMAD.IADD-able add
     asm volatile("{\n\t.reg .pred py, px;\n\t.reg .b32 ty, tx, c, yc, xc;\n\t"
       "and.b32 ty, %2, %5;\n\tsetp.ne.b32 py, ty, 0;\n\tand.b32 tx, %3, %5;\n\tsetp.ne.b32 px, tx, 0;\n\t"
@@ -137,16 +157,16 @@ int main() {
     float t0 = run<0>(bits, pitch, W, D, xs, ys, out, wps, 3);
     cudaMemcpy(ref.data(), out + (size_t)(D - 1) * W, 4096 * 8, cudaMemcpyDeviceToHost);
     float t[4] = {t0, 0, 0, 0};
-    t[1] = run<1>(bits, pitch, W, D, xs, ys, out, wps, 3);
+    t[1] = run<6>(bits, pitch, W, D, xs, ys, out, wps, 3);
     cudaMemcpy(got.data(), out + (size_t)(D - 1) * W, 4096 * 8, cudaMemcpyDeviceToHost);
     bool ok1 = got == ref;
     t[2] = run<5>(bits, pitch, W, D, xs, ys, out, wps, 3);
     cudaMemcpy(got.data(), out + (size_t)(D - 1) * W, 4096 * 8, cudaMemcpyDeviceToHost);
     bool ok2 = got == ref;
-    t[3] = run<4>(bits, pitch, W, D, xs, ys, out, wps, 3);
+    t[3] = run<7>(bits, pitch, W, D, xs, ys, out, wps, 3);
     cudaMemcpy(got.data(), out + (size_t)(D - 1) * W, 4096 * 8, cudaMemcpyDeviceToHost);
     bool ok3 = got == ref;
-    printf("warps/SM %d: V0 %.3f ms (%.1f G/s)  V1 %.3f (%.1f) %s  V5 %.3f (%.1f) %s  V4 %.3f (%.1f) %s\n", wps,
+    printf("warps/SM %d: V0 %.3f ms (%.1f G/s)  V6 %.3f (%.1f) %s  V5 %.3f (%.1f) %s  V7 %.3f (%.1f) %s\n", wps,
            t[0], labels / t[0] / 1e6, t[1], labels / t[1] / 1e6, ok1 ? "ok" : "MISMATCH", t[2], labels / t[2] / 1e6,
            ok2 ? "ok" : "MISMATCH", t[3], labels / t[3] / 1e6, ok3 ? "ok" : "MISMATCH");
   }
