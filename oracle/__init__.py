@@ -82,7 +82,12 @@ def _bind_optional(L):
     opt = {
         "or_lr_rank_seq": (ctypes.c_int, [i64, P, i64, P]),
         "or_lr_run": (ctypes.c_int, [u64, u32, u32, u64, i64, P, P, i64, i64, P, P, P, P]),
-        "or_mc_run": (ctypes.c_int, [P, P, P, P]),
+        "or_mc_run": (ctypes.c_int, [P, ctypes.c_int, f64, f64, u64, u32, u32, u64, u64, u64, u64,
+                                     u64, u32, f64, P, P, P]),
+        "or_mc_xi": (f64, [u64]),
+        "or_mc_hg": (f64, [f64, f64]),
+        "or_mc_fresnel": (f64, [f64, f64, f64, P]),
+        "or_mc_q": (u64, [f64]),
     }
     for name, (res, args) in opt.items():
         fn = getattr(L, name, None)
@@ -201,3 +206,44 @@ def lr_run(succ, pred, head: int, seed: int, m: int = 1 << 32, l: int = 64, l0: 
     return {"rank": rank, "removed_round": removed, "is_splitter": spl.astype(bool),
             "rounds": int(info[0]), "reduced": int(info[1]), "splitters": int(info[2]),
             "draws": int(info[3])}
+
+
+# ---------------------------------------------------------------- Monte Carlo
+MC_TALLY_NAMES = ("launched", "specular", "R_d", "T_t", "terminated")
+
+# R19: MCML's sample slab (n, mua [1/cm], mus [1/cm], g, d [cm]); ambient n = 1.
+MC_LAYERS_R19 = ((1.37, 1.0, 100.0, 0.9, 0.1), (1.37, 1.0, 10.0, 0.0, 0.1), (1.37, 2.0, 10.0, 0.7, 0.2))
+
+
+def mc_run(layers=MC_LAYERS_R19, n_top=1.0, n_bottom=1.0, seed=0x5EED0004, walker0=0,
+           nthreads=64, photons_total=256, threads_total=None, D=192, w_th=1e-4,
+           m=1 << 32, l=64, l0=64, per_thread=False):
+    """Sequential replica of the GPU photon-migration run (mc_oracle.c)."""
+    layers = np.ascontiguousarray(np.array(layers, dtype=np.float64).reshape(-1, 5))
+    nl = layers.shape[0]
+    threads_total = nthreads if threads_total is None else threads_total
+    tal = np.zeros(5 + nl, dtype=np.int64)
+    pt = np.zeros((nthreads, 5 + nl), dtype=np.int64) if per_thread else None
+    stats = np.zeros(4, dtype=np.int64)
+    rc = lib().or_mc_run(_ptr(layers), nl, n_top, n_bottom, m, l, l0, seed, walker0, nthreads,
+                         photons_total, threads_total, D, w_th, _ptr(tal),
+                         None if pt is None else _ptr(pt), _ptr(stats))
+    if rc != 0:
+        raise ValueError("or_mc_run")
+    out = {k: int(tal[i]) for i, k in enumerate(MC_TALLY_NAMES)}
+    out["absorbed"] = [int(v) for v in tal[5:]]
+    out["tallies"] = tal
+    out["photons"], out["draws"], out["epochs"], out["interactions"] = (int(v) for v in stats)
+    if per_thread:
+        out["per_thread"] = pt
+    return out
+
+
+def mc_hg(g: float, xi: float) -> float:
+    return float(lib().or_mc_hg(g, xi))
+
+
+def mc_fresnel(n1: float, n2: float, ca1: float):
+    ca2 = np.zeros(1)
+    r = lib().or_mc_fresnel(n1, n2, ca1, _ptr(ca2))
+    return float(r), float(ca2[0])
