@@ -64,6 +64,55 @@ int gg_list_rank(prng_t *h, int64_t n, const int32_t *succ, const int32_t *pred,
                  int32_t *rank, int32_t *removed_round, int32_t *is_splitter, int64_t *info,
                  void *stream);
 
+/* ---------------------------------------------------------------------------
+ * Monte Carlo photon migration (§VI, Alg.4): photons from a
+ * pencil beam at the origin travel through a stack of layers; at every
+ * interaction a fraction mua/(mua+mus) of the weight is absorbed and the
+ * packet is scattered (Henyey-Greenstein); packets below the weight
+ * threshold are terminated; boundaries reflect/refract by Fresnel's law.
+ * Weights are drawn on demand with prng_next (Alg.4 l.3), as are step
+ * lengths, scattering angles and Fresnel decisions.  Readings R19-R22 in
+ * DESIGN.md §3 fix what the paper leaves open (draw order, fixed point).
+ * ------------------------------------------------------------------------- */
+#define GG_MC_MAX_LAYERS 16
+#define GG_MC_TALLY_FIXED 5
+
+typedef struct {
+    double n;    /* refractive index */
+    double mua;  /* absorption coefficient [1/cm] */
+    double mus;  /* scattering coefficient [1/cm] */
+    double g;    /* Henyey-Greenstein anisotropy, (-1, 1) */
+    double d;    /* thickness [cm], > 0 */
+} gg_mc_layer;
+
+typedef struct {
+    const gg_mc_layer *layers;  /* host array of nlayers (1..GG_MC_MAX_LAYERS) */
+    int nlayers;
+    double n_top, n_bottom;     /* ambient refractive indices above / below */
+    uint64_t photons_total;     /* P over all shards */
+    uint64_t threads_total;     /* global GPU threads over all shards */
+    uint64_t thread0;           /* global id of this call's thread 0 (= walker_base) */
+    uint64_t threads;           /* threads of this call; walker i serves thread i */
+    uint32_t epoch_draws;       /* D = 3K draws per walker per epoch, multiple of 3 */
+    double w_threshold;         /* terminate below this weight (1e-4) */
+} gg_mc_config;
+
+/*
+ * Run the simulation for global threads [thread0, thread0 + threads); thread
+ * tg simulates P/Tg photons (+1 if tg < P mod Tg), so shards over GPUs sum to
+ * the single-GPU result exactly.
+ *   tallies    : HOST int64[GG_MC_TALLY_FIXED + nlayers], ADDED to, weight
+ *                units 2^-32: launched, specular, diffuse reflectance R_d,
+ *                transmittance T_t, terminated, absorbed per layer.
+ *                launched = sum of the others exactly.
+ *   per_thread : optional DEVICE int64[threads * (5 + nlayers)] (parity checks).
+ *   stats      : optional HOST int64[6]: photons, draws, epochs,
+ *                interactions, kernel microseconds, total microseconds.
+ * Synchronous.  The handle needs >= threads walkers and no open epoch.
+ */
+int gg_mc_run(prng_t *h, const gg_mc_config *cfg, int64_t *tallies, int64_t *per_thread,
+              int64_t *stats, void *stream);
+
 #ifdef __cplusplus
 }
 #endif

@@ -125,6 +125,15 @@ __device__ __forceinline__ void gg_walk64(const uint32_t w[6], uint32_t &x, uint
     gg_word10<4>(w[5] >> 20, x, y);
 }
 
+/* Read-only 32-bit load that the compiler may not sink below later volatile
+ * asm (the walk): used to prefetch the next draw's record a full walk ahead. */
+__device__ __forceinline__ uint32_t gg_ldg_early(const uint32_t *p)
+{
+    uint32_t v;
+    asm volatile("ld.global.nc.L1::no_allocate.u32 %0, [%1];" : "=r"(v) : "l"(p));
+    return v;
+}
+
 /* One step, any m (generic path).  Non power-of-two m requires m <= 2^30 and
  * x, y < m: the pre-reduction value 2*src + target + 2 < 4m fits in 32 bits. */
 __device__ __forceinline__ void gg_step_generic(uint32_t b, uint32_t &x, uint32_t &y,

@@ -68,6 +68,7 @@ class Generator:
                  epoch_draws: int = 16, host_threads: int = 0, bits_fn=None):
         self._h = ctypes.c_void_p()
         self.walkers, self.seed, self.m, self.walk_len = walkers, seed, m, walk_len
+        self._walker_base = walker_base
         self._bits_fn = None
         if bits_fn is not None:
             # bits_fn(walker0, nwalkers, word0, nwords) -> numpy uint32 [nwords, nwalkers]
@@ -168,6 +169,33 @@ class Generator:
         keys = ("rounds", "reduced", "splitters", "draws", "phase1_us", "phase2_us", "phase3_us",
                 "rounds2")
         return rank, {k: info[i] for i, k in enumerate(keys)}
+
+    def mc_run(self, layers, photons_total: int, threads: int | None = None, n_top: float = 1.0,
+               n_bottom: float = 1.0, threads_total: int | None = None, thread0: int | None = None,
+               epoch_draws: int = 192, w_threshold: float = 1e-4, per_thread=None, stream=None):
+        """gg_mc_run: Monte Carlo photon migration (Alg.4) driven by prng_next.
+
+        layers: sequence of (n, mua, mus, g, d).  Returns a dict of fixed-point
+        tallies (units 2^-32) and run statistics."""
+        threads = self.walkers if threads is None else threads
+        threads_total = threads if threads_total is None else threads_total
+        thread0 = self._walker_base if thread0 is None else thread0
+        arr = (_lib.gg_mc_layer * len(layers))(*[_lib.gg_mc_layer(*map(float, L)) for L in layers])
+        cfg = _lib.gg_mc_config(arr, len(layers), n_top, n_bottom, photons_total, threads_total,
+                                thread0, threads, epoch_draws, w_threshold)
+        nt = 5 + len(layers)
+        tal = (ctypes.c_int64 * nt)()
+        stats = (ctypes.c_int64 * 6)()
+        check(_lib.gg_mc_run(self._h, ctypes.byref(cfg), tal,
+                             None if per_thread is None else per_thread.data_ptr(), stats,
+                             _stream_handle(stream)), "gg_mc_run")
+        names = ("launched", "specular", "R_d", "T_t", "terminated")
+        out = {k: tal[i] for i, k in enumerate(names)}
+        out["absorbed"] = [tal[i] for i in range(5, nt)]
+        out["tallies"] = [tal[i] for i in range(nt)]
+        for i, k in enumerate(("photons", "draws", "epochs", "interactions", "kernel_us", "total_us")):
+            out[k] = stats[i]
+        return out
 
     def view(self) -> _lib.prng_view:
         v = _lib.prng_view()

@@ -55,6 +55,18 @@ class prng_stats(ctypes.Structure):
                 ("d2h_bytes", u64), ("kernel_launches", u64), ("feed_seconds", ctypes.c_double)]
 
 
+class gg_mc_layer(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_double), ("mua", ctypes.c_double), ("mus", ctypes.c_double),
+                ("g", ctypes.c_double), ("d", ctypes.c_double)]
+
+
+class gg_mc_config(ctypes.Structure):
+    _fields_ = [("layers", ctypes.POINTER(gg_mc_layer)), ("nlayers", c_int),
+                ("n_top", ctypes.c_double), ("n_bottom", ctypes.c_double),
+                ("photons_total", u64), ("threads_total", u64), ("thread0", u64),
+                ("threads", u64), ("epoch_draws", u32), ("w_threshold", ctypes.c_double)]
+
+
 class prng_view(ctypes.Structure):
     """Mirror of struct prng_view (include/prng_device.cuh)."""
     _fields_ = [("bits", vp), ("x", vp), ("y", vp), ("j", vp), ("flags", vp), ("pitch", u64),
@@ -87,6 +99,7 @@ _SIGS = {
     # include/gg_apps.h
     "gg_consume": (c_int, [vp, u64, vp, u32, vp, vp, vp, vp]),
     "gg_list_rank": (c_int, [vp, ctypes.c_int64, vp, vp, ctypes.c_int64, vp, vp, vp, vp, vp]),
+    "gg_mc_run": (c_int, [vp, ctypes.POINTER(gg_mc_config), vp, vp, vp, vp]),
 }
 
 for _name, (_res, _args) in _SIGS.items():

@@ -23,6 +23,9 @@ ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 CUDA_FLAGS = ARCH + ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O2",
                      "-Xptxas", "-O3", "--expt-relaxed-constexpr"]
 CXX_FLAGS = ["-O3", "-fPIC", "-std=c++17", "-fno-fast-math"]
+# mc.cu: fp64 physics evaluated exactly as written (no FMA contraction), to
+# match the CPU oracle expression by expression.
+PER_FILE_FLAGS = {"mc.cu": ["-fmad=false"]}
 
 
 def sources():
@@ -55,7 +58,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
     procs = []
     for src in cu:
         obj = os.path.join(objdir, os.path.basename(src) + ".o")
-        cmd = [NVCC] + CUDA_FLAGS + ["-I", INCLUDE, "-I", CSRC, "-c", src, "-o", obj]
+        extra = PER_FILE_FLAGS.get(os.path.basename(src), [])
+        cmd = [NVCC] + CUDA_FLAGS + extra + ["-I", INCLUDE, "-I", CSRC, "-c", src, "-o", obj]
         procs.append((cmd, subprocess.Popen(cmd, stdout=subprocess.PIPE, stderr=subprocess.STDOUT)))
         objs.append(obj)
     for src in cpp:

@@ -73,20 +73,30 @@ __global__ void __launch_bounds__(64) gg_fill64_kernel(FillArgs a, uint32_t unit
         if (j0 >= j1) continue;
         uint32_t x = a.x[t], y = a.y[t];
         const uint32_t *col = a.bits + t;
-        uint32_t w[6];
+        // Two-deep register pipeline of draw records: the loads issued while
+        // walking draw j are for draw j+2, so wherever the scheduler places
+        // them inside the iteration they get a whole walk (~450 SASS) of
+        // latency hiding.  Indices are clamped so the loads are unconditional.
+        uint32_t w0[6], w1[6];
         {
-            const uint32_t *rec = col + (uint64_t)(j0 - a.Jw) * 6u * a.pitch;
+            const uint32_t *r0 = col + (uint64_t)(j0 - a.Jw) * 6u * a.pitch;
+            const uint32_t j1c = (j0 + 1 < j1) ? j0 + 1 : j0;
+            const uint32_t *r1 = col + (uint64_t)(j1c - a.Jw) * 6u * a.pitch;
 #pragma unroll
-            for (int r = 0; r < 6; r++) w[r] = __ldg(rec + (uint64_t)r * a.pitch);
+            for (int r = 0; r < 6; r++) {
+                w0[r] = __ldg(r0 + (uint64_t)r * a.pitch);
+                w1[r] = __ldg(r1 + (uint64_t)r * a.pitch);
+            }
         }
         for (uint32_t j = j0; j < j1; j++) {
-            uint32_t wn[6];
-            if (j + 1 < j1) {
-                const uint32_t *rec = col + (uint64_t)(j + 1 - a.Jw) * 6u * a.pitch;
+            uint32_t w2[6];
+            {
+                const uint32_t jn = (j + 2 < j1) ? j + 2 : j;
+                const uint32_t *rec = col + (uint64_t)(jn - a.Jw) * 6u * a.pitch;
 #pragma unroll
-                for (int r = 0; r < 6; r++) wn[r] = __ldg(rec + (uint64_t)r * a.pitch);
+                for (int r = 0; r < 6; r++) w2[r] = __ldg(rec + (uint64_t)r * a.pitch);
             }
-            gg_walk64(w, x, y);
+            gg_walk64(w0, x, y);
             const uint64_t lab = gg_label(x, y, a.m, a.log2m, true);
             const uint64_t g = (uint64_t)j * a.W + t;
             if (OUT32)
@@ -94,7 +104,10 @@ __global__ void __launch_bounds__(64) gg_fill64_kernel(FillArgs a, uint32_t unit
             else
                 reinterpret_cast<uint64_t *>(a.out)[g - a.g_origin] = lab;
 #pragma unroll
-            for (int r = 0; r < 6; r++) w[r] = wn[r];
+            for (int r = 0; r < 6; r++) {
+                w0[r] = w1[r];
+                w1[r] = w2[r];
+            }
         }
         a.x[t] = x;
         a.y[t] = y;

@@ -1,0 +1,419 @@
+// Monte Carlo photon migration with on-demand random numbers
+// (§VI, Alg.4 MCPhotonMigration).  C ABI: gg_mc_run
+// (include/gg_apps.h).  Compiled with -fmad=false: every fp64 expression is
+// evaluated as written (IEEE add/mul/div/sqrt, no contraction), in the same
+// order as the CPU oracle's, so the two agree exactly unless a libm log/sin/
+// cos result differs by an ulp right at a decision threshold.
+//
+// One GPU thread per walker; the photon state lives in SoA arrays between
+// epochs.  An epoch = one on-demand window of D = 3K draws per walker
+// (prng_epoch_begin); every iteration of a thread with work takes exactly
+// three prng_next draws at the same program point (so a warp walks the
+// expander in lockstep; only the physics diverges) and uses what it needs:
+// launch (W0 from draw a), or hop (sleft from a when needed) + boundary
+// (Fresnel test with b) or drop + spin (HG cos(theta) from b, psi from c).
+// Weights and tallies are int64 fixed point (units 2^-32), so tallies are
+// exact integer sums and order independent; the host allreduces them across
+// GPUs (NCCL) if sharded.
+#include <cmath>
+#include <cstdint>
+#include <vector>
+
+#include <cuda_runtime.h>
+
+#include "gg_apps.h"
+#include "prng.h"
+#include "prng_device.cuh"
+
+namespace {
+
+constexpr int kMaxL = GG_MC_MAX_LAYERS;
+constexpr int kFixed = 5;  // launched, specular, R_d, T_t, terminated
+constexpr double kPi = 3.14159265358979323846;
+
+struct McParams {
+    double zb[kMaxL + 1];     // layer boundaries, zb[0] = 0
+    double nidx[kMaxL + 2];   // refractive index: 0 = top ambient, nl+1 = bottom ambient
+    double mua[kMaxL + 1], mus[kMaxL + 1], g[kMaxL + 1];  // 1-based
+    uint64_t qabs[kMaxL + 1]; // round(2^32 mua/mut)
+    uint64_t q_sp;            // round(2^32 Rsp)
+    uint64_t w_th;            // floor(2^32 w_threshold)
+    uint64_t photons_total, threads_total, thread0, threads;
+    int nl;
+    uint32_t K;               // iterations per epoch (D = 3K)
+};
+
+struct McState {
+    double *x, *y, *z, *ux, *uy, *uz, *sleft;
+    uint64_t *w;
+    int32_t *layer;
+    uint32_t *alive, *launched;
+};
+
+__device__ __forceinline__ double mc_xi(uint64_t label) {
+    return (double)((label >> 11) + 1) * (1.0 / 9007199254740992.0);
+}
+
+__device__ __forceinline__ uint64_t mc_frac(uint64_t w, uint64_t q) {
+    // (w * q) >> 32 over the full 128-bit product
+    return (__umul64hi(w, q) << 32) | ((w * q) >> 32);
+}
+
+__device__ __forceinline__ double mc_hg(double g, double xi) {
+    double cost;
+    if (g == 0.0) {
+        cost = 2.0 * xi - 1.0;
+    } else {
+        double temp = (1.0 - g * g) / (1.0 - g + 2.0 * g * xi);
+        cost = (1.0 + g * g - temp * temp) / (2.0 * g);
+        if (cost < -1.0)
+            cost = -1.0;
+        else if (cost > 1.0)
+            cost = 1.0;
+    }
+    return cost;
+}
+
+__device__ __forceinline__ double mc_fresnel(double n1, double n2, double ca1, double *ca2) {
+    double r;
+    if (n1 == n2) {
+        *ca2 = ca1;
+        r = 0.0;
+    } else if (ca1 > 1.0 - 1.0e-12) {
+        *ca2 = ca1;
+        r = (n2 - n1) / (n2 + n1);
+        r = r * r;
+    } else if (ca1 < 1.0e-6) {
+        *ca2 = 0.0;
+        r = 1.0;
+    } else {
+        double sa1 = sqrt(1.0 - ca1 * ca1);
+        double sa2 = n1 * sa1 / n2;
+        if (sa2 >= 1.0) {
+            *ca2 = 0.0;
+            r = 1.0;
+        } else {
+            double c2 = sqrt(1.0 - sa2 * sa2);
+            double cap = ca1 * c2 - sa1 * sa2;
+            double cam = ca1 * c2 + sa1 * sa2;
+            double sap = sa1 * c2 + ca1 * sa2;
+            double sam = sa1 * c2 - ca1 * sa2;
+            *ca2 = c2;
+            r = 0.5 * sam * sam * (cam * cam + cap * cap) / (sap * sap * cam * cam);
+        }
+    }
+    return r;
+}
+
+__global__ void mc_init_state(McState s, uint64_t n) {
+    const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    s.alive[i] = 0;
+    s.launched[i] = 0;
+    s.w[i] = 0;
+}
+
+__global__ void __launch_bounds__(128) mc_epoch(prng_view v, McParams P, McState S,
+                                                unsigned long long *tallies,
+                                                long long *per_thread,
+                                                unsigned long long *counters) {
+    const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int nt = kFixed + P.nl;
+    long long tal[kFixed + kMaxL];
+#pragma unroll
+    for (int k = 0; k < kFixed + kMaxL; k++) tal[k] = 0;
+    unsigned long long launched_now = 0, interactions = 0, draws = 0, done = 0;
+    if (i < P.threads) {
+        const uint64_t tg = P.thread0 + i;
+        const uint64_t budget =
+            P.photons_total / P.threads_total + (tg < P.photons_total % P.threads_total ? 1 : 0);
+        double x = S.x[i], y = S.y[i], z = S.z[i], ux = S.ux[i], uy = S.uy[i], uz = S.uz[i];
+        double sleft = S.sleft[i];
+        uint64_t w = S.w[i];
+        int layer = S.layer[i];
+        bool alive = S.alive[i] != 0;
+        uint32_t launched = S.launched[i];
+        prng_state st = prng_state_load(&v, (uint32_t)i);
+        for (uint32_t it = 0; it < P.K; it++) {
+            if (!alive && launched == budget) break;
+            // three draws at a convergent point (R22)
+            const uint64_t la = prng_next(&st, &v);
+            const uint64_t lb = prng_next(&st, &v);
+            const uint64_t lc = prng_next(&st, &v);
+            draws += 3;
+            if (!alive) {
+                // Alg.4 l.3: launch a photon with its weight from getnextrand()
+                const uint64_t w0 = (la >> 32) + 1;
+                const uint64_t sp = mc_frac(w0, P.q_sp);
+                tal[0] += (long long)w0;
+                tal[1] += (long long)sp;
+                w = w0 - sp;
+                x = 0.0;
+                y = 0.0;
+                z = 0.0;
+                ux = 0.0;
+                uy = 0.0;
+                uz = 1.0;
+                sleft = 0.0;
+                layer = 1;
+                alive = true;
+                launched++;
+                launched_now++;
+                continue;
+            }
+            const double mua = P.mua[layer], mus = P.mus[layer], g = P.g[layer];
+            const double mut = mua + mus;
+            if (sleft == 0.0) sleft = -log(mc_xi(la));
+            double db;
+            if (uz > 0.0)
+                db = (P.zb[layer] - z) / uz;
+            else if (uz < 0.0)
+                db = (P.zb[layer - 1] - z) / uz;
+            else
+                db = INFINITY;
+            const double s = sleft / mut;
+            if (s > db) {
+                x = x + db * ux;
+                y = y + db * uy;
+                z = z + db * uz;
+                sleft = sleft - db * mut;
+                const int nb = uz < 0.0 ? layer - 1 : layer + 1;
+                const double n1 = P.nidx[layer], n2 = P.nidx[nb];
+                double ca2;
+                const double r = mc_fresnel(n1, n2, fabs(uz), &ca2);
+                bool reflect = false;
+                if (n1 != n2) reflect = mc_xi(lb) <= r;
+                if (reflect) {
+                    uz = -uz;
+                } else if (nb == 0 || nb == P.nl + 1) {
+                    tal[nb == 0 ? 2 : 3] += (long long)w;
+                    w = 0;
+                    alive = false;
+                } else {
+                    layer = nb;
+                    if (n1 != n2) {
+                        ux = ux * (n1 / n2);
+                        uy = uy * (n1 / n2);
+                        uz = uz > 0.0 ? ca2 : -ca2;
+                    }
+                }
+            } else {
+                x = x + s * ux;
+                y = y + s * uy;
+                z = z + s * uz;
+                sleft = 0.0;
+                const uint64_t dw = mc_frac(w, P.qabs[layer]);
+                w -= dw;
+                tal[kFixed + layer - 1] += (long long)dw;
+                const double cost = mc_hg(g, mc_xi(lb));
+                const double psi = 2.0 * kPi * mc_xi(lc);
+                const double cosp = cos(psi), sinp = sin(psi);
+                const double sint = sqrt(1.0 - cost * cost);
+                const double ox = ux, oy = uy, oz = uz;
+                if (fabs(oz) > 0.99999) {
+                    ux = sint * cosp;
+                    uy = sint * sinp;
+                    uz = oz >= 0.0 ? cost : -cost;
+                } else {
+                    const double temp = sqrt(1.0 - oz * oz);
+                    ux = sint * (ox * oz * cosp - oy * sinp) / temp + ox * cost;
+                    uy = sint * (oy * oz * cosp + ox * sinp) / temp + oy * cost;
+                    uz = -sint * cosp * temp + oz * cost;
+                }
+                interactions++;
+                if (w < P.w_th) {
+                    tal[4] += (long long)w;
+                    w = 0;
+                    alive = false;
+                }
+            }
+        }
+        prng_state_store(&v, &st);
+        S.x[i] = x;
+        S.y[i] = y;
+        S.z[i] = z;
+        S.ux[i] = ux;
+        S.uy[i] = uy;
+        S.uz[i] = uz;
+        S.sleft[i] = sleft;
+        S.w[i] = w;
+        S.layer[i] = layer;
+        S.alive[i] = alive ? 1u : 0u;
+        S.launched[i] = launched;
+        done = (!alive && launched == budget) ? 1 : 0;
+        if (per_thread)
+            for (int k = 0; k < nt; k++) per_thread[i * nt + k] += tal[k];
+    }
+    // warp-level integer reductions, one atomic per warp and counter
+    const unsigned full = 0xFFFFFFFFu;
+    for (int k = 0; k < nt; k++) {
+        unsigned long long vsum = (unsigned long long)tal[k];
+        for (int o = 16; o > 0; o >>= 1) vsum += __shfl_down_sync(full, vsum, o);
+        if ((threadIdx.x & 31) == 0 && vsum) atomicAdd(&tallies[k], vsum);
+    }
+    unsigned long long c[4] = {launched_now, draws, interactions, done};
+    for (int k = 0; k < 4; k++) {
+        unsigned long long vsum = c[k];
+        for (int o = 16; o > 0; o >>= 1) vsum += __shfl_down_sync(full, vsum, o);
+        if ((threadIdx.x & 31) == 0 && vsum) atomicAdd(&counters[k], vsum);
+    }
+}
+
+struct Fail {
+    int rc;
+};
+#define MCK(call)                                              \
+    do {                                                       \
+        cudaError_t _e = (call);                               \
+        if (_e != cudaSuccess) throw Fail{PRNG_E_CUDA};        \
+    } while (0)
+#define MRC(call)                                              \
+    do {                                                       \
+        int _r = (call);                                       \
+        if (_r != PRNG_OK) throw Fail{_r};                     \
+    } while (0)
+
+uint64_t q32(double f) { return (uint64_t)llround(ldexp(f, 32)); }
+
+}  // namespace
+
+extern "C" int gg_mc_run(prng_t *h, const gg_mc_config *cfg, int64_t *tallies, int64_t *per_thread,
+                         int64_t *stats, void *stream) {
+    if (!h || !cfg || !tallies || !cfg->layers) return PRNG_E_INVALID;
+    if (cfg->nlayers < 1 || cfg->nlayers > kMaxL || cfg->threads == 0 ||
+        cfg->threads_total == 0 || cfg->epoch_draws < 3 || cfg->epoch_draws % 3 != 0 ||
+        cfg->thread0 + cfg->threads > cfg->threads_total)
+        return PRNG_E_INVALID;
+    cudaStream_t s = (cudaStream_t)stream;
+    McParams P{};
+    P.nl = cfg->nlayers;
+    P.zb[0] = 0.0;
+    P.nidx[0] = cfg->n_top;
+    for (int l = 1; l <= P.nl; l++) {
+        const gg_mc_layer &L = cfg->layers[l - 1];
+        if (!(L.d > 0.0) || L.mua < 0.0 || L.mus < 0.0 || !(L.mua + L.mus > 0.0) || L.g <= -1.0 ||
+            L.g >= 1.0)
+            return PRNG_E_INVALID;
+        P.zb[l] = P.zb[l - 1] + L.d;
+        P.nidx[l] = L.n;
+        P.mua[l] = L.mua;
+        P.mus[l] = L.mus;
+        P.g[l] = L.g;
+        P.qabs[l] = q32(L.mua / (L.mua + L.mus));
+    }
+    P.nidx[P.nl + 1] = cfg->n_bottom;
+    double rsp = (cfg->n_top - P.nidx[1]) / (cfg->n_top + P.nidx[1]);
+    rsp = rsp * rsp;
+    P.q_sp = q32(rsp);
+    P.w_th = (uint64_t)floor(ldexp(cfg->w_threshold, 32));
+    P.photons_total = cfg->photons_total;
+    P.threads_total = cfg->threads_total;
+    P.thread0 = cfg->thread0;
+    P.threads = cfg->threads;
+    P.K = cfg->epoch_draws / 3;
+    const int nt = kFixed + P.nl;
+
+    std::vector<void *> bufs;
+    auto alloc = [&](size_t bytes) -> void * {
+        void *p = nullptr;
+        MCK(cudaMallocAsync(&p, bytes, s));
+        bufs.push_back(p);
+        return p;
+    };
+    int rc = PRNG_OK;
+    try {
+        const uint64_t n = cfg->threads;
+        McState S;
+        S.x = (double *)alloc(n * 8);
+        S.y = (double *)alloc(n * 8);
+        S.z = (double *)alloc(n * 8);
+        S.ux = (double *)alloc(n * 8);
+        S.uy = (double *)alloc(n * 8);
+        S.uz = (double *)alloc(n * 8);
+        S.sleft = (double *)alloc(n * 8);
+        S.w = (uint64_t *)alloc(n * 8);
+        S.layer = (int32_t *)alloc(n * 4);
+        S.alive = (uint32_t *)alloc(n * 4);
+        S.launched = (uint32_t *)alloc(n * 4);
+        unsigned long long *d_tal = (unsigned long long *)alloc(nt * 8);
+        unsigned long long *d_cnt = (unsigned long long *)alloc(4 * 8);
+        MCK(cudaMemsetAsync(d_tal, 0, nt * 8, s));
+        MCK(cudaMemsetAsync(d_cnt, 0, 4 * 8, s));
+        if (per_thread) MCK(cudaMemsetAsync(per_thread, 0, n * nt * 8, s));
+        mc_init_state<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(S, n);
+        cudaEvent_t e0, e1;
+        MCK(cudaEventCreate(&e0));
+        MCK(cudaEventCreate(&e1));
+        MCK(cudaEventRecord(e0, s));
+        unsigned long long *counters = nullptr;  // pinned: the D2H read must not block the feed
+        MCK(cudaMallocHost(&counters, 4 * sizeof(unsigned long long)));
+        int64_t epochs = 0;
+        double kernel_ms = 0.0;
+        cudaEvent_t k0, k1, kc;
+        MCK(cudaEventCreate(&k0));
+        MCK(cudaEventCreate(&k1));
+        MCK(cudaEventCreateWithFlags(&kc, cudaEventDisableTiming));
+        try {
+            MRC(prng_epoch_begin(h, n, cfg->epoch_draws, s));
+            for (;;) {
+                prng_view v;
+                MRC(prng_device_view(h, &v, sizeof(v)));
+                MCK(cudaMemsetAsync(d_cnt + 3, 0, 8, s));  // 'done' is recounted each epoch
+                MCK(cudaEventRecord(k0, s));
+                mc_epoch<<<(unsigned)((n + 127) / 128), 128, 0, s>>>(v, P, S, d_tal,
+                                                                     (long long *)per_thread, d_cnt);
+                MCK(cudaGetLastError());
+                MCK(cudaEventRecord(k1, s));
+                MRC(prng_epoch_end(h, s));
+                epochs++;
+                MCK(cudaMemcpyAsync(counters, d_cnt, 4 * sizeof(unsigned long long),
+                                    cudaMemcpyDeviceToHost, s));
+                MCK(cudaEventRecord(kc, s));
+                // FEED + TRANSFER of the next epoch overlap this epoch's kernel
+                // (Alg.4 l.7: "Generate and transfer new bin in an overlapping
+                // manner"); if every thread turns out to be done, that one
+                // speculative window is discarded.
+                MRC(prng_epoch_begin(h, n, cfg->epoch_draws, s));
+                MCK(cudaEventSynchronize(kc));
+                float ms = 0.0f;
+                MCK(cudaEventElapsedTime(&ms, k0, k1));
+                kernel_ms += ms;
+                if (counters[3] == n) {
+                    MRC(prng_epoch_end(h, s));
+                    break;
+                }
+            }
+        } catch (const Fail &) {
+            cudaFreeHost(counters);
+            throw;
+        }
+        const unsigned long long c_launched = counters[0], c_draws = counters[1],
+                                 c_inter = counters[2];
+        cudaFreeHost(counters);
+        MCK(cudaEventRecord(e1, s));
+        std::vector<unsigned long long> ht(nt);
+        MCK(cudaMemcpyAsync(ht.data(), d_tal, nt * 8, cudaMemcpyDeviceToHost, s));
+        MCK(cudaStreamSynchronize(s));
+        for (int k = 0; k < nt; k++) tallies[k] += (int64_t)ht[k];
+        if (stats) {
+            float total_ms = 0.0f;
+            MCK(cudaEventElapsedTime(&total_ms, e0, e1));
+            stats[0] = (int64_t)c_launched;    // photons launched
+            stats[1] = (int64_t)c_draws;       // draws taken by the physics
+            stats[2] = epochs;
+            stats[3] = (int64_t)c_inter;       // interactions
+            stats[4] = (int64_t)(kernel_ms * 1000.0);  // microseconds in mc_epoch kernels
+            stats[5] = (int64_t)(total_ms * 1000.0);   // microseconds end to end (feed incl.)
+        }
+        cudaEventDestroy(e0);
+        cudaEventDestroy(e1);
+        cudaEventDestroy(k0);
+        cudaEventDestroy(k1);
+        cudaEventDestroy(kc);
+    } catch (const Fail &f) {
+        rc = f.rc;
+    }
+    for (void *p : bufs) cudaFreeAsync(p, s);
+    if (cudaStreamSynchronize(s) != cudaSuccess && rc == PRNG_OK) rc = PRNG_E_CUDA;
+    return rc;
+}

@@ -146,8 +146,11 @@ struct prng_s {
     bool od_open = false, od_started = false;
     uint64_t od_J0 = 0, od_Wv = 0, od_pitch = 0;
     uint32_t od_D = 0;
-    uint32_t *od_bits = nullptr;
-    size_t od_cap = 0;
+    uint32_t *od_bits = nullptr;       // window of the open epoch (= od_buf[od_slot])
+    uint32_t *od_buf[2] = {};          // double-buffered: epoch e+1 is fed while e runs
+    size_t od_cap[2] = {};
+    cudaEvent_t od_free[2] = {};       // recorded at epoch_end: kernels done with the slot
+    int od_slot = 1;
 
     cudaEvent_t ev_tmp = nullptr;
     prng_stats stats{};
@@ -161,7 +164,7 @@ void free_all(prng_s *h) {
     cudaSetDevice(h->o.device);
     cudaDeviceSynchronize();
     for (auto p : {h->x, h->y, h->j, h->flags, h->xs, h->ys, h->js, h->res_bits, h->ring[0],
-                   h->ring[1], h->od_bits})
+                   h->ring[1], h->od_buf[0], h->od_buf[1]})
         if (p) cudaFree(p);
     for (auto p : h->hout)
         if (p) cudaFree(p);
@@ -172,6 +175,7 @@ void free_all(prng_s *h) {
     for (int i = 0; i < 2; i++) {
         if (h->ring_free[i]) cudaEventDestroy(h->ring_free[i]);
         if (h->hout_free[i]) cudaEventDestroy(h->hout_free[i]);
+        if (h->od_free[i]) cudaEventDestroy(h->od_free[i]);
     }
     if (h->ev_tmp) cudaEventDestroy(h->ev_tmp);
     for (auto s : {h->copy_stream, h->d2h_stream, h->work_stream})
@@ -435,6 +439,7 @@ int prng_create(prng_t **out, const prng_graph_params *g, uint64_t walkers, uint
         for (int i = 0; i < 2; i++) {
             CK(cudaEventCreateWithFlags(&h->ring_free[i], cudaEventDisableTiming));
             CK(cudaEventCreateWithFlags(&h->hout_free[i], cudaEventDisableTiming));
+            CK(cudaEventCreateWithFlags(&h->od_free[i], cudaEventDisableTiming));
         }
         const size_t sb = (size_t)walkers * 4;
         for (uint32_t **p : {&h->x, &h->y, &h->j, &h->xs, &h->ys, &h->js}) CK(cudaMalloc(p, sb));
@@ -687,14 +692,20 @@ int prng_epoch_begin(prng_t *h, uint64_t active_walkers, uint32_t draws, void *s
         if (J0 + draws > 0xFFFFFFFFull) return PRNG_E_UNSUPPORTED;
         const uint64_t pitch = round_up(active_walkers, 32);
         const size_t bytes = (size_t)draws * h->R * pitch * 4;
-        if (bytes > h->od_cap) {
-            CK(cudaDeviceSynchronize());
-            ensure_dev(h->od_bits, h->od_cap, bytes);
+        const int slot = h->od_slot ^ 1;
+        if (bytes > h->od_cap[slot]) {
+            CK(cudaEventSynchronize(h->od_free[slot]));
+            if (h->od_buf[slot]) CK(cudaFree(h->od_buf[slot]));
+            h->od_buf[slot] = nullptr;
+            h->od_cap[slot] = 0;
+            CK(cudaMalloc(&h->od_buf[slot], bytes));
+            h->od_cap[slot] = bytes;
         } else {
-            // the previous epoch's kernels must be done reading the window
-            CK(cudaEventRecord(h->ev_tmp, s));
-            CK(cudaStreamWaitEvent(h->copy_stream, h->ev_tmp, 0));
+            // kernels of the epoch that last used this slot must be done with it
+            CK(cudaStreamWaitEvent(h->copy_stream, h->od_free[slot], 0));
         }
+        h->od_slot = slot;
+        h->od_bits = h->od_buf[slot];
         stage_rows(h, 2 + h->R0 + h->R * J0, (uint64_t)draws * h->R, active_walkers, h->od_bits,
                    pitch);
         join_copies(h, s);
@@ -709,9 +720,12 @@ int prng_epoch_begin(prng_t *h, uint64_t active_walkers, uint32_t draws, void *s
 }
 
 int prng_epoch_end(prng_t *h, void *stream) {
-    (void)stream;
     if (!h) return PRNG_E_INVALID;
     if (!h->od_open) return PRNG_E_STATE;
+    if (cudaEventRecord(h->od_free[h->od_slot], (cudaStream_t)stream) != cudaSuccess) {
+        h->poisoned = true;
+        return PRNG_E_CUDA;
+    }
     h->od_J0 += h->od_D;
     h->od_open = false;
     h->N = h->od_J0 * h->W;  // a later bulk fill starts with every walker at draw J0
