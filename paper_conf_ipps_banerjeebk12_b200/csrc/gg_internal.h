@@ -31,6 +31,7 @@ cudaError_t launch_init(const InitArgs &a, cudaStream_t s);
 struct FillArgs {
     const uint32_t *bits;
     uint64_t pitch;
+    uint64_t rows;   // rows of the window (for the TMA tensor map)
     uint32_t Jw;
     uint32_t ja, jb;
     uint32_t W;

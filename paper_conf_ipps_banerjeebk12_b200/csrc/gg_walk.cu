@@ -11,6 +11,11 @@
 // number of units (static balance, ~1-2% tail) instead of relying on a
 // partially filled last wave.
 #include <cstdint>
+#include <cstdlib>
+#include <cstring>
+
+#include <cuda.h>
+#include <cudaTypedefs.h>
 
 #include "gg_internal.h"
 #include "prng_device.cuh"
@@ -114,6 +119,155 @@ __global__ void __launch_bounds__(64) gg_fill64_kernel(FillArgs a, uint32_t unit
     }
 }
 
+// ---------------------------------------------------------------------------
+// TMA-staged variant (the default for l = 64, m = 2^k).  Each warp owns a
+// 32-walker unit at a time; lane 0 issues one cp.async.bulk.tensor per draw
+// that copies the draw's 6 x 32-word record tile (768 B) from the SoA window
+// into a per-warp shared-memory stage, completing on an mbarrier.  Two stages:
+// the tile for draw j+2 is in flight while draw j+1 is walked, so the walk
+// never waits on HBM and no per-lane address arithmetic or register
+// rotation is needed; each lane then reads its 6 words with conflict-free LDS
+// (column `lane` of the tile).
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ uint32_t smem_u32(const void *p) {
+    return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t *bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)),
+                 "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n"
+        "GG_WAIT:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+        "@!p bra GG_WAIT;\n\t}" ::"r"(smem_u32(bar)),
+        "r"(parity)
+        : "memory");
+}
+__device__ __forceinline__ void tma_load_tile(uint32_t *dst, const CUtensorMap *map, uint64_t *bar,
+                                              int32_t c0, int32_t c1) {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, "
+        "%3}], [%4];" ::"r"(smem_u32(dst)),
+        "l"(map), "r"(c0), "r"(c1), "r"(smem_u32(bar))
+        : "memory");
+}
+
+constexpr int kTileWords = 6 * 32;  // one draw record for 32 walkers
+constexpr int kFillWarps = 2;       // warps per block
+
+template <int OUT32>
+__global__ void __launch_bounds__(64) gg_fill64_tma_kernel(const __grid_constant__ CUtensorMap tmap,
+                                                           FillArgs a, uint32_t units) {
+    __shared__ __align__(128) uint32_t tiles[kFillWarps][2][kTileWords];
+    __shared__ __align__(8) uint64_t bars[kFillWarps][2];
+    const uint32_t lane = threadIdx.x & 31u, wib = threadIdx.x >> 5;
+    const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+    uint32_t *buf0 = tiles[wib][0], *buf1 = tiles[wib][1];
+    uint64_t *bar0 = &bars[wib][0], *bar1 = &bars[wib][1];
+    if (lane == 0) {
+        mbar_init(bar0, 1);
+        mbar_init(bar1, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncwarp();
+    uint32_t ph0 = 0, ph1 = 0;
+    const uint32_t kBytes = kTileWords * 4;
+    for (uint32_t u = warp; u < units; u += nwarps) {
+        const uint32_t t = u * 32u + lane;
+        uint32_t j0 = 0xFFFFFFFFu, j1 = 0;
+        if (t < a.W) {
+            walker_draw_range(a.N, a.nl, a.W, t, j0, j1);
+            j0 = max(j0, a.ja);
+            j1 = min(j1, a.jb);
+        }
+        const uint32_t jlo = __reduce_min_sync(0xFFFFFFFFu, j0);
+        const uint32_t jhi = __reduce_max_sync(0xFFFFFFFFu, j1);
+        if (jlo >= jhi) continue;  // warp-uniform
+        uint32_t x = 0, y = 0;
+        if (t < a.W) {
+            x = a.x[t];
+            y = a.y[t];
+        }
+        if (lane == 0) {
+            mbar_expect_tx(bar0, kBytes);
+            tma_load_tile(buf0, &tmap, bar0, (int32_t)(u * 32u), (int32_t)((jlo - a.Jw) * 6u));
+            if (jlo + 1 < jhi) {
+                mbar_expect_tx(bar1, kBytes);
+                tma_load_tile(buf1, &tmap, bar1, (int32_t)(u * 32u), (int32_t)((jlo + 1 - a.Jw) * 6u));
+            }
+        }
+        for (uint32_t j = jlo; j < jhi; j++) {
+            const bool odd = ((j - jlo) & 1u) != 0;
+            uint32_t *buf = odd ? buf1 : buf0;
+            uint64_t *bar = odd ? bar1 : bar0;
+            mbar_wait(bar, odd ? ph1 : ph0);
+            if (odd) ph1 ^= 1u; else ph0 ^= 1u;
+            uint32_t w[6];
+#pragma unroll
+            for (int r = 0; r < 6; r++) w[r] = buf[r * 32 + lane];
+            uint32_t nx = x, ny = y;
+            gg_walk64(w, nx, ny);
+            const bool active = j >= j0 && j < j1;
+            if (active) {
+                x = nx;
+                y = ny;
+                const uint64_t lab = gg_label(x, y, a.m, a.log2m, true);
+                const uint64_t g = (uint64_t)j * a.W + t;
+                if (OUT32)
+                    reinterpret_cast<uint32_t *>(a.out)[g - a.g_origin] = (uint32_t)lab;
+                else
+                    reinterpret_cast<uint64_t *>(a.out)[g - a.g_origin] = lab;
+            }
+            __syncwarp();  // every lane has read this stage
+            if (lane == 0 && j + 2 < jhi) {
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                mbar_expect_tx(bar, kBytes);
+                tma_load_tile(buf, &tmap, bar, (int32_t)(u * 32u), (int32_t)((j + 2 - a.Jw) * 6u));
+            }
+        }
+        if (t < a.W) {
+            a.x[t] = x;
+            a.y[t] = y;
+        }
+    }
+}
+
+static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
+    static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+    static bool tried = false;
+    if (!tried) {
+        tried = true;
+        void *p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) ==
+                cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = (PFN_cuTensorMapEncodeTiled_v12000)p;
+    }
+    return fn;
+}
+
+// 2D map over the SoA window: dim0 = walkers (pitch), dim1 = rows; box 32 x 6.
+static bool make_window_map(CUtensorMap *map, const uint32_t *bits, uint64_t pitch, uint64_t rows) {
+    auto enc = get_encode();
+    if (!enc || rows == 0 || rows > 0x7FFFFFFFull) return false;
+    cuuint64_t dims[2] = {(cuuint64_t)pitch, (cuuint64_t)rows};
+    cuuint64_t strides[1] = {(cuuint64_t)(pitch * 4)};
+    cuuint32_t box[2] = {32, 6};
+    cuuint32_t estr[2] = {1, 1};
+    CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, (void *)bits, dims, strides, box, estr,
+                     CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                     CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    return r == CUDA_SUCCESS;
+}
+
 // Any l, any m (power of two, or <= 2^30): the record is read field by
 // field from global memory.
 __global__ void __launch_bounds__(64) gg_fill_generic_kernel(FillArgs a, uint32_t units) {
@@ -147,9 +301,10 @@ __global__ void __launch_bounds__(64) gg_fill_generic_kernel(FillArgs a, uint32_
 // Grid so that every warp owns the same number k of 32-walker units and the
 // SMs hold <= ~40 warps each (enough to hide the 4-cycle ALU/FMA latency of
 // the step chain several times over).
-static void plan_grid(uint32_t units, int sm_count, uint32_t &blocks, uint32_t &threads) {
+static void plan_grid(uint32_t units, int sm_count, uint32_t warps_per_sm, uint32_t &blocks,
+                      uint32_t &threads) {
     threads = 64;
-    const uint32_t max_warps = (uint32_t)sm_count * 40u;
+    const uint32_t max_warps = (uint32_t)sm_count * warps_per_sm;
     const uint32_t k = (units + max_warps - 1) / max_warps;  // units per warp
     const uint32_t warps = (units + k - 1) / k;
     blocks = (warps + 1) / 2;
@@ -160,12 +315,23 @@ cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count) {
     if (a.jb <= a.ja || a.nl == 0) return cudaSuccess;
     const uint32_t units = (a.W + 31u) / 32u;
     uint32_t blocks, threads;
-    plan_grid(units, sm_count, blocks, threads);
+    plan_grid(units, sm_count, 40, blocks, threads);
     if (a.l == 64 && a.pow2) {
-        if (a.out_u32)
+        CUtensorMap map;
+        static const bool use_tma = getenv("GG_FILL_NO_TMA") == nullptr;
+        if (use_tma && a.rows && make_window_map(&map, a.bits, a.pitch, a.rows)) {
+            // 35 registers, 4 KB smem per 2-warp block: full occupancy (64 warps/SM)
+            static const uint32_t wps = getenv("GG_FILL_WARPS") ? atoi(getenv("GG_FILL_WARPS")) : 64;
+            plan_grid(units, sm_count, wps, blocks, threads);
+            if (a.out_u32)
+                gg_fill64_tma_kernel<1><<<blocks, threads, 0, s>>>(map, a, units);
+            else
+                gg_fill64_tma_kernel<0><<<blocks, threads, 0, s>>>(map, a, units);
+        } else if (a.out_u32) {
             gg_fill64_kernel<1><<<blocks, threads, 0, s>>>(a, units);
-        else
+        } else {
             gg_fill64_kernel<0><<<blocks, threads, 0, s>>>(a, units);
+        }
     } else {
         gg_fill_generic_kernel<<<blocks, threads, 0, s>>>(a, units);
     }

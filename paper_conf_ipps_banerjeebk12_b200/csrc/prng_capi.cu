@@ -265,12 +265,13 @@ int check_fmt(const prng_s *h, uint64_t n, int fmt) {
     return PRNG_OK;
 }
 
-gg::FillArgs fill_args(prng_s *h, const uint32_t *bits, uint64_t pitch, uint64_t Jw, uint64_t ja,
-                       uint64_t jb, uint64_t N, uint64_t nl, uint64_t g_origin, void *out,
-                       int out_u32) {
+gg::FillArgs fill_args(prng_s *h, const uint32_t *bits, uint64_t pitch, uint64_t rows,
+                       uint64_t Jw, uint64_t ja, uint64_t jb, uint64_t N, uint64_t nl,
+                       uint64_t g_origin, void *out, int out_u32) {
     gg::FillArgs a{};
     a.bits = bits;
     a.pitch = pitch;
+    a.rows = rows;
     a.Jw = (uint32_t)Jw;
     a.ja = (uint32_t)ja;
     a.jb = (uint32_t)jb;
@@ -302,7 +303,7 @@ void run_pieces(prng_s *h, uint64_t N, uint64_t nl, cudaStream_t s, Emit emit) {
     while (j < jhi) {
         if (h->res_bits && j >= h->res_J && j < h->res_J + h->res_D) {
             const uint64_t jb = std::min(jhi, h->res_J + h->res_D);
-            emit(j, jb, h->res_bits, pitch, h->res_J, s);
+            emit(j, jb, h->res_bits, pitch, h->res_D * h->R, h->res_J, s);
             j = jb;
             continue;
         }
@@ -324,7 +325,7 @@ void run_pieces(prng_s *h, uint64_t N, uint64_t nl, cudaStream_t s, Emit emit) {
         CK(cudaStreamWaitEvent(h->copy_stream, h->ring_free[slot], 0));  // slot no longer read
         stage_rows(h, 2 + h->R0 + h->R * j, (jb - j) * h->R, W, h->ring[slot], pitch);
         join_copies(h, s);
-        emit(j, jb, h->ring[slot], pitch, j, s);
+        emit(j, jb, h->ring[slot], pitch, (jb - j) * h->R, j, s);
         CK(cudaEventRecord(h->ring_free[slot], s));
         j = jb;
     }
@@ -505,10 +506,10 @@ int prng_fill(prng_t *h, void *dev_ptr, uint64_t n, int fmt, void *stream) {
         const int out_u32 = (fmt == PRNG_FMT_U32 && h->g.m <= 65536ull) ? 1 : 0;
         const uint64_t N = h->N;
         run_pieces(h, N, nl, s,
-                   [&](uint64_t ja, uint64_t jb, const uint32_t *bits, uint64_t pitch, uint64_t Jw,
-                       cudaStream_t st) {
-                       gg::FillArgs a =
-                           fill_args(h, bits, pitch, Jw, ja, jb, N, nl, N, dev_ptr, out_u32);
+                   [&](uint64_t ja, uint64_t jb, const uint32_t *bits, uint64_t pitch,
+                       uint64_t rows, uint64_t Jw, cudaStream_t st) {
+                       gg::FillArgs a = fill_args(h, bits, pitch, rows, Jw, ja, jb, N, nl, N,
+                                                  dev_ptr, out_u32);
                        CK(gg::launch_fill(a, st, h->sm_count));
                        h->stats.kernel_launches++;
                    });
@@ -545,8 +546,8 @@ int prng_fill_host(prng_t *h, void *host_ptr, uint64_t n, int fmt) {
         char *dst = (char *)host_ptr;
         cudaStream_t s = h->work_stream;
         run_pieces(h, N, nl, s,
-                   [&](uint64_t ja, uint64_t jb, const uint32_t *bits, uint64_t pitch, uint64_t Jw,
-                       cudaStream_t st) {
+                   [&](uint64_t ja, uint64_t jb, const uint32_t *bits, uint64_t pitch,
+                       uint64_t rows, uint64_t Jw, cudaStream_t st) {
                        // a resident window may span many ring slots' worth: split
                        for (uint64_t a0 = ja; a0 < jb; a0 += Ds) {
                            const uint64_t a1 = std::min(jb, a0 + Ds);
@@ -554,8 +555,8 @@ int prng_fill_host(prng_t *h, void *host_ptr, uint64_t n, int fmt) {
                            const uint64_t gB = std::min(N + nl, a1 * h->W);
                            if (gB <= gA) continue;
                            CK(cudaStreamWaitEvent(st, h->hout_free[oslot], 0));
-                           gg::FillArgs a = fill_args(h, bits, pitch, Jw, a0, a1, N, nl, gA,
-                                                      h->hout[oslot], out_u32);
+                           gg::FillArgs a = fill_args(h, bits, pitch, rows, Jw, a0, a1, N, nl,
+                                                      gA, h->hout[oslot], out_u32);
                            CK(gg::launch_fill(a, st, h->sm_count));
                            h->stats.kernel_launches++;
                            CK(cudaEventRecord(h->ev_tmp, st));

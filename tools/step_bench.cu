@@ -88,6 +88,59 @@ __device__ __forceinline__ void walk64(const uint32_t w[6], uint32_t &x, uint32_
   word10<V,10>(__funnelshift_r(w[4], w[5], 22), x, y, four);
   word10<V,4>(w[5] >> 20, x, y, four);
 }
+template <int V, int NK>
+__device__ __forceinline__ void word10x2(uint32_t Qa, uint32_t Qb, uint32_t &xa, uint32_t &ya,
+                                         uint32_t &xb, uint32_t &yb, uint32_t four) {
+  const uint32_t f1a = Qa >> 1, f2a = Qa >> 2, f1b = Qb >> 1, f2b = Qb >> 2;
+  const uint32_t MYa = ~f2a & (f1a | Qa), MXa = f2a & ~(f1a & Qa), Ca = Qa - (MYa & 0x09249249u);
+  const uint32_t MYb = ~f2b & (f1b | Qb), MXb = f2b & ~(f1b & Qb), Cb = Qb - (MYb & 0x09249249u);
+#define S2(k) if (NK > k) { step<V, k>(MYa, MXa, Ca, xa, ya, four); step<V, k>(MYb, MXb, Cb, xb, yb, four); }
+  S2(0) S2(1) S2(2) S2(3) S2(4) S2(5) S2(6) S2(7) S2(8) S2(9)
+#undef S2
+}
+template <int V>
+__device__ __forceinline__ void walk64x2(const uint32_t a[6], const uint32_t b[6], uint32_t &xa, uint32_t &ya,
+                                         uint32_t &xb, uint32_t &yb, uint32_t four) {
+  word10x2<V,10>(a[0], b[0], xa, ya, xb, yb, four);
+  word10x2<V,10>(__funnelshift_r(a[0], a[1], 30), __funnelshift_r(b[0], b[1], 30), xa, ya, xb, yb, four);
+  word10x2<V,10>(__funnelshift_r(a[1], a[2], 28), __funnelshift_r(b[1], b[2], 28), xa, ya, xb, yb, four);
+  word10x2<V,10>(__funnelshift_r(a[2], a[3], 26), __funnelshift_r(b[2], b[3], 26), xa, ya, xb, yb, four);
+  word10x2<V,10>(__funnelshift_r(a[3], a[4], 24), __funnelshift_r(b[3], b[4], 24), xa, ya, xb, yb, four);
+  word10x2<V,10>(__funnelshift_r(a[4], a[5], 22), __funnelshift_r(b[4], b[5], 22), xa, ya, xb, yb, four);
+  word10x2<V,4>(a[5] >> 20, b[5] >> 20, xa, ya, xb, yb, four);
+}
+// two walkers per thread (t and t+32 of a 64-walker unit), interleaved step by step
+template <int V>
+__global__ void __launch_bounds__(64) kfill2(const uint32_t* __restrict__ bits, uint64_t pitch, uint32_t W, uint32_t D,
+                                             uint32_t* xs, uint32_t* ys, uint64_t* out, uint32_t units, uint32_t four) {
+  const uint32_t lane = threadIdx.x & 31u, warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+  for (uint32_t u = warp; u < units / 2; u += nwarps) {
+    const uint32_t ta = u * 64u + lane, tb = ta + 32u;
+    uint32_t xa = xs[ta], ya = ys[ta], xb = xs[tb], yb = ys[tb];
+    uint32_t a0[6], b0[6], a1[6], b1[6];
+#pragma unroll
+    for (int r = 0; r < 6; r++) {
+      a0[r] = __ldg(bits + ta + (uint64_t)r * pitch); b0[r] = __ldg(bits + tb + (uint64_t)r * pitch);
+      a1[r] = __ldg(bits + ta + (uint64_t)(6 + r) * pitch); b1[r] = __ldg(bits + tb + (uint64_t)(6 + r) * pitch);
+    }
+    for (uint32_t j = 0; j < D; j++) {
+      uint32_t a2[6], b2[6];
+      const uint32_t jn = (j + 2 < D) ? j + 2 : j;
+#pragma unroll
+      for (int r = 0; r < 6; r++) {
+        a2[r] = __ldg(bits + ta + ((uint64_t)jn * 6 + r) * pitch);
+        b2[r] = __ldg(bits + tb + ((uint64_t)jn * 6 + r) * pitch);
+      }
+      walk64x2<V>(a0, b0, xa, ya, xb, yb, four);
+      out[(uint64_t)j * W + ta] = ((uint64_t)ya << 32) | xa;
+      out[(uint64_t)j * W + tb] = ((uint64_t)yb << 32) | xb;
+#pragma unroll
+      for (int r = 0; r < 6; r++) { a0[r] = a1[r]; a1[r] = a2[r]; b0[r] = b1[r]; b1[r] = b2[r]; }
+    }
+    xs[ta] = xa; ys[ta] = ya; xs[tb] = xb; ys[tb] = yb;
+  }
+}
 template <int V>
 __global__ void __launch_bounds__(64) kfill(const uint32_t* __restrict__ bits, uint64_t pitch, uint32_t W, uint32_t D,
                                             uint32_t* xs, uint32_t* ys, uint64_t* out, uint32_t units, uint32_t four) {
@@ -97,19 +150,18 @@ __global__ void __launch_bounds__(64) kfill(const uint32_t* __restrict__ bits, u
     const uint32_t t = u * 32u + lane;
     uint32_t x = xs[t], y = ys[t];
     const uint32_t* col = bits + t;
-    uint32_t w[6];
+    uint32_t w[6], w1[6];
 #pragma unroll
-    for (int r = 0; r < 6; r++) w[r] = __ldg(col + (uint64_t)r * pitch);
+    for (int r = 0; r < 6; r++) { w[r] = __ldg(col + (uint64_t)r * pitch); w1[r] = __ldg(col + (uint64_t)(6 + r) * pitch); }
     for (uint32_t j = 0; j < D; j++) {
       uint32_t wn[6];
-      if (j + 1 < D) {
+      const uint32_t jn = (j + 2 < D) ? j + 2 : j;
 #pragma unroll
-        for (int r = 0; r < 6; r++) wn[r] = __ldg(col + ((uint64_t)(j + 1) * 6 + r) * pitch);
-      }
+      for (int r = 0; r < 6; r++) wn[r] = __ldg(col + ((uint64_t)jn * 6 + r) * pitch);
       walk64<V>(w, x, y, four);
       out[(uint64_t)j * W + t] = ((uint64_t)y << 32) | x;
 #pragma unroll
-      for (int r = 0; r < 6; r++) w[r] = wn[r];
+      for (int r = 0; r < 6; r++) { w[r] = w1[r]; w1[r] = wn[r]; }
     }
     xs[t] = x; ys[t] = y;
   }
@@ -143,6 +195,27 @@ float run(const uint32_t* bits, uint64_t pitch, uint32_t W, uint32_t D, uint32_t
   float ms; cudaEventElapsedTime(&ms, a, b);
   return ms / reps;
 }
+template <int V>
+float run2(const uint32_t* bits, uint64_t pitch, uint32_t W, uint32_t D, uint32_t* xs, uint32_t* ys, uint64_t* out,
+           int warps_per_sm, int reps) {
+  uint32_t units = W / 32;
+  uint32_t max_warps = 148u * warps_per_sm;
+  uint32_t k = (units / 2 + max_warps - 1) / max_warps;
+  uint32_t warps = (units / 2 + k - 1) / k;
+  uint32_t blocks = (warps + 1) / 2;
+  cudaEvent_t a, b; cudaEventCreate(&a); cudaEventCreate(&b);
+  kinit<<<1184, 256>>>(xs, W); kinit<<<1184, 256>>>(ys, W);
+  kfill2<V><<<blocks, 64>>>(bits, pitch, W, D, xs, ys, out, units, 4u);
+  kinit<<<1184, 256>>>(xs, W); kinit<<<1184, 256>>>(ys, W);
+  cudaEventRecord(a);
+  for (int r = 0; r < reps; r++) {
+    kinit<<<1, 32>>>(xs, 0);
+    kfill2<V><<<blocks, 64>>>(bits, pitch, W, D, xs, ys, out, units, 4u);
+  }
+  cudaEventRecord(b); cudaEventSynchronize(b);
+  float ms; cudaEventElapsedTime(&ms, a, b);
+  return ms / reps;
+}
 int main() {
   const uint32_t W = 1u << 20, D = 128;
   const uint64_t pitch = W;
@@ -153,6 +226,14 @@ int main() {
   kinit<<<4096, 256>>>(bits, (uint64_t)D * 6 * pitch);
   std::vector<uint64_t> ref(4096), got(4096);
   double labels = (double)W * D;
+  for (int wps : {12, 16, 20, 24, 32}) {
+    float t0 = run<6>(bits, pitch, W, D, xs, ys, out, 2 * wps, 3);
+    cudaMemcpy(ref.data(), out + (size_t)(D - 1) * W, 4096 * 8, cudaMemcpyDeviceToHost);
+    float t2 = run2<6>(bits, pitch, W, D, xs, ys, out, wps, 3);
+    cudaMemcpy(got.data(), out + (size_t)(D - 1) * W, 4096 * 8, cudaMemcpyDeviceToHost);
+    printf("x2 warps/SM %d: V6x1 %.3f ms (%.1f G/s)  V6x2 %.3f ms (%.1f G/s) %s\n", wps, t0, labels / t0 / 1e6, t2,
+           labels / t2 / 1e6, got == ref ? "ok" : "MISMATCH");
+  }
   for (int wps : {24, 32, 40, 48}) {
     float t0 = run<0>(bits, pitch, W, D, xs, ys, out, wps, 3);
     cudaMemcpy(ref.data(), out + (size_t)(D - 1) * W, 4096 * 8, cudaMemcpyDeviceToHost);
