@@ -248,6 +248,11 @@ def run_ours(args, rank, world, local_rank):
         g.close()
         torch.cuda.empty_cache()
 
+    # ---- on-demand consumers of the paper at full size (C3, C4), one run each
+    if not args.no_apps:
+        res["apps"] = run_apps(args, rank, world, local_rank, max_over_ranks)
+        torch.cuda.empty_cache()
+
     # ---- e2e: host buffers through prng_fill_host (FEED + H2D + walk + D2H)
     if not args.no_e2e:
         e2e_steps = max(1, min(args.steps, args.e2e_steps))
@@ -279,6 +284,66 @@ def run_ours(args, rank, world, local_rank):
     return res
 
 
+def run_apps(args, rank, world, local_rank, max_over_ranks):
+    """C3 list ranking (2^24 nodes, replica per GPU) and C4 Monte Carlo (2^20
+    threads per GPU, 20 photons each, ~2^32 draws per GPU; integer tallies
+    all-reduced over ranks).  Numbers are device-timed inside the C ABI."""
+    import torch
+
+    import inputs
+    from paper_conf_ipps_banerjeebk12_b200 import Generator
+    dev = torch.device("cuda", local_rank)
+    out = {}
+    # C3: list ranking of a 2^24-node random list (every rank ranks its own copy)
+    n = 1 << 24
+    succ, pred, head = inputs.random_list(n, 0x5EED0003)
+    g = Generator(walkers=n, seed=0x5EED0003, device=local_rank)
+    s_t, p_t = torch.from_numpy(succ).to(dev), torch.from_numpy(pred).to(dev)
+    torch.cuda.synchronize()
+    t = time.perf_counter()
+    rank_t, info = g.list_rank(s_t, p_t, head)
+    torch.cuda.synchronize()
+    wall = max_over_ranks(time.perf_counter() - t)
+    ok = int(rank_t[head].item()) == 0 and int(rank_t.max().item()) == n - 1
+    dev_us = info["phase1_us"] + info["phase2_us"] + info["phase3_us"]
+    out["list_ranking"] = {
+        "config": "C3: random list of 2^24 nodes, walker = active slot, b(u) = bit 63",
+        "rounds": info["rounds"], "reduced": info["reduced"], "splitters": info["splitters"],
+        "draws": info["draws"], "ms_device": dev_us / 1e3, "ms_wall": wall * 1e3,
+        "phase_ms": [info["phase1_us"] / 1e3, info["phase2_us"] / 1e3, info["phase3_us"] / 1e3],
+        "draws_per_s_e2e": info["draws"] / wall / 1e9, "unit": "GNumbers/s",
+        "ranks_ok": ok,
+        "note": "on-demand: the host feeds exactly the draws of each round after learning the "
+                "active count (FEED + H2D inside the measured time)"}
+    g.close()
+    del s_t, p_t, rank_t
+    torch.cuda.empty_cache()
+    # C4: Monte Carlo photon migration, R19 slab
+    from paper_conf_ipps_banerjeebk12_b200 import dist as gd
+    thread0, T, T_total = gd.mc_shard(rank, world, W_PER_GPU)
+    P_per = 20
+    g = Generator(walkers=T, seed=0x5EED0004, walker_base=thread0, device=local_rank)
+    layers = ((1.37, 1.0, 100.0, 0.9, 0.1), (1.37, 1.0, 10.0, 0.0, 0.1), (1.37, 2.0, 10.0, 0.7, 0.2))
+    torch.cuda.synchronize()
+    t = time.perf_counter()
+    r = g.mc_run(layers, photons_total=P_per * T_total, threads=T, threads_total=T_total,
+                 thread0=thread0, epoch_draws=192)
+    wall = max_over_ranks(time.perf_counter() - t)
+    tal = gd.allreduce_tallies(r["tallies"], device=dev)  # exact int64 sums (NCCL over NVLink)
+    draws = r["draws"] * world
+    kern = max_over_ranks(r["kernel_us"] / 1e6)
+    out["monte_carlo"] = {
+        "config": "C4: R19 3-layer slab, 2^20 threads/GPU x 20 photons, 3 draws per iteration",
+        "photons": P_per * T * world, "draws": draws, "epochs": r["epochs"],
+        "draws_per_s_kernel": draws / kern / 1e9, "draws_per_s_e2e": draws / wall / 1e9,
+        "unit": "GNumbers/s", "ms_wall": wall * 1e3, "ms_kernel": kern * 1e3,
+        "R_d": tal[2] / tal[0], "T_t": tal[3] / tal[0], "specular": tal[1] / tal[0],
+        "absorbed": [v / tal[0] for v in tal[5:]], "conserved": tal[0] == sum(tal[1:]),
+        "host_bits_GB": draws * BITS_BYTES_PER_LABEL / 1e9}
+    g.close()
+    return out
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -288,6 +353,7 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-ondemand", action="store_true")
+    ap.add_argument("--no-apps", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=8.0)
     args = ap.parse_args()
@@ -328,7 +394,7 @@ def main():
                        "parallelism": f"walker shards dp{world}, no data-path collective"},
             "roofline": res["roofline"], "cpu_baseline": cpu, "e2e": res.get("e2e"),
             "clocks": res["clocks"], "gpu_launches": res["launches"],
-            "on_demand": res.get("on_demand"),
+            "on_demand": res.get("on_demand"), "apps": res.get("apps"),
         }
         print(json.dumps(line))
     if world > 1:

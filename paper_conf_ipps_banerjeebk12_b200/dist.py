@@ -1,0 +1,46 @@
+"""Multi-GPU plumbing: walker shards and the one collective the path needs.
+
+One process per GPU (torch.distributed, NCCL over NVLink on the GPU box,
+gloo in the CPU tests).  The generator shards naturally: GPU r owns global
+walkers [r*W, (r+1)*W) and therefore disjoint seed-bit streams (reading R9:
+a walker's stream depends only on its global id), so bulk generation needs
+no communication and the union over GPUs equals the one-GPU output walker by
+walker (§I-B: "Each thread performing the walk is essentially executing
+independent of other threads").  The Monte Carlo consumer (§VI) sums
+integer fixed-point tallies across GPUs with one all-reduce; sums of int64
+are exact and order independent, so the sharded result equals the one-GPU
+result bit for bit.
+"""
+from __future__ import annotations
+
+
+def walker_shard(rank: int, world: int, walkers_per_rank: int):
+    """(walker_base, walkers) of rank `rank` for weak scaling (fixed walkers per GPU)."""
+    if not 0 <= rank < world:
+        raise ValueError("rank out of range")
+    return rank * walkers_per_rank, walkers_per_rank
+
+
+def global_bulk_index(rank: int, world: int, walkers_per_rank: int, local_index):
+    """Map a shard's local bulk position g = j*W + t to the position of the same
+    (walker, draw) in the one-GPU sequence over W*world walkers (reading R11)."""
+    W = walkers_per_rank
+    j = local_index // W
+    t = local_index % W
+    return j * (W * world) + rank * W + t
+
+
+def mc_shard(rank: int, world: int, threads_per_rank: int):
+    """(thread0, threads, threads_total) for gg_mc_run on rank `rank`."""
+    base, n = walker_shard(rank, world, threads_per_rank)
+    return base, n, threads_per_rank * world
+
+
+def allreduce_tallies(tallies, group=None, device=None):
+    """Exact integer sum of Monte Carlo tallies over all ranks (SUM all-reduce)."""
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor(list(tallies), dtype=torch.int64, device=device)
+    if dist.is_available() and dist.is_initialized() and dist.get_world_size(group) > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)
+    return [int(v) for v in t.cpu().tolist()]
