@@ -97,10 +97,12 @@ template <int NK>
 __device__ __forceinline__ void gg_word10(uint32_t Q, uint32_t &x, uint32_t &y)
 {
     const uint32_t f1 = Q >> 1, f2 = Q >> 2;
-    const uint32_t MY = ~f2 & (f1 | Q);   /* b2=0 and b != 0 */
-    const uint32_t MX = f2 & ~(f1 & Q);   /* b2=1 and b != 7 */
-    /* y-move fields hold b-1 (no borrow: b>=1); MY is masked to the fields' LSBs */
-    const uint32_t C = Q - (MY & 0x09249249u);
+    /* MY: b2=0 and b != 0, kept only at the fields' LSBs (it is subtracted
+     * below); MX: b2=1 and b != 7 (only its LSB bits are ever tested) */
+    const uint32_t MY = ((f1 | Q) & 0x09249249u) & ~f2;
+    const uint32_t MX = f2 & ~(f1 & Q);
+    /* y-move fields hold b-1 (no borrow: b>=1) */
+    const uint32_t C = Q - MY;
     if (NK > 0) gg_step_swar<0>(MY, MX, C, x, y);
     if (NK > 1) gg_step_swar<1>(MY, MX, C, x, y);
     if (NK > 2) gg_step_swar<2>(MY, MX, C, x, y);
@@ -132,6 +134,37 @@ __device__ __forceinline__ uint32_t gg_ldg_early(const uint32_t *p)
     uint32_t v;
     asm volatile("ld.global.nc.L1::no_allocate.u32 %0, [%1];" : "=r"(v) : "l"(p));
     return v;
+}
+
+/* Two independent walkers interleaved step by step (more ILP per warp:
+ * the scheduler always has an instruction of the other walker ready). */
+template <int NK>
+__device__ __forceinline__ void gg_word10x2(uint32_t Qa, uint32_t Qb, uint32_t &xa, uint32_t &ya,
+                                            uint32_t &xb, uint32_t &yb)
+{
+    const uint32_t f1a = Qa >> 1, f2a = Qa >> 2, f1b = Qb >> 1, f2b = Qb >> 2;
+    const uint32_t MYa = ((f1a | Qa) & 0x09249249u) & ~f2a, MXa = f2a & ~(f1a & Qa);
+    const uint32_t MYb = ((f1b | Qb) & 0x09249249u) & ~f2b, MXb = f2b & ~(f1b & Qb);
+    const uint32_t Ca = Qa - MYa, Cb = Qb - MYb;
+#define GG_S2(k)                                               \
+    if (NK > k) {                                              \
+        gg_step_swar<k>(MYa, MXa, Ca, xa, ya);                 \
+        gg_step_swar<k>(MYb, MXb, Cb, xb, yb);                 \
+    }
+    GG_S2(0) GG_S2(1) GG_S2(2) GG_S2(3) GG_S2(4) GG_S2(5) GG_S2(6) GG_S2(7) GG_S2(8) GG_S2(9)
+#undef GG_S2
+}
+
+__device__ __forceinline__ void gg_walk64x2(const uint32_t a[6], const uint32_t b[6], uint32_t &xa,
+                                            uint32_t &ya, uint32_t &xb, uint32_t &yb)
+{
+    gg_word10x2<10>(a[0], b[0], xa, ya, xb, yb);
+    gg_word10x2<10>(__funnelshift_r(a[0], a[1], 30), __funnelshift_r(b[0], b[1], 30), xa, ya, xb, yb);
+    gg_word10x2<10>(__funnelshift_r(a[1], a[2], 28), __funnelshift_r(b[1], b[2], 28), xa, ya, xb, yb);
+    gg_word10x2<10>(__funnelshift_r(a[2], a[3], 26), __funnelshift_r(b[2], b[3], 26), xa, ya, xb, yb);
+    gg_word10x2<10>(__funnelshift_r(a[3], a[4], 24), __funnelshift_r(b[3], b[4], 24), xa, ya, xb, yb);
+    gg_word10x2<10>(__funnelshift_r(a[4], a[5], 22), __funnelshift_r(b[4], b[5], 22), xa, ya, xb, yb);
+    gg_word10x2<4>(a[5] >> 20, b[5] >> 20, xa, ya, xb, yb);
 }
 
 /* One step, any m (generic path).  Non power-of-two m requires m <= 2^30 and

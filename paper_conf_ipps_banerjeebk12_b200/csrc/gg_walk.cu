@@ -161,8 +161,23 @@ __device__ __forceinline__ void tma_load_tile(uint32_t *dst, const CUtensorMap *
 constexpr int kTileWords = 6 * 32;  // one draw record for 32 walkers
 constexpr int kFillWarps = 2;       // warps per block
 
-template <int OUT32>
-__global__ void __launch_bounds__(64) gg_fill64_tma_kernel(const __grid_constant__ CUtensorMap tmap,
+// EMIT: 0 = u64 label, m = 2^32 ((y << 32) | x, no masking); 1 = u64 label,
+// m = 2^k < 2^32; 2 = low u32 word of the label (m <= 2^16).
+template <int EMIT>
+__device__ __forceinline__ void emit_label(const FillArgs &a, uint64_t idx, uint32_t x, uint32_t y) {
+    if (EMIT == 0) {
+        reinterpret_cast<uint2 *>(a.out)[idx] = make_uint2(x, y);
+    } else {
+        const uint64_t lab = gg_label(x, y, a.m, a.log2m, true);
+        if (EMIT == 2)
+            reinterpret_cast<uint32_t *>(a.out)[idx] = (uint32_t)lab;
+        else
+            reinterpret_cast<uint64_t *>(a.out)[idx] = lab;
+    }
+}
+
+template <int EMIT>
+__global__ void __launch_bounds__(64, 32) gg_fill64_tma_kernel(const __grid_constant__ CUtensorMap tmap,
                                                            FillArgs a, uint32_t units) {
     __shared__ __align__(128) uint32_t tiles[kFillWarps][2][kTileWords];
     __shared__ __align__(8) uint64_t bars[kFillWarps][2];
@@ -218,12 +233,7 @@ __global__ void __launch_bounds__(64) gg_fill64_tma_kernel(const __grid_constant
             if (active) {
                 x = nx;
                 y = ny;
-                const uint64_t lab = gg_label(x, y, a.m, a.log2m, true);
-                const uint64_t g = (uint64_t)j * a.W + t;
-                if (OUT32)
-                    reinterpret_cast<uint32_t *>(a.out)[g - a.g_origin] = (uint32_t)lab;
-                else
-                    reinterpret_cast<uint64_t *>(a.out)[g - a.g_origin] = lab;
+                emit_label<EMIT>(a, (uint64_t)j * a.W + t - a.g_origin, x, y);
             }
             __syncwarp();  // every lane has read this stage
             if (lane == 0 && j + 2 < jhi) {
@@ -235,6 +245,103 @@ __global__ void __launch_bounds__(64) gg_fill64_tma_kernel(const __grid_constant
         if (t < a.W) {
             a.x[t] = x;
             a.y[t] = y;
+        }
+    }
+}
+
+// Two walkers per lane: a warp owns 64 walkers (u*64 + lane, u*64 + 32 +
+// lane); one TMA box of 64 x 6 words (1.5 KB) per draw; the two walks are
+// interleaved step by step.
+template <int EMIT>
+__global__ void __launch_bounds__(64) gg_fill64x2_tma_kernel(const __grid_constant__ CUtensorMap tmap,
+                                                         FillArgs a, uint32_t units64) {
+    constexpr int kTile = 6 * 64;
+    __shared__ __align__(128) uint32_t tiles[kFillWarps][2][kTile];
+    __shared__ __align__(8) uint64_t bars[kFillWarps][2];
+    const uint32_t lane = threadIdx.x & 31u, wib = threadIdx.x >> 5;
+    const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+    uint32_t *buf0 = tiles[wib][0], *buf1 = tiles[wib][1];
+    uint64_t *bar0 = &bars[wib][0], *bar1 = &bars[wib][1];
+    if (lane == 0) {
+        mbar_init(bar0, 1);
+        mbar_init(bar1, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncwarp();
+    uint32_t ph0 = 0, ph1 = 0;
+    const uint32_t kBytes = kTile * 4;
+    for (uint32_t u = warp; u < units64; u += nwarps) {
+        const uint32_t ta = u * 64u + lane, tb = ta + 32u;
+        uint32_t ja0 = 0xFFFFFFFFu, ja1 = 0, jb0 = 0xFFFFFFFFu, jb1 = 0;
+        if (ta < a.W) {
+            walker_draw_range(a.N, a.nl, a.W, ta, ja0, ja1);
+            ja0 = max(ja0, a.ja);
+            ja1 = min(ja1, a.jb);
+        }
+        if (tb < a.W) {
+            walker_draw_range(a.N, a.nl, a.W, tb, jb0, jb1);
+            jb0 = max(jb0, a.ja);
+            jb1 = min(jb1, a.jb);
+        }
+        const uint32_t jlo = __reduce_min_sync(0xFFFFFFFFu, min(ja0, jb0));
+        const uint32_t jhi = __reduce_max_sync(0xFFFFFFFFu, max(ja1, jb1));
+        if (jlo >= jhi) continue;
+        uint32_t xa = 0, ya = 0, xb = 0, yb = 0;
+        if (ta < a.W) {
+            xa = a.x[ta];
+            ya = a.y[ta];
+        }
+        if (tb < a.W) {
+            xb = a.x[tb];
+            yb = a.y[tb];
+        }
+        if (lane == 0) {
+            mbar_expect_tx(bar0, kBytes);
+            tma_load_tile(buf0, &tmap, bar0, (int32_t)(u * 64u), (int32_t)((jlo - a.Jw) * 6u));
+            if (jlo + 1 < jhi) {
+                mbar_expect_tx(bar1, kBytes);
+                tma_load_tile(buf1, &tmap, bar1, (int32_t)(u * 64u), (int32_t)((jlo + 1 - a.Jw) * 6u));
+            }
+        }
+        for (uint32_t j = jlo; j < jhi; j++) {
+            const bool odd = ((j - jlo) & 1u) != 0;
+            uint32_t *buf = odd ? buf1 : buf0;
+            uint64_t *bar = odd ? bar1 : bar0;
+            mbar_wait(bar, odd ? ph1 : ph0);
+            if (odd) ph1 ^= 1u; else ph0 ^= 1u;
+            uint32_t wa[6], wb[6];
+#pragma unroll
+            for (int r = 0; r < 6; r++) {
+                wa[r] = buf[r * 64 + lane];
+                wb[r] = buf[r * 64 + 32 + lane];
+            }
+            uint32_t nxa = xa, nya = ya, nxb = xb, nyb = yb;
+            gg_walk64x2(wa, wb, nxa, nya, nxb, nyb);
+            if (j >= ja0 && j < ja1) {
+                xa = nxa;
+                ya = nya;
+                emit_label<EMIT>(a, (uint64_t)j * a.W + ta - a.g_origin, xa, ya);
+            }
+            if (j >= jb0 && j < jb1) {
+                xb = nxb;
+                yb = nyb;
+                emit_label<EMIT>(a, (uint64_t)j * a.W + tb - a.g_origin, xb, yb);
+            }
+            __syncwarp();
+            if (lane == 0 && j + 2 < jhi) {
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                mbar_expect_tx(bar, kBytes);
+                tma_load_tile(buf, &tmap, bar, (int32_t)(u * 64u), (int32_t)((j + 2 - a.Jw) * 6u));
+            }
+        }
+        if (ta < a.W) {
+            a.x[ta] = xa;
+            a.y[ta] = ya;
+        }
+        if (tb < a.W) {
+            a.x[tb] = xb;
+            a.y[tb] = yb;
         }
     }
 }
@@ -255,12 +362,13 @@ static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
 }
 
 // 2D map over the SoA window: dim0 = walkers (pitch), dim1 = rows; box 32 x 6.
-static bool make_window_map(CUtensorMap *map, const uint32_t *bits, uint64_t pitch, uint64_t rows) {
+static bool make_window_map(CUtensorMap *map, const uint32_t *bits, uint64_t pitch, uint64_t rows,
+                            uint32_t box_walkers = 32) {
     auto enc = get_encode();
     if (!enc || rows == 0 || rows > 0x7FFFFFFFull) return false;
     cuuint64_t dims[2] = {(cuuint64_t)pitch, (cuuint64_t)rows};
     cuuint64_t strides[1] = {(cuuint64_t)(pitch * 4)};
-    cuuint32_t box[2] = {32, 6};
+    cuuint32_t box[2] = {box_walkers, 6};
     cuuint32_t estr[2] = {1, 1};
     CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, (void *)bits, dims, strides, box, estr,
                      CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
@@ -298,16 +406,28 @@ __global__ void __launch_bounds__(64) gg_fill_generic_kernel(FillArgs a, uint32_
     }
 }
 
-// Grid so that every warp owns the same number k of 32-walker units and the
-// SMs hold <= ~40 warps each (enough to hide the 4-cycle ALU/FMA latency of
-// the step chain several times over).
-static void plan_grid(uint32_t units, int sm_count, uint32_t warps_per_sm, uint32_t &blocks,
-                      uint32_t &threads) {
+// One full wave: as many 64-thread blocks as can be resident on every SM at
+// once (occupancy API for the actual kernel), never more than the units need.
+// Units (32 walkers) go round-robin over all warps, so every SM gets the same
+// number of units +-1 and there is no partially filled second wave.
+template <class K>
+static void plan_grid(K kernel, uint32_t units, int sm_count, uint32_t &blocks, uint32_t &threads) {
     threads = 64;
-    const uint32_t max_warps = (uint32_t)sm_count * warps_per_sm;
-    const uint32_t k = (units + max_warps - 1) / max_warps;  // units per warp
-    const uint32_t warps = (units + k - 1) / k;
-    blocks = (warps + 1) / 2;
+    int per_sm = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, (int)threads, 0) !=
+            cudaSuccess ||
+        per_sm <= 0)
+        per_sm = 16;
+    static const int bps_env = getenv("GG_FILL_BPS") ? atoi(getenv("GG_FILL_BPS")) : 0;
+    if (bps_env > 0 && bps_env < per_sm) per_sm = bps_env;
+    const uint32_t cap = (uint32_t)sm_count * (uint32_t)per_sm;
+    const uint32_t need = (units + 1) / 2;  // 2 warps per block, >= 1 unit per warp
+    blocks = need < cap ? need : cap;
+    static const int kpw = getenv("GG_FILL_KPW") ? atoi(getenv("GG_FILL_KPW")) : 0;
+    if (kpw > 0) {  // experiment: exactly kpw units per warp (may exceed one wave)
+        const uint32_t warps = (units + kpw - 1) / kpw;
+        blocks = (warps + 1) / 2;
+    }
     if (blocks == 0) blocks = 1;
 }
 
@@ -315,24 +435,42 @@ cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count) {
     if (a.jb <= a.ja || a.nl == 0) return cudaSuccess;
     const uint32_t units = (a.W + 31u) / 32u;
     uint32_t blocks, threads;
-    plan_grid(units, sm_count, 40, blocks, threads);
     if (a.l == 64 && a.pow2) {
         CUtensorMap map;
         static const bool use_tma = getenv("GG_FILL_NO_TMA") == nullptr;
-        if (use_tma && a.rows && make_window_map(&map, a.bits, a.pitch, a.rows)) {
-            // 35 registers, 4 KB smem per 2-warp block: full occupancy (64 warps/SM)
-            static const uint32_t wps = getenv("GG_FILL_WARPS") ? atoi(getenv("GG_FILL_WARPS")) : 64;
-            plan_grid(units, sm_count, wps, blocks, threads);
-            if (a.out_u32)
-                gg_fill64_tma_kernel<1><<<blocks, threads, 0, s>>>(map, a, units);
-            else
+        static const bool use_x2 = getenv("GG_FILL_X1") == nullptr;
+        const uint32_t units64 = (a.W + 63u) / 64u;
+        if (use_tma && use_x2 && a.rows && make_window_map(&map, a.bits, a.pitch, a.rows, 64)) {
+            if (a.out_u32) {
+                plan_grid(gg_fill64x2_tma_kernel<2>, units64 * 2, sm_count, blocks, threads);
+                gg_fill64x2_tma_kernel<2><<<blocks, threads, 0, s>>>(map, a, units64);
+            } else if (a.log2m == 32) {
+                plan_grid(gg_fill64x2_tma_kernel<0>, units64 * 2, sm_count, blocks, threads);
+                gg_fill64x2_tma_kernel<0><<<blocks, threads, 0, s>>>(map, a, units64);
+            } else {
+                plan_grid(gg_fill64x2_tma_kernel<1>, units64 * 2, sm_count, blocks, threads);
+                gg_fill64x2_tma_kernel<1><<<blocks, threads, 0, s>>>(map, a, units64);
+            }
+        } else if (use_tma && a.rows && make_window_map(&map, a.bits, a.pitch, a.rows)) {
+            if (a.out_u32) {
+                plan_grid(gg_fill64_tma_kernel<2>, units, sm_count, blocks, threads);
+                gg_fill64_tma_kernel<2><<<blocks, threads, 0, s>>>(map, a, units);
+            } else if (a.log2m == 32) {
+                plan_grid(gg_fill64_tma_kernel<0>, units, sm_count, blocks, threads);
                 gg_fill64_tma_kernel<0><<<blocks, threads, 0, s>>>(map, a, units);
+            } else {
+                plan_grid(gg_fill64_tma_kernel<1>, units, sm_count, blocks, threads);
+                gg_fill64_tma_kernel<1><<<blocks, threads, 0, s>>>(map, a, units);
+            }
         } else if (a.out_u32) {
+            plan_grid(gg_fill64_kernel<1>, units, sm_count, blocks, threads);
             gg_fill64_kernel<1><<<blocks, threads, 0, s>>>(a, units);
         } else {
+            plan_grid(gg_fill64_kernel<0>, units, sm_count, blocks, threads);
             gg_fill64_kernel<0><<<blocks, threads, 0, s>>>(a, units);
         }
     } else {
+        plan_grid(gg_fill_generic_kernel, units, sm_count, blocks, threads);
         gg_fill_generic_kernel<<<blocks, threads, 0, s>>>(a, units);
     }
     return cudaGetLastError();

@@ -19,9 +19,9 @@ M = 0xFFFFFFFF
 
 def _word10(Q, nk, x, y):
     f1, f2 = Q >> 1, Q >> 2
-    MY = (~f2 & (f1 | Q)) & M
+    MY = ((f1 | Q) & 0x09249249) & ~f2 & M
     MX = (f2 & ~(f1 & Q)) & M
-    C = (Q - (MY & 0x09249249)) & M
+    C = (Q - MY) & M
     for k in range(nk):
         py, px = MY & (1 << 3 * k), MX & (1 << 3 * k)
         ct = (C << (30 - 3 * k)) & M          # IMAD.SHL
