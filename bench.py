@@ -106,7 +106,7 @@ class ClockSampler:
         try:
             self.proc = subprocess.Popen(
                 ["nvidia-smi", "-i", self.gpu_id, f"--query-gpu={self.FIELDS}",
-                 "--format=csv,noheader,nounits", "-lms", "200"],
+                 "--format=csv,noheader,nounits", "-lms", "20"],
                 stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.th = threading.Thread(target=self._read, daemon=True)
             self.th.start()
@@ -139,6 +139,19 @@ class ClockSampler:
         return {"sm_mhz": statistics.median(sm) if sm else None,
                 "sm_max_mhz": max(mx) if mx else None, "reasons": reasons,
                 "power_w_max": max(pw) if pw else None, "samples": len(self.rows)}
+
+
+def committed_traffic():
+    """dram read+write bytes per launch of the fill kernel from the committed
+    ncu --set full capture (profiles/r01_fill_ncu.json), or None."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "r01_fill_ncu.json")) as f:
+            d = json.load(f)
+        gb = d["dram__bytes_read.sum"]["value"] + d["dram__bytes_write.sum"]["value"]
+        return {"bytes": gb * 1e9, "source": "profiles/r01_fill_ncu.json (ncu --set full, one launch)",
+                "kernel": d.get("Kernel Name", {}).get("value")}
+    except (OSError, KeyError, ValueError):
+        return None
 
 
 def measured_peaks():
@@ -208,10 +221,14 @@ def run_ours(args, rank, world, local_rank):
     sm_max = float(peaks.get("sm_max_mhz", 1965.0))
     peak_ops = props.multi_processor_count * 128 * sm_max * 1e6  # int lanes/clk/SM x clock
     achieved_ops = LABELS_PER_STEP * OPS_PER_LABEL / (kern_ms / 1e3)
+    tr = committed_traffic()
     roofline = {
         "bound": "alu", "achieved": achieved_ops / 1e12, "peak": peak_ops / 1e12,
         "unit": "Tops/s (32-bit integer ops)", "frac": achieved_ops / peak_ops,
-        "traffic": None, "kernel": "gg_fill64_kernel",
+        "traffic": tr["bytes"] if tr else None,
+        "traffic_note": (f"DRAM bytes per launch, {tr['source']}; algorithmic bytes per launch "
+                         f"{LABELS_PER_STEP * (BITS_BYTES_PER_LABEL + 8):.4g}") if tr else None,
+        "kernel": "gg_fill64x2_tma_kernel",
         "kernel_ms": kern_ms, "ops_per_label": OPS_PER_LABEL,
         "peak_basis": (f"{props.multi_processor_count} SMs x 128 int lanes/clk (ALU 64 + FMA 64, "
                        f"issue 4x32) x {sm_max:.0f} MHz (MEASURED_PEAKS sm_max_mhz)"),

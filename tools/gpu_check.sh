@@ -9,7 +9,7 @@ timeout 300 python __graft_entry__.py > gpurun_out/smoke.log 2>&1; echo "smoke r
 timeout 900 python bench.py ${BENCH_ARGS} > gpurun_out/bench.json 2> gpurun_out/bench.err; echo "bench rc=$?" >> gpurun_out/bench.err
 [ -x tools/step_bench ] && timeout 300 tools/step_bench > gpurun_out/step_bench.txt 2>&1
 if [ -n "$NCU" ]; then
-  timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches.csv python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu-baseline --no-ondemand > gpurun_out/ncu_bench.log 2>&1
+  timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches.csv python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu-baseline --no-ondemand --no-apps > gpurun_out/ncu_bench.log 2>&1
   timeout 900 ncu --set full --clock-control none --import-source on -k regex:gg_fill64 -s 1 -c 1 -o gpurun_out/prof_fill python tools/prof_fill.py > gpurun_out/ncu_full.log 2>&1
 fi
 exit 0
