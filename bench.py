@@ -356,7 +356,8 @@ def run_apps(args, rank, world, local_rank, max_over_ranks):
         "unit": "GNumbers/s", "ms_wall": wall * 1e3, "ms_kernel": kern * 1e3,
         "R_d": tal[2] / tal[0], "T_t": tal[3] / tal[0], "specular": tal[1] / tal[0],
         "absorbed": [v / tal[0] for v in tal[5:]], "conserved": tal[0] == sum(tal[1:]),
-        "host_bits_GB": draws * BITS_BYTES_PER_LABEL / 1e9}
+        "host_bits_GB_used": draws * BITS_BYTES_PER_LABEL / 1e9,
+        "host_bits_GB_fed": r["walker_epochs_fed"] * 192 * BITS_BYTES_PER_LABEL / 1e9 * world}
     g.close()
     return out
 

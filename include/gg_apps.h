@@ -106,8 +106,12 @@ typedef struct {
  *                transmittance T_t, terminated, absorbed per layer.
  *                launched = sum of the others exactly.
  *   per_thread : optional DEVICE int64[threads * (5 + nlayers)] (parity checks).
- *   stats      : optional HOST int64[6]: photons, draws, epochs,
- *                interactions, kernel microseconds, total microseconds.
+ *   stats      : optional HOST int64[7]: photons, draws, epochs,
+ *                interactions, kernel microseconds, total microseconds,
+ *                walker-epochs fed (each = D draws of host bits).  Each
+ *                epoch's window holds only the threads that still had work
+ *                one epoch earlier (prng_epoch_begin_list), fed while the
+ *                previous epoch's kernel runs.
  * Synchronous.  The handle needs >= threads walkers and no open epoch.
  */
 int gg_mc_run(prng_t *h, const gg_mc_config *cfg, int64_t *tallies, int64_t *per_thread,

@@ -175,6 +175,16 @@ int prng_load(prng_t *h, const void *host_buf, size_t bytes);
  */
 int prng_epoch_begin(prng_t *h, uint64_t active_walkers, uint32_t draws, void *stream);
 
+/*
+ * Same as prng_epoch_begin, but the window holds the walkers listed in
+ * `walkers` (HOST array of `count` distinct handle-local walker indices):
+ * slot k of the window (the index kernels pass to prng_state_load) is walker
+ * walkers[k].  Only those walkers' bits are fed and copied; the numbers each
+ * walker receives are unchanged (still draw J0 + i of that walker).
+ */
+int prng_epoch_begin_list(prng_t *h, const uint32_t *walkers, uint64_t count, uint32_t draws,
+                          void *stream);
+
 /* Close the epoch: cursor J0 += draws; unused draws are skipped (R10). */
 int prng_epoch_end(prng_t *h, void *stream);
 

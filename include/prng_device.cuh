@@ -7,7 +7,7 @@
  *   the walker's vertex label returned as a 64-bit number (§III-B).
  *
  * Usage inside a user kernel (after prng_epoch_begin + prng_device_view):
- *     prng_state st = prng_state_load(&view, walker);
+ *     prng_state st = prng_state_load(&view, slot);   // slot = walker by default
  *     uint64_t r = prng_next(&st, &view);      // as often as the epoch allows
  *     prng_state_store(&view, &st);
  * A walker must be used by one thread at a time (that is what makes the
@@ -25,7 +25,8 @@
 
 /* Everything a device thread needs; filled by prng_device_view(). */
 struct prng_view {
-    const uint32_t *bits;  /* epoch window, SoA: word (d*R + r) of walker t at bits[(d*R+r)*pitch + t] */
+    const uint32_t *bits;  /* epoch window, SoA: word (d*R + r) of window slot k at bits[(d*R+r)*pitch + k] */
+    const uint32_t *wmap;  /* slot -> walker (prng_epoch_begin_list), or NULL: slot k = walker k */
     uint32_t *x;           /* walker vertex, x coordinate (wrapped mod 2^32 when m is a power of two) */
     uint32_t *y;           /* walker vertex, y coordinate */
     uint32_t *j;           /* next absolute draw index of each walker */
@@ -34,7 +35,7 @@ struct prng_view {
     uint64_t m;            /* modulus */
     uint32_t J0;           /* first draw of the window */
     uint32_t D;            /* draws per walker in the window */
-    uint32_t Wv;           /* walkers covered by the window: [0, Wv) */
+    uint32_t Wv;           /* slots covered by the window: [0, Wv) */
     uint32_t R;            /* words per draw record = ceil(3l/32) */
     uint32_t l;            /* steps per number */
     uint32_t log2m;        /* log2(m) if m is a power of two, else 0 */
@@ -44,7 +45,8 @@ struct prng_view {
 
 struct prng_state {
     uint32_t x, y;     /* current vertex */
-    uint32_t walker;   /* walker id (window-local) */
+    uint32_t walker;   /* walker id (handle-local): index of the state arrays */
+    uint32_t slot;     /* column of the epoch window holding this walker's bits */
     uint32_t used;     /* draws consumed in this epoch */
 };
 
@@ -217,12 +219,16 @@ __device__ __forceinline__ uint64_t gg_label(uint32_t x, uint32_t y, uint64_t m,
 
 /* ------------------------------ on-demand API -------------------------- */
 
-__device__ __forceinline__ prng_state prng_state_load(const prng_view *v, uint32_t walker)
+/* State of the walker in window slot `slot` (= the walker itself unless the
+ * epoch was opened with an explicit walker list). */
+__device__ __forceinline__ prng_state prng_state_load(const prng_view *v, uint32_t slot)
 {
     prng_state st;
+    const uint32_t walker = v->wmap ? v->wmap[slot] : slot;
     st.x = v->x[walker];
     st.y = v->y[walker];
     st.walker = walker;
+    st.slot = slot;
     const uint32_t j = v->j[walker];
     st.used = (j > v->J0) ? (j - v->J0) : 0u; /* walkers that skipped epochs jump to J0 */
     return st;
@@ -244,11 +250,11 @@ __device__ __forceinline__ uint32_t prng_available(const prng_view *v, const prn
 /* Alg.2 GetNextRand: walk l steps with the bits of draw (J0 + used). */
 __device__ __forceinline__ uint64_t prng_next(prng_state *st, const prng_view *v)
 {
-    if (st->used >= v->D || st->walker >= v->Wv) {
+    if (st->used >= v->D || st->slot >= v->Wv) {
         atomicOr(v->flags, PRNG_FLAG_OVERRUN);
         return 0ull;
     }
-    const uint32_t *rec = v->bits + (uint64_t)st->used * v->R * v->pitch + st->walker;
+    const uint32_t *rec = v->bits + (uint64_t)st->used * v->R * v->pitch + st->slot;
     uint32_t x = st->x, y = st->y;
     if (v->l == 64u && v->pow2) {
         uint32_t w[6];

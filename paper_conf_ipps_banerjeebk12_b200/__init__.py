@@ -136,6 +136,13 @@ class Generator:
         check(_lib.prng_epoch_begin(self._h, active_walkers, draws, _stream_handle(stream)),
               "prng_epoch_begin")
 
+    def epoch_begin_list(self, walkers, draws: int, stream=None) -> None:
+        """prng_epoch_begin_list: window slot k holds walker walkers[k] (host uint32 array)."""
+        import numpy as np
+        ids = np.ascontiguousarray(walkers, dtype=np.uint32)
+        check(_lib.prng_epoch_begin_list(self._h, ids.ctypes.data, ids.size, draws,
+                                         _stream_handle(stream)), "prng_epoch_begin_list")
+
     def epoch_end(self, stream=None) -> None:
         check(_lib.prng_epoch_end(self._h, _stream_handle(stream)), "prng_epoch_end")
 
@@ -185,7 +192,7 @@ class Generator:
                                 thread0, threads, epoch_draws, w_threshold)
         nt = 5 + len(layers)
         tal = (ctypes.c_int64 * nt)()
-        stats = (ctypes.c_int64 * 6)()
+        stats = (ctypes.c_int64 * 7)()
         check(_lib.gg_mc_run(self._h, ctypes.byref(cfg), tal,
                              None if per_thread is None else per_thread.data_ptr(), stats,
                              _stream_handle(stream)), "gg_mc_run")
@@ -193,7 +200,8 @@ class Generator:
         out = {k: tal[i] for i, k in enumerate(names)}
         out["absorbed"] = [tal[i] for i in range(5, nt)]
         out["tallies"] = [tal[i] for i in range(nt)]
-        for i, k in enumerate(("photons", "draws", "epochs", "interactions", "kernel_us", "total_us")):
+        for i, k in enumerate(("photons", "draws", "epochs", "interactions", "kernel_us", "total_us",
+                               "walker_epochs_fed")):
             out[k] = stats[i]
         return out
 

@@ -69,7 +69,7 @@ class gg_mc_config(ctypes.Structure):
 
 class prng_view(ctypes.Structure):
     """Mirror of struct prng_view (include/prng_device.cuh)."""
-    _fields_ = [("bits", vp), ("x", vp), ("y", vp), ("j", vp), ("flags", vp), ("pitch", u64),
+    _fields_ = [("bits", vp), ("wmap", vp), ("x", vp), ("y", vp), ("j", vp), ("flags", vp), ("pitch", u64),
                 ("m", u64), ("J0", u32), ("D", u32), ("Wv", u32), ("R", u32), ("l", u32),
                 ("log2m", u32), ("pow2", u32), ("_pad", u32)]
 
@@ -91,6 +91,7 @@ _SIGS = {
     "prng_save": (c_int, [vp, vp, sz]),
     "prng_load": (c_int, [vp, vp, sz]),
     "prng_epoch_begin": (c_int, [vp, u64, u32, vp]),
+    "prng_epoch_begin_list": (c_int, [vp, vp, u64, u32, vp]),
     "prng_epoch_end": (c_int, [vp, vp]),
     "prng_device_view": (c_int, [vp, vp, sz]),
     "prng_check": (c_int, [vp]),

@@ -49,5 +49,8 @@ cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count);
 //   out[r*pitch + i] = word32(seed, tg0 + i, k0 + r),  r < nrows, i < count
 void feed_splitmix_rows(uint64_t seed, uint64_t tg0, uint64_t count, uint64_t k0,
                         uint32_t nrows, uint32_t *out, uint64_t pitch);
+// Same for an explicit walker list: column i = global walker base + ids[i].
+void feed_splitmix_rows_ids(uint64_t seed, uint64_t base, const uint32_t *ids, uint64_t count,
+                            uint64_t k0, uint32_t nrows, uint32_t *out, uint64_t pitch);
 
 }  // namespace gg

@@ -19,6 +19,7 @@
 #include <cstdint>
 #include <vector>
 
+#include <cub/cub.cuh>
 #include <cuda_runtime.h>
 
 #include "gg_apps.h"
@@ -48,6 +49,7 @@ struct McState {
     uint64_t *w;
     int32_t *layer;
     uint32_t *alive, *launched;
+    uint8_t *busy;   // 1 while the thread still has photons to simulate
 };
 
 __device__ __forceinline__ double mc_xi(uint64_t label) {
@@ -105,25 +107,29 @@ __device__ __forceinline__ double mc_fresnel(double n1, double n2, double ca1, d
     return r;
 }
 
-__global__ void mc_init_state(McState s, uint64_t n) {
+__global__ void mc_init_state(McState s, uint64_t n, uint32_t *iota) {
     const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= n) return;
     s.alive[i] = 0;
     s.launched[i] = 0;
     s.w[i] = 0;
+    s.busy[i] = 1;
+    iota[i] = (uint32_t)i;
 }
 
 __global__ void __launch_bounds__(128) mc_epoch(prng_view v, McParams P, McState S,
                                                 unsigned long long *tallies,
                                                 long long *per_thread,
                                                 unsigned long long *counters) {
-    const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const uint64_t slot = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const int nt = kFixed + P.nl;
     long long tal[kFixed + kMaxL];
 #pragma unroll
     for (int k = 0; k < kFixed + kMaxL; k++) tal[k] = 0;
     unsigned long long launched_now = 0, interactions = 0, draws = 0, done = 0;
-    if (i < P.threads) {
+    if (slot < v.Wv) {
+        // the window holds the threads that still had work one epoch ago
+        const uint64_t i = v.wmap ? v.wmap[slot] : slot;
         const uint64_t tg = P.thread0 + i;
         const uint64_t budget =
             P.photons_total / P.threads_total + (tg < P.photons_total % P.threads_total ? 1 : 0);
@@ -133,7 +139,7 @@ __global__ void __launch_bounds__(128) mc_epoch(prng_view v, McParams P, McState
         int layer = S.layer[i];
         bool alive = S.alive[i] != 0;
         uint32_t launched = S.launched[i];
-        prng_state st = prng_state_load(&v, (uint32_t)i);
+        prng_state st = prng_state_load(&v, (uint32_t)slot);
         for (uint32_t it = 0; it < P.K; it++) {
             if (!alive && launched == budget) break;
             // three draws at a convergent point (R22)
@@ -241,6 +247,7 @@ __global__ void __launch_bounds__(128) mc_epoch(prng_view v, McParams P, McState
         S.alive[i] = alive ? 1u : 0u;
         S.launched[i] = launched;
         done = (!alive && launched == budget) ? 1 : 0;
+        S.busy[i] = done ? 0 : 1;
         if (per_thread)
             for (int k = 0; k < nt; k++) per_thread[i * nt + k] += tal[k];
     }
@@ -335,61 +342,92 @@ extern "C" int gg_mc_run(prng_t *h, const gg_mc_config *cfg, int64_t *tallies, i
         S.layer = (int32_t *)alloc(n * 4);
         S.alive = (uint32_t *)alloc(n * 4);
         S.launched = (uint32_t *)alloc(n * 4);
+        S.busy = (uint8_t *)alloc(n);
+        uint32_t *iota = (uint32_t *)alloc(n * 4);
+        uint32_t *d_list = (uint32_t *)alloc(n * 4);
+        int32_t *d_count = (int32_t *)alloc(8);
+        size_t sel_bytes = 0;
+        MCK(cub::DeviceSelect::Flagged(nullptr, sel_bytes, iota, S.busy, d_list, d_count, (int)n, s));
+        void *sel_tmp = alloc(sel_bytes);
         unsigned long long *d_tal = (unsigned long long *)alloc(nt * 8);
         unsigned long long *d_cnt = (unsigned long long *)alloc(4 * 8);
         MCK(cudaMemsetAsync(d_tal, 0, nt * 8, s));
         MCK(cudaMemsetAsync(d_cnt, 0, 4 * 8, s));
         if (per_thread) MCK(cudaMemsetAsync(per_thread, 0, n * nt * 8, s));
-        mc_init_state<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(S, n);
+        mc_init_state<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(S, n, iota);
         cudaEvent_t e0, e1;
         MCK(cudaEventCreate(&e0));
         MCK(cudaEventCreate(&e1));
         MCK(cudaEventRecord(e0, s));
-        unsigned long long *counters = nullptr;  // pinned: the D2H read must not block the feed
-        MCK(cudaMallocHost(&counters, 4 * sizeof(unsigned long long)));
+        // pinned host buffers: counters, active count and active list (the D2H
+        // reads must not block the host FEED of the next window)
+        unsigned long long *counters = nullptr;
+        uint32_t *h_list = nullptr;
+        MCK(cudaMallocHost(&counters, 4 * sizeof(unsigned long long) + 8));
+        MCK(cudaMallocHost(&h_list, n * 4));
+        int32_t *h_count = (int32_t *)(counters + 4);
+        std::vector<uint32_t> feed_list;  // walkers of the next window (one epoch of lag)
         int64_t epochs = 0;
         double kernel_ms = 0.0;
+        uint64_t window_slots = 0;
         cudaEvent_t k0, k1, kc;
         MCK(cudaEventCreate(&k0));
         MCK(cudaEventCreate(&k1));
         MCK(cudaEventCreateWithFlags(&kc, cudaEventDisableTiming));
         try {
             MRC(prng_epoch_begin(h, n, cfg->epoch_draws, s));
+            uint64_t wslots = n;
             for (;;) {
                 prng_view v;
                 MRC(prng_device_view(h, &v, sizeof(v)));
-                MCK(cudaMemsetAsync(d_cnt + 3, 0, 8, s));  // 'done' is recounted each epoch
                 MCK(cudaEventRecord(k0, s));
-                mc_epoch<<<(unsigned)((n + 127) / 128), 128, 0, s>>>(v, P, S, d_tal,
-                                                                     (long long *)per_thread, d_cnt);
+                mc_epoch<<<(unsigned)((wslots + 127) / 128), 128, 0, s>>>(
+                    v, P, S, d_tal, (long long *)per_thread, d_cnt);
                 MCK(cudaGetLastError());
                 MCK(cudaEventRecord(k1, s));
                 MRC(prng_epoch_end(h, s));
                 epochs++;
+                window_slots += wslots;
+                // threads that still have work after this epoch
+                MCK(cub::DeviceSelect::Flagged(sel_tmp, sel_bytes, iota, S.busy, d_list, d_count,
+                                               (int)n, s));
+                MCK(cudaMemcpyAsync(h_count, d_count, 4, cudaMemcpyDeviceToHost, s));
+                MCK(cudaMemcpyAsync(h_list, d_list, n * 4, cudaMemcpyDeviceToHost, s));
                 MCK(cudaMemcpyAsync(counters, d_cnt, 4 * sizeof(unsigned long long),
                                     cudaMemcpyDeviceToHost, s));
                 MCK(cudaEventRecord(kc, s));
-                // FEED + TRANSFER of the next epoch overlap this epoch's kernel
+                // FEED + TRANSFER of the next window overlap this epoch's kernel
                 // (Alg.4 l.7: "Generate and transfer new bin in an overlapping
-                // manner"); if every thread turns out to be done, that one
-                // speculative window is discarded.
-                MRC(prng_epoch_begin(h, n, cfg->epoch_draws, s));
+                // manner").  Its walkers are the threads known to be busy one
+                // epoch ago (a superset of those busy now); a thread that has
+                // finished in between simply does not draw.
+                if (epochs == 1) {
+                    MRC(prng_epoch_begin(h, n, cfg->epoch_draws, s));
+                    wslots = n;
+                } else {
+                    MRC(prng_epoch_begin_list(h, feed_list.data(), feed_list.size(),
+                                              cfg->epoch_draws, s));
+                    wslots = feed_list.size();
+                }
                 MCK(cudaEventSynchronize(kc));
                 float ms = 0.0f;
                 MCK(cudaEventElapsedTime(&ms, k0, k1));
                 kernel_ms += ms;
-                if (counters[3] == n) {
-                    MRC(prng_epoch_end(h, s));
+                if (*h_count == 0) {
+                    MRC(prng_epoch_end(h, s));  // discard the speculative window
                     break;
                 }
+                feed_list.assign(h_list, h_list + *h_count);
             }
         } catch (const Fail &) {
             cudaFreeHost(counters);
+            cudaFreeHost(h_list);
             throw;
         }
         const unsigned long long c_launched = counters[0], c_draws = counters[1],
                                  c_inter = counters[2];
         cudaFreeHost(counters);
+        cudaFreeHost(h_list);
         MCK(cudaEventRecord(e1, s));
         std::vector<unsigned long long> ht(nt);
         MCK(cudaMemcpyAsync(ht.data(), d_tal, nt * 8, cudaMemcpyDeviceToHost, s));
@@ -404,6 +442,7 @@ extern "C" int gg_mc_run(prng_t *h, const gg_mc_config *cfg, int64_t *tallies, i
             stats[3] = (int64_t)c_inter;       // interactions
             stats[4] = (int64_t)(kernel_ms * 1000.0);  // microseconds in mc_epoch kernels
             stats[5] = (int64_t)(total_ms * 1000.0);   // microseconds end to end (feed incl.)
+            stats[6] = (int64_t)window_slots;          // walker-epochs fed (x D draws of bits)
         }
         cudaEventDestroy(e0);
         cudaEventDestroy(e1);

@@ -151,6 +151,9 @@ struct prng_s {
     size_t od_cap[2] = {};
     cudaEvent_t od_free[2] = {};       // recorded at epoch_end: kernels done with the slot
     int od_slot = 1;
+    uint32_t *od_wmap_buf[2] = {};     // slot -> walker maps (prng_epoch_begin_list)
+    size_t od_wmap_cap[2] = {};
+    const uint32_t *od_wmap = nullptr; // map of the open epoch, or nullptr
 
     cudaEvent_t ev_tmp = nullptr;
     prng_stats stats{};
@@ -164,7 +167,7 @@ void free_all(prng_s *h) {
     cudaSetDevice(h->o.device);
     cudaDeviceSynchronize();
     for (auto p : {h->x, h->y, h->j, h->flags, h->xs, h->ys, h->js, h->res_bits, h->ring[0],
-                   h->ring[1], h->od_buf[0], h->od_buf[1]})
+                   h->ring[1], h->od_buf[0], h->od_buf[1], h->od_wmap_buf[0], h->od_wmap_buf[1]})
         if (p) cudaFree(p);
     for (auto p : h->hout)
         if (p) cudaFree(p);
@@ -186,7 +189,8 @@ void free_all(prng_s *h) {
 
 // Generate rows [k0, k0+nrows) of the streams of local walkers [wa, wb)
 // into buf (pitch = wb - wa words), in parallel over walkers.
-void feed_chunk(prng_s *h, uint64_t wa, uint64_t wb, uint64_t k0, uint32_t nrows, uint32_t *buf) {
+void feed_chunk(prng_s *h, uint64_t wa, uint64_t wb, uint64_t k0, uint32_t nrows, uint32_t *buf,
+                const uint32_t *ids) {
     const uint64_t cw = wb - wa;
     const unsigned nt = h->pool->size();
     auto t0 = std::chrono::steady_clock::now();
@@ -195,6 +199,17 @@ void feed_chunk(prng_s *h, uint64_t wa, uint64_t wb, uint64_t k0, uint32_t nrows
         uint64_t per = round_up((cw + nt - 1) / nt, 16);
         uint64_t lo = std::min<uint64_t>(cw, per * ti), hi = std::min<uint64_t>(cw, lo + per);
         if (lo >= hi) return;
+        if (ids) {
+            if (h->o.bit_source == PRNG_BITS_CALLBACK) {
+                for (uint64_t i = lo; i < hi; i++)  // one walker at a time
+                    h->o.bits_fn(h->o.bits_ctx, h->o.walker_base + ids[wa + i], 1, k0, nrows,
+                                 buf + i, cw);
+            } else {
+                gg::feed_splitmix_rows_ids(h->seed, h->o.walker_base, ids + wa + lo, hi - lo, k0,
+                                           nrows, buf + lo, cw);
+            }
+            return;
+        }
         const uint64_t tg0 = h->o.walker_base + wa + lo;
         if (h->o.bit_source == PRNG_BITS_CALLBACK)
             h->o.bits_fn(h->o.bits_ctx, tg0, hi - lo, k0, nrows, buf + lo, cw);
@@ -211,7 +226,7 @@ void feed_chunk(prng_s *h, uint64_t wa, uint64_t wb, uint64_t k0, uint32_t nrows
 // pinned chunk while the previous chunks are DMA'd on copy_stream.
 // On return every copy is enqueued on copy_stream.
 void stage_rows(prng_s *h, uint64_t k0, uint64_t nrows, uint64_t Wv, uint32_t *dst,
-                uint64_t dpitch) {
+                uint64_t dpitch, const uint32_t *ids = nullptr) {
     if (nrows == 0 || Wv == 0) return;
     const uint64_t chunk_words = h->chunk_bytes / 4;
     uint64_t rows_per, walkers_per;
@@ -229,7 +244,7 @@ void stage_rows(prng_s *h, uint64_t k0, uint64_t nrows, uint64_t Wv, uint32_t *d
             const int b = h->chunk_next;
             h->chunk_next = (b + 1) % prng_s::kChunks;
             CK(cudaEventSynchronize(h->chunk_done[b]));  // pinned chunk free again
-            feed_chunk(h, wa, wb, k0 + r, nr, h->chunk[b]);
+            feed_chunk(h, wa, wb, k0 + r, nr, h->chunk[b], ids);
             const uint64_t cw = wb - wa;
             CK(cudaMemcpy2DAsync(dst + r * dpitch + wa, dpitch * 4, h->chunk[b], cw * 4, cw * 4,
                                  nr, cudaMemcpyHostToDevice, h->copy_stream));
@@ -683,10 +698,8 @@ int prng_load(prng_t *h, const void *host_buf, size_t bytes) {
     });
 }
 
-int prng_epoch_begin(prng_t *h, uint64_t active_walkers, uint32_t draws, void *stream) {
-    if (!h) return PRNG_E_INVALID;
-    if (active_walkers == 0 || active_walkers > h->W || draws == 0) return PRNG_E_INVALID;
-    if (h->od_open) return PRNG_E_STATE;
+static int epoch_begin_impl(prng_t *h, uint64_t active_walkers, const uint32_t *ids,
+                            uint32_t draws, void *stream) {
     return guard(h, [&] {
         cudaStream_t s = (cudaStream_t)stream;
         const uint64_t J0 = h->od_started ? h->od_J0 : (h->N + h->W - 1) / h->W;
@@ -694,21 +707,39 @@ int prng_epoch_begin(prng_t *h, uint64_t active_walkers, uint32_t draws, void *s
         const uint64_t pitch = round_up(active_walkers, 32);
         const size_t bytes = (size_t)draws * h->R * pitch * 4;
         const int slot = h->od_slot ^ 1;
-        if (bytes > h->od_cap[slot]) {
+        if (bytes > h->od_cap[slot] || (ids && active_walkers * 4 > h->od_wmap_cap[slot])) {
             CK(cudaEventSynchronize(h->od_free[slot]));
-            if (h->od_buf[slot]) CK(cudaFree(h->od_buf[slot]));
-            h->od_buf[slot] = nullptr;
-            h->od_cap[slot] = 0;
-            CK(cudaMalloc(&h->od_buf[slot], bytes));
-            h->od_cap[slot] = bytes;
+            if (bytes > h->od_cap[slot]) {
+                if (h->od_buf[slot]) CK(cudaFree(h->od_buf[slot]));
+                h->od_buf[slot] = nullptr;
+                h->od_cap[slot] = 0;
+                CK(cudaMalloc(&h->od_buf[slot], bytes));
+                h->od_cap[slot] = bytes;
+            }
+            if (ids && active_walkers * 4 > h->od_wmap_cap[slot]) {
+                if (h->od_wmap_buf[slot]) CK(cudaFree(h->od_wmap_buf[slot]));
+                h->od_wmap_buf[slot] = nullptr;
+                h->od_wmap_cap[slot] = 0;
+                CK(cudaMalloc(&h->od_wmap_buf[slot], active_walkers * 4));
+                h->od_wmap_cap[slot] = active_walkers * 4;
+            }
         } else {
             // kernels of the epoch that last used this slot must be done with it
             CK(cudaStreamWaitEvent(h->copy_stream, h->od_free[slot], 0));
         }
         h->od_slot = slot;
         h->od_bits = h->od_buf[slot];
+        h->od_wmap = nullptr;
+        if (ids) {
+            // the map travels with the bits (pageable source: the copy is staged by
+            // the runtime, so the caller may reuse its array on return)
+            CK(cudaMemcpyAsync(h->od_wmap_buf[slot], ids, active_walkers * 4,
+                               cudaMemcpyHostToDevice, h->copy_stream));
+            h->od_wmap = h->od_wmap_buf[slot];
+            h->stats.h2d_bytes += active_walkers * 4;
+        }
         stage_rows(h, 2 + h->R0 + h->R * J0, (uint64_t)draws * h->R, active_walkers, h->od_bits,
-                   pitch);
+                   pitch, ids);
         join_copies(h, s);
         h->od_J0 = J0;
         h->od_D = draws;
@@ -718,6 +749,23 @@ int prng_epoch_begin(prng_t *h, uint64_t active_walkers, uint32_t draws, void *s
         h->od_started = true;
         return PRNG_OK;
     });
+}
+
+int prng_epoch_begin(prng_t *h, uint64_t active_walkers, uint32_t draws, void *stream) {
+    if (!h) return PRNG_E_INVALID;
+    if (active_walkers == 0 || active_walkers > h->W || draws == 0) return PRNG_E_INVALID;
+    if (h->od_open) return PRNG_E_STATE;
+    return epoch_begin_impl(h, active_walkers, nullptr, draws, stream);
+}
+
+int prng_epoch_begin_list(prng_t *h, const uint32_t *walkers, uint64_t count, uint32_t draws,
+                          void *stream) {
+    if (!h || !walkers) return PRNG_E_INVALID;
+    if (count == 0 || count > h->W || draws == 0) return PRNG_E_INVALID;
+    for (uint64_t i = 0; i < count; i++)
+        if (walkers[i] >= h->W) return PRNG_E_INVALID;
+    if (h->od_open) return PRNG_E_STATE;
+    return epoch_begin_impl(h, count, walkers, draws, stream);
 }
 
 int prng_epoch_end(prng_t *h, void *stream) {
@@ -738,6 +786,7 @@ int prng_device_view(prng_t *h, void *view, size_t view_bytes) {
     if (!h->od_open) return PRNG_E_STATE;
     prng_view v{};
     v.bits = h->od_bits;
+    v.wmap = h->od_wmap;
     v.x = h->x;
     v.y = h->y;
     v.j = h->j;

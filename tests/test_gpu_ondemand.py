@@ -110,3 +110,33 @@ def test_bulk_after_on_demand_realigns():
         ow = OracleWalker(M32, seed, t)
         ow.draw(0)  # the one used draw; draw 1 skipped
         assert int(z[t]) == ow.draw(2)
+
+
+def test_epoch_with_walker_list():
+    # prng_epoch_begin_list: slot k holds walker ids[k]; numbers per walker are
+    # unchanged (draw J0 + i of that walker), only the fed bits differ.
+    import torch
+    from paper_conf_ipps_banerjeebk12_b200 import Generator
+    W, D, seed = 1000, 3, 17
+    g = Generator(walkers=W, seed=seed)
+    ids = np.array([999, 3, 500, 0, 42], dtype=np.uint32)
+    g.epoch_begin_list(ids, D)
+    o = torch.empty(ids.size * D, dtype=torch.int64, device="cuda")
+    g.consume(ids.size, uniform=D, out=o)
+    g.epoch_end()
+    # second epoch over all walkers: listed walkers continue, others start at J0 = 3
+    g.epoch_begin(W, 1)
+    o2 = torch.empty(W, dtype=torch.int64, device="cuda")
+    g.consume(W, uniform=1, out=o2)
+    g.epoch_end()
+    assert g.check() == 0
+    z = o.view(ids.size, D).cpu().numpy().view(np.uint64)
+    z2 = o2.cpu().numpy().view(np.uint64)
+    for k, t in enumerate(ids):
+        assert np.array_equal(z[k], O.walker_draws(M32, 64, 64, seed, int(t), 0, D))
+        ow = OracleWalker(M32, seed, int(t))
+        for j in range(D):
+            ow.draw(j)
+        assert int(z2[t]) == ow.draw(3)
+    ow = OracleWalker(M32, seed, 7)   # not listed: skipped draws 0..2
+    assert int(z2[7]) == ow.draw(3)
