@@ -242,6 +242,40 @@ def run_ours(args, rank, world, local_rank):
     del out
     torch.cuda.empty_cache()
 
+    # ---- f1: l = 1 ("emit every vertex"): 4 B read + 8 B written
+    # per number, HBM-bound; 2^20 walkers x 1024 draws, bits resident
+    if not args.no_l1:
+        g = Generator(walkers=W_PER_GPU, seed=SEED, walk_len=1, walker_base=rank * W_PER_GPU,
+                      device=local_rank)
+        D1 = 1024
+        g.prefetch(D1)
+        g.mark()
+        o1 = torch.empty(W_PER_GPU * D1, dtype=torch.int64, device=dev)
+        for _ in range(args.warmup):
+            g.rewind()
+            g.fill(o1)
+        e0 = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+        e1 = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+        torch.cuda.synchronize()
+        for i in range(args.steps):
+            g.rewind()
+            e0[i].record(stream)
+            g.fill(o1)
+            e1[i].record(stream)
+        torch.cuda.synchronize()
+        ms1 = max_over_ranks(statistics.median(a.elapsed_time(b) for a, b in zip(e0, e1)))
+        labels1 = W_PER_GPU * D1
+        gbs = labels1 * 12 / (ms1 / 1e3) / 1e9
+        res["l1_fill"] = {
+            "config": "l = 1 (one 3-bit step per number), m = 2^32, 2^20 walkers x 1024 draws per GPU",
+            "value": world * labels1 / (ms1 / 1e3) / 1e9, "unit": UNIT, "ms_kernel": ms1,
+            "roofline": {"bound": "hbm", "achieved": gbs, "peak": measured_peaks().get("hbm_gbs"),
+                         "unit": "GB/s", "frac": gbs / measured_peaks().get("hbm_gbs", 6460.9),
+                         "bytes_per_number": 12, "kernel": "gg_fill_l1_tma_kernel"}}
+        g.close()
+        del o1
+        torch.cuda.empty_cache()
+
     # ---- on-demand: every thread calls prng_next S = 100 times (Fig.4 batch)
     if not args.no_ondemand:
         S = 100
@@ -372,6 +406,7 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-ondemand", action="store_true")
     ap.add_argument("--no-apps", action="store_true")
+    ap.add_argument("--no-l1", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=8.0)
     args = ap.parse_args()
@@ -413,6 +448,7 @@ def main():
             "roofline": res["roofline"], "cpu_baseline": cpu, "e2e": res.get("e2e"),
             "clocks": res["clocks"], "gpu_launches": res["launches"],
             "on_demand": res.get("on_demand"), "apps": res.get("apps"),
+            "l1_fill": res.get("l1_fill"),
         }
         print(json.dumps(line))
     if world > 1:

@@ -70,7 +70,9 @@ typedef struct {
     uint32_t degree;     /* must be 7 (Gabber–Galil), else PRNG_E_UNSUPPORTED */
     uint32_t walk_len;   /* l = 64 steps per number (Alg.2, R6); 1..4096 */
     uint32_t burnin_len; /* l0 = 64 steps of Alg.1 ("initial walk of length 64"); 0..4096 */
-    uint32_t variant;    /* 0 = forward maps sigma_k (R2); others PRNG_E_UNSUPPORTED */
+    uint32_t variant;    /* 0 = forward maps sigma_k at every step (R2); 1 = bipartite
+                            walk: global step s applies sigma_k (s even, X -> Y) or
+                            sigma_k^{-1} (s odd, Y -> X) */
 } prng_graph_params;
 
 /*

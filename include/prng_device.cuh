@@ -40,6 +40,8 @@ struct prng_view {
     uint32_t l;            /* steps per number */
     uint32_t log2m;        /* log2(m) if m is a power of two, else 0 */
     uint32_t pow2;         /* 1 if m is a power of two */
+    uint32_t variant;      /* 0 = forward maps; 1 = bipartite (sigma / sigma^-1 alternating) */
+    uint32_t l0;           /* burn-in steps (global step parity for variant 1) */
     uint32_t _pad;
 };
 
@@ -170,19 +172,31 @@ __device__ __forceinline__ void gg_walk64x2(const uint32_t a[6], const uint32_t 
 }
 
 /* One step, any m (generic path).  Non power-of-two m requires m <= 2^30 and
- * x, y < m: the pre-reduction value 2*src + target + 2 < 4m fits in 32 bits. */
+ * x, y < m: every pre-reduction value is < 4m and fits in 32 bits.
+ * inv: apply sigma_k^{-1} (variant 1, odd steps): y - 2x - c / x - 2y - c. */
+__device__ __forceinline__ uint32_t gg_reduce(uint32_t t, uint32_t m, bool pow2)
+{
+    if (!pow2) {
+        t = (t >= 2u * m) ? t - 2u * m : t;
+        t = (t >= m) ? t - m : t;
+    }
+    return t;
+}
+
 __device__ __forceinline__ void gg_step_generic(uint32_t b, uint32_t &x, uint32_t &y,
-                                                uint32_t m, bool pow2)
+                                                uint32_t m, bool pow2, bool inv = false)
 {
     const uint32_t cy = b - 1u, cx = b - 4u;
     if (cy < 3u) {
-        uint32_t t = y + 2u * x + cy;
-        if (!pow2) { t = (t >= 2u * m) ? t - 2u * m : t; t = (t >= m) ? t - m : t; }
-        y = t;
+        if (!inv)
+            y = gg_reduce(y + 2u * x + cy, m, pow2);
+        else
+            y = pow2 ? y - 2u * x - cy : gg_reduce(y + 3u * m - 2u * x - cy, m, false);
     } else if (cx < 3u) {
-        uint32_t t = x + 2u * y + cx;
-        if (!pow2) { t = (t >= 2u * m) ? t - 2u * m : t; t = (t >= m) ? t - m : t; }
-        x = t;
+        if (!inv)
+            x = gg_reduce(x + 2u * y + cx, m, pow2);
+        else
+            x = pow2 ? x - 2u * y - cx : gg_reduce(x + 3u * m - 2u * y - cx, m, false);
     }
 }
 
@@ -197,13 +211,16 @@ __device__ __forceinline__ uint32_t gg_field(const uint32_t *rec, uint64_t strid
     return __funnelshift_r(lo, hi, s) & 7u;
 }
 
-/* nsteps steps reading the record from global memory (generic l / m). */
+/* nsteps steps reading the record from global memory (generic l / m /
+ * variant); s0 = global step index of the first step (variant 1 parity). */
 __device__ __forceinline__ void gg_walk_generic(const uint32_t *rec, uint64_t stride,
                                                 uint32_t nsteps, uint32_t &x, uint32_t &y,
-                                                uint32_t m, bool pow2)
+                                                uint32_t m, bool pow2, uint32_t variant = 0,
+                                                uint64_t s0 = 0)
 {
     for (uint32_t i = 0; i < nsteps; i++)
-        gg_step_generic(gg_field(rec, stride, i), x, y, m, pow2);
+        gg_step_generic(gg_field(rec, stride, i), x, y, m, pow2,
+                        variant == 1 && ((s0 + i) & 1) != 0);
 }
 
 /* Vertex label x + m*y (R8), reducing wrapped coordinates for m = 2^k. */
@@ -256,14 +273,15 @@ __device__ __forceinline__ uint64_t prng_next(prng_state *st, const prng_view *v
     }
     const uint32_t *rec = v->bits + (uint64_t)st->used * v->R * v->pitch + st->slot;
     uint32_t x = st->x, y = st->y;
-    if (v->l == 64u && v->pow2) {
+    if (v->l == 64u && v->pow2 && v->variant == 0) {
         uint32_t w[6];
 #pragma unroll
         for (int r = 0; r < 6; r++)
             w[r] = __ldg(rec + (uint64_t)r * v->pitch);
         gg_walk64(w, x, y);
     } else {
-        gg_walk_generic(rec, v->pitch, v->l, x, y, (uint32_t)v->m, v->pow2 != 0);
+        const uint64_t s0 = (uint64_t)v->l0 + (uint64_t)v->l * (v->J0 + st->used);
+        gg_walk_generic(rec, v->pitch, v->l, x, y, (uint32_t)v->m, v->pow2 != 0, v->variant, s0);
     }
     st->x = x;
     st->y = y;

@@ -67,6 +67,11 @@ def lib():
                 "or_walker_draws": (ctypes.c_int, [u64, u32, u32, u64, u64, u64, u64, P]),
                 "or_sigma_array": (None, [u64, ctypes.c_int, P, P, P, P, u64]),
                 "or_stream_block": (None, [u64, u64, u64, u64, u32, P]),
+                "or_sigma_inv": (None, [u64, ctypes.c_int, u64, u64, P, P]),
+                "or_walk_bipartite": (None, [u64, P, P, P, u32, u64]),
+                "or_walker_init_v": (ctypes.c_int, [u64, u32, u32, u64, u64, P, P]),
+                "or_walker_draw_v": (u64, [u64, u32, u32, u32, u64, u64, u64, P, P]),
+                "or_bulk_v": (ctypes.c_int, [u64, u32, u32, u32, u64, u64, u64, u64, P]),
             }
             for name, (res, args) in sig.items():
                 fn = getattr(L, name)
@@ -170,6 +175,21 @@ def bulk(m: int, l: int, l0: int, seed: int, W: int, g0: int, n: int) -> np.ndar
     rc = lib().or_bulk(m, l, l0, seed, W, g0, n, _ptr(out))
     if rc != 0:
         raise ValueError("or_bulk failed")
+    return out
+
+
+def sigma_inv(m: int, k: int, x: int, y: int):
+    nx = np.zeros(1, np.uint64)
+    ny = np.zeros(1, np.uint64)
+    lib().or_sigma_inv(m, k, x, y, _ptr(nx), _ptr(ny))
+    return int(nx[0]), int(ny[0])
+
+
+def bulk_v(m: int, l: int, l0: int, variant: int, seed: int, W: int, g0: int, n: int) -> np.ndarray:
+    out = np.empty(n, dtype=np.uint64)
+    rc = lib().or_bulk_v(m, l, l0, variant, seed, W, g0, n, _ptr(out))
+    if rc != 0:
+        raise ValueError("or_bulk_v failed")
     return out
 
 

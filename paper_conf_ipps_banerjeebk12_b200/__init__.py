@@ -65,7 +65,7 @@ class Generator:
 
     def __init__(self, walkers: int, seed: int, m: int = 1 << 32, walk_len: int = 64,
                  burnin_len: int = 64, device: int = 0, walker_base: int = 0,
-                 epoch_draws: int = 16, host_threads: int = 0, bits_fn=None):
+                 epoch_draws: int = 16, host_threads: int = 0, bits_fn=None, variant: int = 0):
         self._h = ctypes.c_void_p()
         self.walkers, self.seed, self.m, self.walk_len = walkers, seed, m, walk_len
         self._walker_base = walker_base
@@ -80,7 +80,7 @@ class Generator:
                 for r in range(nwords):
                     buf[r * pitch:r * pitch + nwalkers] = a[r]
             self._bits_fn = _lib.PRNG_BITS_FN(_cb)
-        p = params(m, walk_len, burnin_len)
+        p = params(m, walk_len, burnin_len, variant=variant)
         o = options(device, walker_base, epoch_draws, host_threads, self._bits_fn)
         check(_lib.prng_create(ctypes.byref(self._h), ctypes.byref(p), walkers, seed,
                                ctypes.byref(o)), "prng_create")

@@ -20,6 +20,7 @@ struct InitArgs {
     uint64_t m;
     uint32_t log2m, pow2;
     uint32_t *x, *y, *j;
+    uint32_t variant;
 };
 cudaError_t launch_init(const InitArgs &a, cudaStream_t s);
 
@@ -42,6 +43,7 @@ struct FillArgs {
     uint32_t l, R;
     uint64_t m;
     uint32_t log2m, pow2;
+    uint32_t variant, l0;
 };
 cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count);
 

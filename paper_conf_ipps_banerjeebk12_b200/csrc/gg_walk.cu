@@ -32,13 +32,14 @@ __global__ void __launch_bounds__(128) gg_init_kernel(InitArgs a) {
         x = (uint32_t)(x % a.m);
         y = (uint32_t)(y % a.m);
     }
-    if (a.l0 == 64 && a.pow2) {
+    if (a.l0 == 64 && a.pow2 && a.variant == 0) {
         uint32_t w[6];
 #pragma unroll
         for (int r = 0; r < 6; r++) w[r] = rec[(uint64_t)(2 + r) * a.pitch];
         gg_walk64(w, x, y);
     } else {
-        gg_walk_generic(rec + 2 * a.pitch, a.pitch, a.l0, x, y, (uint32_t)a.m, a.pow2 != 0);
+        gg_walk_generic(rec + 2 * a.pitch, a.pitch, a.l0, x, y, (uint32_t)a.m, a.pow2 != 0,
+                        a.variant, 0);
     }
     const uint32_t t = a.w0 + i;
     a.x[t] = x;
@@ -346,6 +347,84 @@ __global__ void __launch_bounds__(64) gg_fill64x2_tma_kernel(const __grid_consta
     }
 }
 
+// l = 1 ("emit every vertex"): one 32-bit record word per
+// number (R = 1: 3 bits used), so a number costs 4 B read + 8 B written and
+// ~10 instructions: the bound is HBM, not the integer pipes.  Each warp owns
+// 32 walkers; lane 0 streams 32-draw x 32-walker tiles (4 KB) by TMA into two
+// smem stages; lanes step through their column and store coalesced.
+constexpr int kL1Draws = 32;
+
+template <int EMIT>
+__global__ void __launch_bounds__(64) gg_fill_l1_tma_kernel(const __grid_constant__ CUtensorMap tmap,
+                                                            FillArgs a, uint32_t units) {
+    constexpr int kTile = kL1Draws * 32;
+    __shared__ __align__(128) uint32_t tiles[kFillWarps][2][kTile];
+    __shared__ __align__(8) uint64_t bars[kFillWarps][2];
+    const uint32_t lane = threadIdx.x & 31u, wib = threadIdx.x >> 5;
+    const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+    uint64_t *bar0 = &bars[wib][0], *bar1 = &bars[wib][1];
+    if (lane == 0) {
+        mbar_init(bar0, 1);
+        mbar_init(bar1, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncwarp();
+    uint32_t ph0 = 0, ph1 = 0;
+    const uint32_t kBytes = kTile * 4;
+    for (uint32_t u = warp; u < units; u += nwarps) {
+        const uint32_t t = u * 32u + lane;
+        uint32_t j0 = 0xFFFFFFFFu, j1 = 0;
+        if (t < a.W) {
+            walker_draw_range(a.N, a.nl, a.W, t, j0, j1);
+            j0 = max(j0, a.ja);
+            j1 = min(j1, a.jb);
+        }
+        const uint32_t jlo = __reduce_min_sync(0xFFFFFFFFu, j0);
+        const uint32_t jhi = __reduce_max_sync(0xFFFFFFFFu, j1);
+        if (jlo >= jhi) continue;
+        const uint32_t ntiles = (jhi - jlo + kL1Draws - 1) / kL1Draws;
+        uint32_t x = 0, y = 0;
+        if (t < a.W) {
+            x = a.x[t];
+            y = a.y[t];
+        }
+        if (lane == 0) {
+            for (uint32_t q = 0; q < 2 && q < ntiles; q++) {
+                mbar_expect_tx(&bars[wib][q], kBytes);
+                tma_load_tile(tiles[wib][q], &tmap, &bars[wib][q], (int32_t)(u * 32u),
+                              (int32_t)(jlo - a.Jw + q * kL1Draws));
+            }
+        }
+        for (uint32_t q = 0; q < ntiles; q++) {
+            const uint32_t sidx = q & 1u;
+            mbar_wait(&bars[wib][sidx], sidx ? ph1 : ph0);
+            if (sidx) ph1 ^= 1u; else ph0 ^= 1u;
+            const uint32_t *buf = tiles[wib][sidx];
+            const uint32_t jt = jlo + q * kL1Draws;
+#pragma unroll 8
+            for (uint32_t d = 0; d < kL1Draws; d++) {
+                const uint32_t j = jt + d;
+                if (j >= j0 && j < j1) {
+                    gg_step_generic(buf[d * 32 + lane] & 7u, x, y, 0, true);
+                    emit_label<EMIT>(a, (uint64_t)j * a.W + t - a.g_origin, x, y);
+                }
+            }
+            __syncwarp();
+            if (lane == 0 && q + 2 < ntiles) {
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                mbar_expect_tx(&bars[wib][sidx], kBytes);
+                tma_load_tile(tiles[wib][sidx], &tmap, &bars[wib][sidx], (int32_t)(u * 32u),
+                              (int32_t)(jt - a.Jw + 2 * kL1Draws));
+            }
+        }
+        if (t < a.W) {
+            a.x[t] = x;
+            a.y[t] = y;
+        }
+    }
+}
+
 static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
     static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
     static bool tried = false;
@@ -363,12 +442,12 @@ static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
 
 // 2D map over the SoA window: dim0 = walkers (pitch), dim1 = rows; box 32 x 6.
 static bool make_window_map(CUtensorMap *map, const uint32_t *bits, uint64_t pitch, uint64_t rows,
-                            uint32_t box_walkers = 32) {
+                            uint32_t box_walkers = 32, uint32_t box_rows = 6) {
     auto enc = get_encode();
     if (!enc || rows == 0 || rows > 0x7FFFFFFFull) return false;
     cuuint64_t dims[2] = {(cuuint64_t)pitch, (cuuint64_t)rows};
     cuuint64_t strides[1] = {(cuuint64_t)(pitch * 4)};
-    cuuint32_t box[2] = {box_walkers, 6};
+    cuuint32_t box[2] = {box_walkers, box_rows};
     cuuint32_t estr[2] = {1, 1};
     CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, (void *)bits, dims, strides, box, estr,
                      CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
@@ -393,7 +472,8 @@ __global__ void __launch_bounds__(64) gg_fill_generic_kernel(FillArgs a, uint32_
         uint32_t x = a.x[t], y = a.y[t];
         for (uint32_t j = j0; j < j1; j++) {
             const uint32_t *rec = a.bits + t + (uint64_t)(j - a.Jw) * a.R * a.pitch;
-            gg_walk_generic(rec, a.pitch, a.l, x, y, (uint32_t)a.m, a.pow2 != 0);
+            gg_walk_generic(rec, a.pitch, a.l, x, y, (uint32_t)a.m, a.pow2 != 0, a.variant,
+                            (uint64_t)a.l0 + (uint64_t)a.l * j);
             const uint64_t lab = gg_label(x, y, a.m, a.log2m, a.pow2 != 0);
             const uint64_t g = (uint64_t)j * a.W + t;
             if (a.out_u32)
@@ -435,7 +515,23 @@ cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count) {
     if (a.jb <= a.ja || a.nl == 0) return cudaSuccess;
     const uint32_t units = (a.W + 31u) / 32u;
     uint32_t blocks, threads;
-    if (a.l == 64 && a.pow2) {
+    if (a.l == 1 && a.pow2 && a.variant == 0) {
+        CUtensorMap map;
+        if (a.rows && make_window_map(&map, a.bits, a.pitch, a.rows, 32, kL1Draws)) {
+            if (a.out_u32) {
+                plan_grid(gg_fill_l1_tma_kernel<2>, units, sm_count, blocks, threads);
+                gg_fill_l1_tma_kernel<2><<<blocks, threads, 0, s>>>(map, a, units);
+            } else if (a.log2m == 32) {
+                plan_grid(gg_fill_l1_tma_kernel<0>, units, sm_count, blocks, threads);
+                gg_fill_l1_tma_kernel<0><<<blocks, threads, 0, s>>>(map, a, units);
+            } else {
+                plan_grid(gg_fill_l1_tma_kernel<1>, units, sm_count, blocks, threads);
+                gg_fill_l1_tma_kernel<1><<<blocks, threads, 0, s>>>(map, a, units);
+            }
+            return cudaGetLastError();
+        }
+    }
+    if (a.l == 64 && a.pow2 && a.variant == 0) {
         CUtensorMap map;
         static const bool use_tma = getenv("GG_FILL_NO_TMA") == nullptr;
         static const bool use_x2 = getenv("GG_FILL_X1") == nullptr;

@@ -303,6 +303,8 @@ gg::FillArgs fill_args(prng_s *h, const uint32_t *bits, uint64_t pitch, uint64_t
     a.m = h->g.m;
     a.log2m = h->log2m;
     a.pow2 = h->pow2;
+    a.variant = h->g.variant;
+    a.l0 = h->g.burnin_len;
     return a;
 }
 
@@ -411,7 +413,7 @@ int prng_create(prng_t **out, const prng_graph_params *g, uint64_t walkers, uint
         o = *opt;
     else
         prng_default_options(&o);
-    if (g->degree != 7 || g->variant != 0) return PRNG_E_UNSUPPORTED;
+    if (g->degree != 7 || g->variant > 1) return PRNG_E_UNSUPPORTED;
     if (g->m < 2 || g->m > (1ull << 32)) return PRNG_E_INVALID;
     const bool pow2 = (g->m & (g->m - 1)) == 0;
     if (!pow2 && g->m > (1ull << 30)) return PRNG_E_UNSUPPORTED;
@@ -485,7 +487,8 @@ int prng_create(prng_t **out, const prng_graph_params *g, uint64_t walkers, uint
             a.m = g->m;
             a.log2m = h->log2m;
             a.pow2 = h->pow2;
-                    a.x = h->x;
+            a.variant = g->variant;
+            a.x = h->x;
             a.y = h->y;
             a.j = h->j;
             CK(gg::launch_init(a, h->work_stream));
@@ -800,6 +803,8 @@ int prng_device_view(prng_t *h, void *view, size_t view_bytes) {
     v.l = h->g.walk_len;
     v.log2m = h->log2m;
     v.pow2 = h->pow2;
+    v.variant = h->g.variant;
+    v.l0 = h->g.burnin_len;
     memcpy(view, &v, sizeof(v));
     return PRNG_OK;
 }

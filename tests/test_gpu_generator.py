@@ -221,3 +221,52 @@ def test_invalid_calls_have_no_side_effects(torch_cuda):
     with pytest.raises(PrngError):
         g.fill(torch.empty(4, dtype=torch.int64, device="cuda"))  # bulk inside an epoch
     g.epoch_end()
+
+
+# ------------------------------------------------------------ f1 walk variants
+@pytest.mark.parametrize("m,l", [(M32, 64), (256, 64), (1000, 64), (M32, 1), (1000, 1), (M32, 11)])
+def test_bipartite_variant_parity(torch_cuda, m, l):
+    torch = torch_cuda
+    W, seed = 320, 13
+    n = W * 6 + 7
+    g = G(walkers=W, seed=seed, m=m, walk_len=l, variant=1)
+    o = torch.empty(n, dtype=torch.int64, device="cuda")
+    g.fill(o)
+    assert np.array_equal(as_u64(o), O.bulk_v(m, l, 64, 1, seed, W, 0, n))
+
+
+@pytest.mark.parametrize("m", [M32, 1 << 16, 256])
+def test_l1_fast_kernel_parity_ragged(torch_cuda, m):
+    # l = 1 ("emit every vertex") takes the HBM-bound TMA kernel; ragged
+    # fills, prefetched and streamed windows, u64 and u32 outputs.
+    torch = torch_cuda
+    W, seed = 1000, 5
+    sizes = [1, 999, 40000, 12345, 31]
+    total = sum(sizes)
+    want = O.bulk(m, 1, 64, seed, W, 0, total)
+    g = G(walkers=W, seed=seed, m=m, walk_len=1, epoch_draws=7)
+    g.prefetch(20)
+    got = []
+    for s in sizes:
+        o = torch.empty(s, dtype=torch.int64, device="cuda")
+        g.fill(o)
+        got.append(as_u64(o))
+    assert np.array_equal(np.concatenate(got), want)
+    if m <= 1 << 16:
+        h = G(walkers=W, seed=seed, m=m, walk_len=1)
+        o32 = torch.empty(total, dtype=torch.int32, device="cuda")
+        h.fill(o32)
+        assert np.array_equal(o32.cpu().numpy().view(np.uint32).astype(np.uint64), want)
+
+
+def test_bipartite_on_demand(torch_cuda):
+    torch = torch_cuda
+    W, D, seed = 256, 4, 77
+    g = G(walkers=W, seed=seed, variant=1)
+    g.epoch_begin(W, D)
+    o = torch.empty(W * D, dtype=torch.int64, device="cuda")
+    g.consume(W, uniform=D, out=o)
+    g.epoch_end()
+    z = o.view(W, D).cpu().numpy().view(np.uint64)
+    want = O.bulk_v(M32, 64, 64, 1, seed, W, 0, W * D).reshape(D, W).T
+    assert np.array_equal(z, want)

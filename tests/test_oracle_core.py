@@ -230,3 +230,45 @@ def test_general_l_uses_ceil_3l_over_32_words():
             rec = np.array([O.stream_word32(seed, t, 2 + 6 + R * j + r) for r in range(R)], np.uint32)
             x, y = O.walk(M32, x, y, rec, l)
             assert int(O.walker_draws(M32, l, 64, seed, t, j, 1)[0]) == O.label(M32, x, y)
+
+
+# ------------------------------------------- f1: bipartite variant (σ / σ⁻¹)
+@pytest.mark.parametrize("m", [2, 5, 8, 16])
+def test_inverse_maps_exhaustive(m):
+    # sigma_k^{-1} undoes sigma_k on every vertex (the neighbours in X of a
+    # vertex of Y are its preimages), for all k
+    for k in range(7):
+        for x in range(m):
+            for y in range(m):
+                nx, ny = O.sigma(m, k, np.array([x], np.uint64), np.array([y], np.uint64))
+                assert O.sigma_inv(m, k, int(nx[0]), int(ny[0])) == (x, y)
+
+
+def test_bipartite_walk_parity_chain_and_alternation():
+    # The bipartite walk alternates sigma (even steps) and sigma^{-1} (odd);
+    # x mod 2 still flips only on k = 5 (x +- 2y +- 1), so the closed form
+    # (1 - (3/4)^t)/2 of P4 holds, and the 2-step chain is doubly stochastic.
+    m = 8
+    n = m * m
+    Pf = np.zeros((n, n))
+    Pb = np.zeros((n, n))
+    for x in range(m):
+        for y in range(m):
+            for b in range(8):
+                rec = np.array([b], np.uint32)
+                xs, ys = np.array([x], np.uint64), np.array([y], np.uint64)
+                O.lib().or_walk_bipartite(m, O._ptr(xs), O._ptr(ys), O._ptr(rec), 1, 0)
+                Pf[x + m * y, int(xs[0]) + m * int(ys[0])] += 1 / 8
+                xs, ys = np.array([x], np.uint64), np.array([y], np.uint64)
+                O.lib().or_walk_bipartite(m, O._ptr(xs), O._ptr(ys), O._ptr(rec), 1, 1)
+                Pb[x + m * y, int(xs[0]) + m * int(ys[0])] += 1 / 8
+    assert np.allclose(Pf.sum(0), 1) and np.allclose(Pb.sum(0), 1)
+    d = np.zeros(n)
+    d[0] = 1
+    xodd = (np.arange(n) % m) % 2 == 1
+    for t in range(1, 21):
+        d = d @ (Pf if t % 2 == 1 else Pb)
+        assert abs(d[xodd].sum() - (1 - 0.75 ** t) / 2) < 1e-12
+    # variant 1 differs from variant 0 (odd steps go backwards)
+    assert not np.array_equal(O.bulk_v(256, 64, 64, 1, 3, 16, 0, 64), O.bulk_v(256, 64, 64, 0, 3, 16, 0, 64))
+    assert np.array_equal(O.bulk_v(256, 64, 64, 0, 3, 16, 0, 64), O.bulk(256, 64, 64, 3, 16, 0, 64))
