@@ -49,10 +49,12 @@ cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count);
 
 // Host feed: SplitMix64 counter-hash stream (R9), SoA rows.
 //   out[r*pitch + i] = word32(seed, tg0 + i, k0 + r),  r < nrows, i < count
+// nt: stream the stores past the CPU caches (bursty feeds; see feed.cpp).
 void feed_splitmix_rows(uint64_t seed, uint64_t tg0, uint64_t count, uint64_t k0,
-                        uint32_t nrows, uint32_t *out, uint64_t pitch);
+                        uint32_t nrows, uint32_t *out, uint64_t pitch, bool nt = false);
 // Same for an explicit walker list: column i = global walker base + ids[i].
 void feed_splitmix_rows_ids(uint64_t seed, uint64_t base, const uint32_t *ids, uint64_t count,
-                            uint64_t k0, uint32_t nrows, uint32_t *out, uint64_t pitch);
+                            uint64_t k0, uint32_t nrows, uint32_t *out, uint64_t pitch,
+                            bool nt = false);
 
 }  // namespace gg

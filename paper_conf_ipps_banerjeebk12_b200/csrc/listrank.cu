@@ -15,7 +15,10 @@
 //   sums over the splitter chain by pointer jumping; rank = prefix + local.
 // Phase III: re-insert removed nodes in reverse round order,
 //   rank(u) = rank(pred at removal) + distance at removal.
+#include <chrono>
 #include <cstdint>
+#include <cstdio>
+#include <cstdlib>
 #include <vector>
 
 #include <cub/cub.cuh>
@@ -223,19 +226,43 @@ extern "C" int gg_list_rank(prng_t *h, int64_t n, const int32_t *succ, const int
         std::vector<int64_t> round_off, round_cnt;
         prng_view view;
         // ---------------- Phase I
+        static const bool trace = getenv("GG_LR_TRACE") != nullptr;
         while (A > target && rounds < 1000) {
+            auto tr0 = std::chrono::steady_clock::now();
             LRC(prng_epoch_begin(h, (uint64_t)A, 1, s));
+            auto tr1 = std::chrono::steady_clock::now();
+            static const bool fine = trace && atoi(getenv("GG_LR_TRACE")) >= 2;
+            auto sync_t = [&](const char *what, std::chrono::steady_clock::time_point &t) {
+                if (!fine) return;
+                cudaStreamSynchronize(s);
+                auto now = std::chrono::steady_clock::now();
+                fprintf(stderr, "   %s %.3f ms\n", what,
+                        std::chrono::duration<double, std::milli>(now - t).count());
+                t = now;
+            };
+            auto tq = std::chrono::steady_clock::now();
+            sync_t("copy-wait", tq);
             LRC(prng_device_view(h, &view, sizeof(view)));
             lr_draw<<<nblk(A, 128), 128, 0, s>>>(view, act, A, bit);
             LRC(prng_epoch_end(h, s));
+            sync_t("draw", tq);
             draws += A;
             lr_decide<<<nblk(A), 256, 0, s>>>(act, A, bit, d_pred, d_succ, (int32_t)head, tail, keep);
             lr_splice<<<nblk(A), 256, 0, s>>>(act, A, keep, d_pred, d_succ, w, rem_pred, rem_dist,
                                               removed_round, (int32_t)rounds);
+            sync_t("decide+splice", tq);
             LCK(cub::DevicePartition::Flagged(tmp, tmp_bytes, act, keep, act2, d_num, (int)A, s));
+            sync_t("partition", tq);
             int32_t kept = 0;
             LCK(cudaMemcpyAsync(&kept, d_num, 4, cudaMemcpyDeviceToHost, s));
             LCK(cudaStreamSynchronize(s));
+            if (trace) {
+                auto tr2 = std::chrono::steady_clock::now();
+                fprintf(stderr, "[lr] round %ld A=%ld feed+enqueue %.3f ms, kernels+sync %.3f ms\n",
+                        (long)rounds, (long)A,
+                        std::chrono::duration<double, std::milli>(tr1 - tr0).count(),
+                        std::chrono::duration<double, std::milli>(tr2 - tr1).count());
+            }
             const int64_t gone = A - kept;
             LCK(cudaMemcpyAsync(rem_log + log_off, act2 + kept, (size_t)gone * 4,
                                 cudaMemcpyDeviceToDevice, s));

@@ -188,10 +188,12 @@ void free_all(prng_s *h) {
 }
 
 // Generate rows [k0, k0+nrows) of the streams of local walkers [wa, wb)
-// into buf (pitch = wb - wa words), in parallel over walkers.
+// (or of walkers ids[wa..wb)) into buf (row pitch bpitch words), in parallel
+// over walkers; streaming_stores: see feed.cpp.
 void feed_chunk(prng_s *h, uint64_t wa, uint64_t wb, uint64_t k0, uint32_t nrows, uint32_t *buf,
-                const uint32_t *ids) {
+                const uint32_t *ids, uint64_t bpitch, bool streaming_stores) {
     const uint64_t cw = wb - wa;
+    const bool nt_st = streaming_stores;
     const unsigned nt = h->pool->size();
     auto t0 = std::chrono::steady_clock::now();
     h->pool->run([&](unsigned ti) {
@@ -203,18 +205,18 @@ void feed_chunk(prng_s *h, uint64_t wa, uint64_t wb, uint64_t k0, uint32_t nrows
             if (h->o.bit_source == PRNG_BITS_CALLBACK) {
                 for (uint64_t i = lo; i < hi; i++)  // one walker at a time
                     h->o.bits_fn(h->o.bits_ctx, h->o.walker_base + ids[wa + i], 1, k0, nrows,
-                                 buf + i, cw);
+                                 buf + i, bpitch);
             } else {
                 gg::feed_splitmix_rows_ids(h->seed, h->o.walker_base, ids + wa + lo, hi - lo, k0,
-                                           nrows, buf + lo, cw);
+                                           nrows, buf + lo, bpitch, nt_st);
             }
             return;
         }
         const uint64_t tg0 = h->o.walker_base + wa + lo;
         if (h->o.bit_source == PRNG_BITS_CALLBACK)
-            h->o.bits_fn(h->o.bits_ctx, tg0, hi - lo, k0, nrows, buf + lo, cw);
+            h->o.bits_fn(h->o.bits_ctx, tg0, hi - lo, k0, nrows, buf + lo, bpitch);
         else
-            gg::feed_splitmix_rows(h->seed, tg0, hi - lo, k0, nrows, buf + lo, cw);
+            gg::feed_splitmix_rows(h->seed, tg0, hi - lo, k0, nrows, buf + lo, bpitch, nt_st);
     });
     auto t1 = std::chrono::steady_clock::now();
     h->stats.feed_seconds += std::chrono::duration<double>(t1 - t0).count();
@@ -226,31 +228,79 @@ void feed_chunk(prng_s *h, uint64_t wa, uint64_t wb, uint64_t k0, uint32_t nrows
 // pinned chunk while the previous chunks are DMA'd on copy_stream.
 // On return every copy is enqueued on copy_stream.
 void stage_rows(prng_s *h, uint64_t k0, uint64_t nrows, uint64_t Wv, uint32_t *dst,
-                uint64_t dpitch, const uint32_t *ids = nullptr) {
+                uint64_t dpitch, const uint32_t *ids = nullptr, bool bursty = false) {
     if (nrows == 0 || Wv == 0) return;
     const uint64_t chunk_words = h->chunk_bytes / 4;
-    uint64_t rows_per, walkers_per;
-    if (Wv <= chunk_words) {
-        walkers_per = Wv;
-        rows_per = std::max<uint64_t>(1, chunk_words / Wv);
-    } else {
-        walkers_per = chunk_words;
-        rows_per = 1;
+    // Chunks hold an even number of rows (>= 2) so each 64-bit SplitMix word
+    // feeds two rows (k even, k+1) with one hash.  Full-width chunks are
+    // generated at the device pitch, so each is ONE contiguous DMA (a 2D copy
+    // with pitch != width ran at 14-26 GB/s instead of ~46); windows wider
+    // than half a chunk are split by walkers, one contiguous DMA per row.
+    static const bool trace = getenv("GG_FEED_TRACE") != nullptr;
+    cudaEvent_t tr0 = nullptr, tr1 = nullptr;
+    auto host_t0 = std::chrono::steady_clock::now();
+    if (trace) {
+        cudaEventCreate(&tr0);
+        cudaEventCreate(&tr1);
+        cudaEventRecord(tr0, h->copy_stream);
     }
-    for (uint64_t r = 0; r < nrows; r += rows_per) {
-        const uint32_t nr = (uint32_t)std::min<uint64_t>(rows_per, nrows - r);
+    struct TraceEnd {
+        prng_s *h;
+        cudaEvent_t a, b;
+        std::chrono::steady_clock::time_point t0;
+        uint64_t bytes0;
+        ~TraceEnd() {
+            if (!a) return;
+            cudaEventRecord(b, h->copy_stream);
+            auto t1 = std::chrono::steady_clock::now();
+            cudaEventSynchronize(b);
+            auto t2 = std::chrono::steady_clock::now();
+            float ms = 0;
+            cudaEventElapsedTime(&ms, a, b);
+            fprintf(stderr, "[feed] %.1f MB: host gen+enqueue %.3f ms, copy stream %.3f ms (events), "
+                    "host wait after enqueue %.3f ms\n",
+                    (h->stats.h2d_bytes - bytes0) / 1e6,
+                    std::chrono::duration<double, std::milli>(t1 - t0).count(), ms,
+                    std::chrono::duration<double, std::milli>(t2 - t1).count());
+            cudaEventDestroy(a);
+            cudaEventDestroy(b);
+        }
+    } trace_end{h, tr0, tr1, host_t0, h->stats.h2d_bytes};
+    if (2 * dpitch <= chunk_words) {
+        uint64_t rows_per = std::max<uint64_t>(2, (chunk_words / dpitch) & ~1ull);
+        for (uint64_t r = 0; r < nrows;) {
+            uint64_t nr = std::min<uint64_t>(rows_per, nrows - r);
+            if (((k0 + r) & 1) && nr > 1) nr -= 1;  // keep later chunks pair-aligned
+            const int b = h->chunk_next;
+            h->chunk_next = (b + 1) % prng_s::kChunks;
+            CK(cudaEventSynchronize(h->chunk_done[b]));  // pinned chunk free again
+            feed_chunk(h, 0, Wv, k0 + r, (uint32_t)nr, h->chunk[b], ids, dpitch, bursty);
+            CK(cudaMemcpyAsync(dst + r * dpitch, h->chunk[b], nr * dpitch * 4,
+                               cudaMemcpyHostToDevice, h->copy_stream));
+            CK(cudaEventRecord(h->chunk_done[b], h->copy_stream));
+            h->stats.h2d_bytes += nr * dpitch * 4;
+            r += nr;
+        }
+        return;
+    }
+    const uint64_t walkers_per = std::max<uint64_t>(32, (chunk_words / 2) & ~31ull);
+    for (uint64_t r = 0; r < nrows;) {
+        uint64_t nr = std::min<uint64_t>(2, nrows - r);
+        if (((k0 + r) & 1) && nr > 1) nr = 1;
         for (uint64_t wa = 0; wa < Wv; wa += walkers_per) {
             const uint64_t wb = std::min<uint64_t>(Wv, wa + walkers_per);
             const int b = h->chunk_next;
             h->chunk_next = (b + 1) % prng_s::kChunks;
-            CK(cudaEventSynchronize(h->chunk_done[b]));  // pinned chunk free again
-            feed_chunk(h, wa, wb, k0 + r, nr, h->chunk[b], ids);
+            CK(cudaEventSynchronize(h->chunk_done[b]));
             const uint64_t cw = wb - wa;
-            CK(cudaMemcpy2DAsync(dst + r * dpitch + wa, dpitch * 4, h->chunk[b], cw * 4, cw * 4,
-                                 nr, cudaMemcpyHostToDevice, h->copy_stream));
+            feed_chunk(h, wa, wb, k0 + r, (uint32_t)nr, h->chunk[b], ids, cw, bursty);
+            for (uint64_t i = 0; i < nr; i++)  // one contiguous DMA per row segment
+                CK(cudaMemcpyAsync(dst + (r + i) * dpitch + wa, h->chunk[b] + i * cw, cw * 4,
+                                   cudaMemcpyHostToDevice, h->copy_stream));
             CK(cudaEventRecord(h->chunk_done[b], h->copy_stream));
             h->stats.h2d_bytes += (uint64_t)nr * cw * 4;
         }
+        r += nr;
     }
 }
 
@@ -741,8 +791,11 @@ static int epoch_begin_impl(prng_t *h, uint64_t active_walkers, const uint32_t *
             h->od_wmap = h->od_wmap_buf[slot];
             h->stats.h2d_bytes += active_walkers * 4;
         }
+        // small windows are bursty (the consumer waits for the last chunk):
+        // stream them past the CPU caches; large windows pipeline like bulk
+        const bool bursty = bytes < (1ull << 30);
         stage_rows(h, 2 + h->R0 + h->R * J0, (uint64_t)draws * h->R, active_walkers, h->od_bits,
-                   pitch, ids);
+                   pitch, ids, bursty);
         join_copies(h, s);
         h->od_J0 = J0;
         h->od_D = draws;
@@ -837,3 +890,85 @@ int prng_destroy(prng_t *h) {
 }
 
 }  // extern "C"
+
+// Diagnostic (not part of the ABI): time H2D copies from the handle's pinned
+// chunk 0 and from fresh pinned buffers allocated different ways.
+extern "C" int gg_debug_h2d_probe(prng_t *h, uint64_t bytes) {
+    if (!h || bytes > h->chunk_bytes) return PRNG_E_INVALID;
+    cudaSetDevice(h->o.device);
+    void *d = nullptr;
+    if (cudaMalloc(&d, bytes) != cudaSuccess) return PRNG_E_NOMEM;
+    cudaPointerAttributes at{};
+    cudaPointerGetAttributes(&at, h->chunk[0]);
+    fprintf(stderr, "[probe] chunk0 %p type %d devicePointer %p\n", (void *)h->chunk[0], (int)at.type,
+            at.devicePointer);
+    void *p_def = nullptr, *p_mh = nullptr, *p_reg = nullptr;
+    cudaHostAlloc(&p_def, bytes, cudaHostAllocDefault);
+    cudaMallocHost(&p_mh, bytes);
+    p_reg = aligned_alloc(4096, (bytes + 4095) / 4096 * 4096);
+    cudaHostRegister(p_reg, (bytes + 4095) / 4096 * 4096, cudaHostRegisterDefault);
+    memset(p_def, 1, bytes);
+    memset(p_mh, 1, bytes);
+    memset(p_reg, 1, bytes);
+    cudaEvent_t a, b;
+    cudaEventCreate(&a);
+    cudaEventCreate(&b);
+    const char *names[4] = {"chunk0(portable)", "hostalloc-default", "mallochost", "registered"};
+    void *srcs[4] = {h->chunk[0], p_def, p_mh, p_reg};
+    for (int k = 0; k < 4; k++) {
+        for (int rep = 0; rep < 3; rep++) {
+            cudaEventRecord(a, h->copy_stream);
+            cudaMemcpyAsync(d, srcs[k], bytes, cudaMemcpyHostToDevice, h->copy_stream);
+            cudaEventRecord(b, h->copy_stream);
+            cudaEventSynchronize(b);
+            float ms = 0;
+            cudaEventElapsedTime(&ms, a, b);
+            fprintf(stderr, "[probe] %-18s %.1f MB: %.3f ms (%.1f GB/s)\n", names[k], bytes / 1e6, ms,
+                    bytes / 1e6 / ms);
+        }
+    }
+    // copy right after the feed wrote the chunk: pool threads vs one thread
+    const uint64_t words = bytes / 4;
+    for (int mode = 0; mode < 3; mode++) {
+        for (int rep = 0; rep < 3; rep++) {
+            auto t0 = std::chrono::steady_clock::now();
+            if (mode == 0)
+                feed_chunk(h, 0, words / 6, 8, 6, h->chunk[0], nullptr, words / 6, true);
+            else if (mode == 1)
+                gg::feed_splitmix_rows(h->seed, 0, words / 6, 8, 6, h->chunk[0], words / 6);
+            else
+                memset(h->chunk[0], rep, bytes);
+            auto t1 = std::chrono::steady_clock::now();
+            cudaEventRecord(a, h->copy_stream);
+            cudaMemcpyAsync(d, h->chunk[0], bytes, cudaMemcpyHostToDevice, h->copy_stream);
+            cudaEventRecord(b, h->copy_stream);
+            cudaEventSynchronize(b);
+            float ms = 0;
+            cudaEventElapsedTime(&ms, a, b);
+            fprintf(stderr, "[probe] after %s write (%.3f ms): copy %.3f ms\n",
+                    mode == 0 ? "pool-feed" : mode == 1 ? "1-thread-feed" : "memset",
+                    std::chrono::duration<double, std::milli>(t1 - t0).count(), ms);
+        }
+    }
+    // same copy on a fresh default-flag stream
+    cudaStream_t s2;
+    cudaStreamCreate(&s2);
+    for (int rep = 0; rep < 3; rep++) {
+        cudaEventRecord(a, s2);
+        cudaMemcpyAsync(d, h->chunk[0], bytes, cudaMemcpyHostToDevice, s2);
+        cudaEventRecord(b, s2);
+        cudaEventSynchronize(b);
+        float ms = 0;
+        cudaEventElapsedTime(&ms, a, b);
+        fprintf(stderr, "[probe] chunk0 on new stream: %.3f ms\n", ms);
+    }
+    cudaStreamDestroy(s2);
+    cudaEventDestroy(a);
+    cudaEventDestroy(b);
+    cudaFreeHost(p_def);
+    cudaFreeHost(p_mh);
+    cudaHostUnregister(p_reg);
+    free(p_reg);
+    cudaFree(d);
+    return PRNG_OK;
+}

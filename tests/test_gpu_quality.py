@@ -1,0 +1,71 @@
+"""Statistical quality of full-size GPU output (SURVEY §8(f) f4, P7-P9 at scale).
+
+The paper's batteries (DIEHARD, TestU01; §IV-B Tables II-III) are not
+available offline; these are the oracle's chi-square / serial / gap tests
+run on 2^26 numbers of the C2 generator (m = 2^32) computed on the GPU,
+with a negative control: with l = 16 steps per number the serial test on
+(x mod 2, y mod 2) of consecutive draws must fail (the parity chain mixes at
+rate 3/4 per step, P4: divergence ~2 (3/4)^32 ~ 2e-4 per pair).
+"""
+import numpy as np
+import pytest
+from scipy import stats
+
+pytestmark = pytest.mark.gpu
+ALPHA = 1e-3
+
+
+def gen(l, n_draws=64, W=1 << 20, seed=0x5EED0002):
+    import torch
+    from paper_conf_ipps_banerjeebk12_b200 import Generator
+    g = Generator(walkers=W, seed=seed, walk_len=l)
+    o = torch.empty(W * n_draws, dtype=torch.int64, device="cuda")
+    g.fill(o)
+    torch.cuda.synchronize()
+    return o.view(n_draws, W)
+
+
+def chi2_p(counts, expected):
+    counts = counts.double().cpu().numpy()
+    chi = ((counts - expected) ** 2 / expected).sum()
+    return stats.chi2.sf(chi, counts.size - 1)
+
+
+def test_bytes_bits_serial_gap_l64():
+    import torch
+    z = gen(64)
+    flat = z.reshape(-1)
+    N = flat.numel()
+    # each byte of the label uniform over 256 values
+    for b in range(8):
+        v = (flat >> (8 * b)) & 0xFF
+        assert chi2_p(torch.bincount(v, minlength=256), N / 256) > ALPHA, b
+    # each of the 64 bits fair within 5 sigma
+    for bit in range(64):
+        ones = ((flat >> bit) & 1).sum().item()
+        assert abs(ones - N / 2) < 5 * 0.5 * N ** 0.5, bit
+    # serial: consecutive draws of the same walker, parity and top-bit projections
+    a, c = z[:-1].reshape(-1), z[1:].reshape(-1)
+    par = lambda v: (v & 1) | (((v >> 32) & 1) << 1)
+    cell = par(a) * 4 + par(c)
+    assert chi2_p(torch.bincount(cell, minlength=16), cell.numel() / 16) > ALPHA
+    top = lambda v: (((v >> 30) & 3) | (((v >> 62) & 3) << 2))
+    cell = top(a) * 16 + top(c)
+    assert chi2_p(torch.bincount(cell, minlength=256), cell.numel() / 256) > ALPHA
+    # gap test on the top bit along each walker's sequence (first 4096 walkers)
+    bits = ((z[:, :4096] >> 63) & 1).T.reshape(-1).cpu().numpy()
+    idx = np.flatnonzero(bits)
+    gaps = np.minimum(np.diff(idx) - 1, 10)
+    counts = np.bincount(gaps, minlength=11).astype(float)
+    p = np.array([0.5 ** (g + 1) for g in range(10)] + [0.5 ** 10])
+    chi = ((counts - p * gaps.size) ** 2 / (p * gaps.size)).sum()
+    assert stats.chi2.sf(chi, 10) > ALPHA
+
+
+def test_negative_control_l16_serial_parity_fails():
+    import torch
+    z = gen(16, n_draws=16)
+    a, c = z[:-1].reshape(-1), z[1:].reshape(-1)
+    par = lambda v: (v & 1) | (((v >> 32) & 1) << 1)
+    cell = par(a) * 4 + par(c)
+    assert chi2_p(torch.bincount(cell, minlength=16), cell.numel() / 16) < 1e-10
