@@ -60,6 +60,10 @@ enum {
 
 enum {
     PRNG_BITS_SPLITMIX = 0, /* canonical counter-addressed SplitMix64 stream (R9) */
+    PRNG_BITS_RANDR = 1,    /* paper-faithful: per-walker glibc rand_r LCG streams (P:14
+                               "the LCG present in the glibc library"); word k of walker t
+                               = low 16 bits of outputs 2k, 2k+1 of the stream seeded with
+                               low32(seed ^ (t+1)*0x9E3779B97F4A7C15) */
     PRNG_BITS_CALLBACK = 2  /* user callback supplies the words (tests, fault injection) */
 };
 

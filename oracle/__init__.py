@@ -68,6 +68,9 @@ def lib():
                 "or_sigma_array": (None, [u64, ctypes.c_int, P, P, P, P, u64]),
                 "or_stream_block": (None, [u64, u64, u64, u64, u32, P]),
                 "or_sigma_inv": (None, [u64, ctypes.c_int, u64, u64, P, P]),
+                "or_rand_r": (ctypes.c_int32, [P]),
+                "or_stream_word32_randr": (u32, [u64, u64, u64]),
+                "or_set_bit_source": (None, [ctypes.c_int]),
                 "or_walk_bipartite": (None, [u64, P, P, P, u32, u64]),
                 "or_walker_init_v": (ctypes.c_int, [u64, u32, u32, u64, u64, P, P]),
                 "or_walker_draw_v": (u64, [u64, u32, u32, u32, u64, u64, u64, P, P]),
@@ -176,6 +179,19 @@ def bulk(m: int, l: int, l0: int, seed: int, W: int, g0: int, n: int) -> np.ndar
     if rc != 0:
         raise ValueError("or_bulk failed")
     return out
+
+
+class bit_source:
+    """Context manager selecting the oracle's seed-bit stream (0 = SplitMix64, 1 = rand_r)."""
+
+    def __init__(self, src: int):
+        self.src = src
+
+    def __enter__(self):
+        lib().or_set_bit_source(self.src)
+
+    def __exit__(self, *exc):
+        lib().or_set_bit_source(0)
 
 
 def sigma_inv(m: int, k: int, x: int, y: int):

@@ -31,10 +31,11 @@ def params(m: int = 1 << 32, walk_len: int = 64, burnin_len: int = 64, degree: i
 
 
 def options(device: int = 0, walker_base: int = 0, epoch_draws: int = 16, host_threads: int = 0,
-            bits_fn=None, bits_ctx=None) -> _lib.prng_options:
+            bits_fn=None, bits_ctx=None, bit_source: int = 0) -> _lib.prng_options:
     o = _lib.prng_options()
     check(_lib.prng_default_options(ctypes.byref(o)))
     o.device, o.walker_base, o.epoch_draws, o.host_threads = device, walker_base, epoch_draws, host_threads
+    o.bit_source = bit_source
     if bits_fn is not None:
         o.bit_source = PRNG_BITS_CALLBACK
         o.bits_fn = bits_fn
@@ -65,7 +66,8 @@ class Generator:
 
     def __init__(self, walkers: int, seed: int, m: int = 1 << 32, walk_len: int = 64,
                  burnin_len: int = 64, device: int = 0, walker_base: int = 0,
-                 epoch_draws: int = 16, host_threads: int = 0, bits_fn=None, variant: int = 0):
+                 epoch_draws: int = 16, host_threads: int = 0, bits_fn=None, variant: int = 0,
+                 bit_source: int = 0):
         self._h = ctypes.c_void_p()
         self.walkers, self.seed, self.m, self.walk_len = walkers, seed, m, walk_len
         self._walker_base = walker_base
@@ -81,7 +83,8 @@ class Generator:
                     buf[r * pitch:r * pitch + nwalkers] = a[r]
             self._bits_fn = _lib.PRNG_BITS_FN(_cb)
         p = params(m, walk_len, burnin_len, variant=variant)
-        o = options(device, walker_base, epoch_draws, host_threads, self._bits_fn)
+        o = options(device, walker_base, epoch_draws, host_threads, self._bits_fn,
+                    bit_source=bit_source)
         check(_lib.prng_create(ctypes.byref(self._h), ctypes.byref(p), walkers, seed,
                                ctypes.byref(o)), "prng_create")
 

@@ -57,4 +57,10 @@ void feed_splitmix_rows_ids(uint64_t seed, uint64_t base, const uint32_t *ids, u
                             uint64_t k0, uint32_t nrows, uint32_t *out, uint64_t pitch,
                             bool nt = false);
 
+// Paper-faithful glibc rand_r seed bits (bit_source 1): see feed.cpp.
+void feed_randr_rows(uint64_t seed, uint64_t tg0, uint64_t count, uint64_t k0, uint32_t nrows,
+                     uint32_t *out, uint64_t pitch);
+void feed_randr_rows_ids(uint64_t seed, uint64_t base, const uint32_t *ids, uint64_t count,
+                         uint64_t k0, uint32_t nrows, uint32_t *out, uint64_t pitch);
+
 }  // namespace gg

@@ -202,7 +202,10 @@ void feed_chunk(prng_s *h, uint64_t wa, uint64_t wb, uint64_t k0, uint32_t nrows
         uint64_t lo = std::min<uint64_t>(cw, per * ti), hi = std::min<uint64_t>(cw, lo + per);
         if (lo >= hi) return;
         if (ids) {
-            if (h->o.bit_source == PRNG_BITS_CALLBACK) {
+            if (h->o.bit_source == PRNG_BITS_RANDR) {
+                gg::feed_randr_rows_ids(h->seed, h->o.walker_base, ids + wa + lo, hi - lo, k0,
+                                        nrows, buf + lo, bpitch);
+            } else if (h->o.bit_source == PRNG_BITS_CALLBACK) {
                 for (uint64_t i = lo; i < hi; i++)  // one walker at a time
                     h->o.bits_fn(h->o.bits_ctx, h->o.walker_base + ids[wa + i], 1, k0, nrows,
                                  buf + i, bpitch);
@@ -213,7 +216,9 @@ void feed_chunk(prng_s *h, uint64_t wa, uint64_t wb, uint64_t k0, uint32_t nrows
             return;
         }
         const uint64_t tg0 = h->o.walker_base + wa + lo;
-        if (h->o.bit_source == PRNG_BITS_CALLBACK)
+        if (h->o.bit_source == PRNG_BITS_RANDR)
+            gg::feed_randr_rows(h->seed, tg0, hi - lo, k0, nrows, buf + lo, bpitch);
+        else if (h->o.bit_source == PRNG_BITS_CALLBACK)
             h->o.bits_fn(h->o.bits_ctx, tg0, hi - lo, k0, nrows, buf + lo, bpitch);
         else
             gg::feed_splitmix_rows(h->seed, tg0, hi - lo, k0, nrows, buf + lo, bpitch, nt_st);
@@ -469,7 +474,8 @@ int prng_create(prng_t **out, const prng_graph_params *g, uint64_t walkers, uint
     if (!pow2 && g->m > (1ull << 30)) return PRNG_E_UNSUPPORTED;
     if (g->walk_len < 1 || g->walk_len > 4096 || g->burnin_len > 4096) return PRNG_E_INVALID;
     if (walkers + o.walker_base > (1ull << 24)) return PRNG_E_INVALID;
-    if (o.bit_source != PRNG_BITS_SPLITMIX && o.bit_source != PRNG_BITS_CALLBACK)
+    if (o.bit_source != PRNG_BITS_SPLITMIX && o.bit_source != PRNG_BITS_RANDR &&
+        o.bit_source != PRNG_BITS_CALLBACK)
         return PRNG_E_INVALID;
     if (o.bit_source == PRNG_BITS_CALLBACK && !o.bits_fn) return PRNG_E_INVALID;
     if (o.epoch_draws == 0) o.epoch_draws = 16;

@@ -75,3 +75,65 @@ def test_walker_list_rows(feed, n, k0, nt):
     got = buf[off:off + rows * pitch].reshape(rows, pitch)[:, :n]
     want = np.stack([O.stream_block(11, 500 + int(t), 1, k0, rows)[:, 0] for t in ids], axis=1)
     assert np.array_equal(got, want)
+
+
+# ------------------------------------------------ f3: glibc rand_r seed bits
+def test_oracle_rand_r_is_glibc():
+    # the oracle's plain rand_r vs the system C library's (an independent
+    # implementation of the paper's "LCG present in the glibc library")
+    libc = ctypes.CDLL("libc.so.6")
+    libc.rand_r.argtypes = [ctypes.POINTER(ctypes.c_uint)]
+    for seed0 in (1, 12345, 0xFFFFFFFF, 0, 0x5EED0002):
+        a = ctypes.c_uint(seed0)
+        b = np.array([seed0], np.uint32)
+        for _ in range(200):
+            assert libc.rand_r(ctypes.byref(a)) == O.lib().or_rand_r(b.ctypes.data)
+            assert a.value == int(b[0])
+
+
+RANDR_SHIM = r'''
+#include <cstdint>
+namespace gg {
+void feed_randr_rows(uint64_t, uint64_t, uint64_t, uint64_t, uint32_t, uint32_t *, uint64_t);
+void feed_randr_rows_ids(uint64_t, uint64_t, const uint32_t *, uint64_t, uint64_t, uint32_t,
+                         uint32_t *, uint64_t);
+}
+extern "C" void run(uint64_t s, uint64_t t0, uint64_t n, uint64_t k0, uint32_t r, uint32_t *o,
+                    uint64_t p) { gg::feed_randr_rows(s, t0, n, k0, r, o, p); }
+extern "C" void run_ids(uint64_t s, uint64_t b, const uint32_t *ids, uint64_t n, uint64_t k0,
+                        uint32_t r, uint32_t *o, uint64_t p) {
+    gg::feed_randr_rows_ids(s, b, ids, n, k0, r, o, p);
+}
+'''
+
+
+@pytest.fixture(scope="module")
+def randr_feed(tmp_path_factory):
+    d = tmp_path_factory.mktemp("randr")
+    src, so = d / "shim.cpp", d / "shim.so"
+    src.write_text(RANDR_SHIM)
+    feed_src = os.path.join(ROOT, "paper_conf_ipps_banerjeebk12_b200", "csrc", "feed.cpp")
+    subprocess.check_call(["g++", "-O2", "-std=c++17", "-shared", "-fPIC", "-I",
+                           os.path.join(ROOT, "paper_conf_ipps_banerjeebk12_b200", "csrc"),
+                           "-I", "/usr/local/cuda/include", "-o", str(so), str(src), feed_src])
+    return ctypes.CDLL(str(so))
+
+
+@pytest.mark.parametrize("k0,rows", [(0, 8), (8, 6), (37, 3), (1000, 2)])
+def test_randr_feed_jump_ahead_matches_plain_replay(randr_feed, k0, rows):
+    n, pitch, seed, t0 = 50, 64, 0x5EED0001, 3
+    buf = np.zeros(rows * pitch, np.uint32)
+    randr_feed.run(ctypes.c_uint64(seed), ctypes.c_uint64(t0), ctypes.c_uint64(n), ctypes.c_uint64(k0),
+                   ctypes.c_uint32(rows), ctypes.c_void_p(buf.ctypes.data), ctypes.c_uint64(pitch))
+    got = buf.reshape(rows, pitch)[:, :n]
+    for i in (0, 7, n - 1):
+        for r in range(rows):
+            assert got[r, i] == O.lib().or_stream_word32_randr(seed, t0 + i, k0 + r)
+    ids = np.array([9, 2, 40], np.uint32)
+    randr_feed.run_ids(ctypes.c_uint64(seed), ctypes.c_uint64(100), ctypes.c_void_p(ids.ctypes.data),
+                       ctypes.c_uint64(3), ctypes.c_uint64(k0), ctypes.c_uint32(rows),
+                       ctypes.c_void_p(buf.ctypes.data), ctypes.c_uint64(pitch))
+    got = buf.reshape(rows, pitch)[:, :3]
+    for i, t in enumerate(ids):
+        for r in range(rows):
+            assert got[r, i] == O.lib().or_stream_word32_randr(seed, 100 + int(t), k0 + r)

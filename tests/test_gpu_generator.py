@@ -270,3 +270,15 @@ def test_bipartite_on_demand(torch_cuda):
     z = o.view(W, D).cpu().numpy().view(np.uint64)
     want = O.bulk_v(M32, 64, 64, 1, seed, W, 0, W * D).reshape(D, W).T
     assert np.array_equal(z, want)
+
+
+def test_randr_bit_source_parity(torch_cuda):
+    # f3: paper-faithful glibc rand_r seed bits (bit_source 1), bulk + on-demand
+    torch = torch_cuda
+    W, seed = 256, 0x5EED0001
+    g = G(walkers=W, seed=seed, bit_source=1, m=256)
+    o = torch.empty(W * 4 + 3, dtype=torch.int64, device="cuda")
+    g.fill(o)
+    with O.bit_source(1):
+        want = O.bulk(256, 64, 64, seed, W, 0, W * 4 + 3)
+    assert np.array_equal(as_u64(o), want)
