@@ -289,4 +289,35 @@ __device__ __forceinline__ uint64_t prng_next(prng_state *st, const prng_view *v
     return gg_label(x, y, v->m, v->log2m, v->pow2 != 0);
 }
 
+/* K draws at once: the K records' loads are issued together before the
+ * first walk, so a consumer that needs several numbers per iteration (the
+ * Monte Carlo consumer takes three) waits for memory once, not K times.
+ * Same numbers, same order, same overrun rule as K calls of prng_next. */
+template <int K>
+__device__ __forceinline__ void prng_next_n(prng_state *st, const prng_view *v, uint64_t (&out)[K])
+{
+    if (!(v->l == 64u && v->pow2 && v->variant == 0) || st->used + K > v->D ||
+        st->slot >= v->Wv) {
+#pragma unroll
+        for (int k = 0; k < K; k++) out[k] = prng_next(st, v);
+        return;
+    }
+    uint32_t w[K][6];
+#pragma unroll
+    for (int k = 0; k < K; k++) {
+        const uint32_t *rec = v->bits + (uint64_t)(st->used + k) * 6u * v->pitch + st->slot;
+#pragma unroll
+        for (int r = 0; r < 6; r++) w[k][r] = __ldg(rec + (uint64_t)r * v->pitch);
+    }
+    uint32_t x = st->x, y = st->y;
+#pragma unroll
+    for (int k = 0; k < K; k++) {
+        gg_walk64(w[k], x, y);
+        out[k] = gg_label(x, y, v->m, v->log2m, true);
+    }
+    st->x = x;
+    st->y = y;
+    st->used += K;
+}
+
 #endif /* GGPRNG_PRNG_DEVICE_CUH */

@@ -22,7 +22,17 @@ __global__ void __launch_bounds__(128) consume_kernel(prng_view v, uint64_t thre
     prng_state st = prng_state_load(&v, (uint32_t)t);
     uint64_t acc = 0;
     const uint64_t base = out ? (offsets ? offsets[t] : t * (uint64_t)uniform) : 0;
-    for (uint32_t r = 0; r < c; r++) {
+    uint32_t r = 0;
+    for (; r + 4 <= c; r += 4) {  // four records' loads in flight together
+        uint64_t z4[4];
+        prng_next_n<4>(&st, &v, z4);
+#pragma unroll
+        for (int k = 0; k < 4; k++) {
+            acc ^= z4[k];
+            if (out) out[base + r + k] = z4[k];
+        }
+    }
+    for (; r < c; r++) {
         const uint64_t z = prng_next(&st, &v);
         acc ^= z;
         if (out) out[base + r] = z;

@@ -17,6 +17,7 @@
 // GPUs (NCCL) if sharded.
 #include <cmath>
 #include <cstdint>
+#include <cstdlib>
 #include <vector>
 
 #include <cub/cub.cuh>
@@ -117,20 +118,28 @@ __global__ void mc_init_state(McState s, uint64_t n, uint32_t *iota) {
     iota[i] = (uint32_t)i;
 }
 
-__global__ void __launch_bounds__(128) mc_epoch(prng_view v, McParams P, McState S,
+template <int MINB>
+__global__ void __launch_bounds__(128, MINB) mc_epoch(prng_view v, McParams P, McState S,
                                                 unsigned long long *tallies,
                                                 long long *per_thread,
                                                 unsigned long long *counters) {
     const uint64_t slot = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const int nt = kFixed + P.nl;
-    long long tal[kFixed + kMaxL];
-#pragma unroll
-    for (int k = 0; k < kFixed + kMaxL; k++) tal[k] = 0;
+    // block tallies in shared memory (int64 atomics: exact, order independent)
+    __shared__ unsigned long long s_tal[kFixed + kMaxL];
+    for (int k = threadIdx.x; k < kFixed + kMaxL; k += blockDim.x) s_tal[k] = 0;
+    __syncthreads();
+    long long *my_row = nullptr;
+    auto tally = [&](int k, uint64_t v) {
+        if (v) atomicAdd(&s_tal[k], (unsigned long long)v);
+        if (my_row) my_row[k] += (long long)v;
+    };
     unsigned long long launched_now = 0, interactions = 0, draws = 0, done = 0;
     if (slot < v.Wv) {
         // the window holds the threads that still had work one epoch ago
         const uint64_t i = v.wmap ? v.wmap[slot] : slot;
         const uint64_t tg = P.thread0 + i;
+        if (per_thread) my_row = per_thread + i * nt;
         const uint64_t budget =
             P.photons_total / P.threads_total + (tg < P.photons_total % P.threads_total ? 1 : 0);
         double x = S.x[i], y = S.y[i], z = S.z[i], ux = S.ux[i], uy = S.uy[i], uz = S.uz[i];
@@ -142,17 +151,17 @@ __global__ void __launch_bounds__(128) mc_epoch(prng_view v, McParams P, McState
         prng_state st = prng_state_load(&v, (uint32_t)slot);
         for (uint32_t it = 0; it < P.K; it++) {
             if (!alive && launched == budget) break;
-            // three draws at a convergent point (R22)
-            const uint64_t la = prng_next(&st, &v);
-            const uint64_t lb = prng_next(&st, &v);
-            const uint64_t lc = prng_next(&st, &v);
+            // three draws at a convergent point (R22), their loads in flight together
+            uint64_t d3[3];
+            prng_next_n<3>(&st, &v, d3);
+            const uint64_t la = d3[0], lb = d3[1], lc = d3[2];
             draws += 3;
             if (!alive) {
                 // Alg.4 l.3: launch a photon with its weight from getnextrand()
                 const uint64_t w0 = (la >> 32) + 1;
                 const uint64_t sp = mc_frac(w0, P.q_sp);
-                tal[0] += (long long)w0;
-                tal[1] += (long long)sp;
+                tally(0, w0);
+                tally(1, sp);
                 w = w0 - sp;
                 x = 0.0;
                 y = 0.0;
@@ -192,7 +201,7 @@ __global__ void __launch_bounds__(128) mc_epoch(prng_view v, McParams P, McState
                 if (reflect) {
                     uz = -uz;
                 } else if (nb == 0 || nb == P.nl + 1) {
-                    tal[nb == 0 ? 2 : 3] += (long long)w;
+                    tally(nb == 0 ? 2 : 3, w);
                     w = 0;
                     alive = false;
                 } else {
@@ -210,7 +219,7 @@ __global__ void __launch_bounds__(128) mc_epoch(prng_view v, McParams P, McState
                 sleft = 0.0;
                 const uint64_t dw = mc_frac(w, P.qabs[layer]);
                 w -= dw;
-                tal[kFixed + layer - 1] += (long long)dw;
+                tally(kFixed + layer - 1, dw);
                 const double cost = mc_hg(g, mc_xi(lb));
                 const double psi = 2.0 * kPi * mc_xi(lc);
                 const double cosp = cos(psi), sinp = sin(psi);
@@ -228,7 +237,7 @@ __global__ void __launch_bounds__(128) mc_epoch(prng_view v, McParams P, McState
                 }
                 interactions++;
                 if (w < P.w_th) {
-                    tal[4] += (long long)w;
+                    tally(4, w);
                     w = 0;
                     alive = false;
                 }
@@ -248,16 +257,11 @@ __global__ void __launch_bounds__(128) mc_epoch(prng_view v, McParams P, McState
         S.launched[i] = launched;
         done = (!alive && launched == budget) ? 1 : 0;
         S.busy[i] = done ? 0 : 1;
-        if (per_thread)
-            for (int k = 0; k < nt; k++) per_thread[i * nt + k] += tal[k];
     }
-    // warp-level integer reductions, one atomic per warp and counter
+    __syncthreads();
+    for (int k = threadIdx.x; k < nt; k += blockDim.x)
+        if (s_tal[k]) atomicAdd(&tallies[k], s_tal[k]);
     const unsigned full = 0xFFFFFFFFu;
-    for (int k = 0; k < nt; k++) {
-        unsigned long long vsum = (unsigned long long)tal[k];
-        for (int o = 16; o > 0; o >>= 1) vsum += __shfl_down_sync(full, vsum, o);
-        if ((threadIdx.x & 31) == 0 && vsum) atomicAdd(&tallies[k], vsum);
-    }
     unsigned long long c[4] = {launched_now, draws, interactions, done};
     for (int k = 0; k < 4; k++) {
         unsigned long long vsum = c[k];
@@ -381,8 +385,28 @@ extern "C" int gg_mc_run(prng_t *h, const gg_mc_config *cfg, int64_t *tallies, i
                 prng_view v;
                 MRC(prng_device_view(h, &v, sizeof(v)));
                 MCK(cudaEventRecord(k0, s));
-                mc_epoch<<<(unsigned)((wslots + 127) / 128), 128, 0, s>>>(
-                    v, P, S, d_tal, (long long *)per_thread, d_cnt);
+                static const int minb = getenv("GG_MC_MINB") ? atoi(getenv("GG_MC_MINB")) : 8;
+                if (minb >= 12)
+                    mc_epoch<12><<<(unsigned)((wslots + 127) / 128), 128, 0, s>>>(
+                        v, P, S, d_tal, (long long *)per_thread, d_cnt);
+                else if (minb >= 10)
+                    mc_epoch<10><<<(unsigned)((wslots + 127) / 128), 128, 0, s>>>(
+                        v, P, S, d_tal, (long long *)per_thread, d_cnt);
+                else if (minb >= 8)
+                    mc_epoch<8><<<(unsigned)((wslots + 127) / 128), 128, 0, s>>>(
+                        v, P, S, d_tal, (long long *)per_thread, d_cnt);
+                else if (minb == 7)
+                    mc_epoch<7><<<(unsigned)((wslots + 127) / 128), 128, 0, s>>>(
+                        v, P, S, d_tal, (long long *)per_thread, d_cnt);
+                else if (minb >= 6)
+                    mc_epoch<6><<<(unsigned)((wslots + 127) / 128), 128, 0, s>>>(
+                        v, P, S, d_tal, (long long *)per_thread, d_cnt);
+                else if (minb == 5)
+                    mc_epoch<5><<<(unsigned)((wslots + 127) / 128), 128, 0, s>>>(
+                        v, P, S, d_tal, (long long *)per_thread, d_cnt);
+                else
+                    mc_epoch<4><<<(unsigned)((wslots + 127) / 128), 128, 0, s>>>(
+                        v, P, S, d_tal, (long long *)per_thread, d_cnt);
                 MCK(cudaGetLastError());
                 MCK(cudaEventRecord(k1, s));
                 MRC(prng_epoch_end(h, s));
