@@ -172,6 +172,9 @@ def run_ours(args, rank, world, local_rank):
     dev = torch.device("cuda", local_rank)
     props = torch.cuda.get_device_properties(dev)
     stream = torch.cuda.current_stream()
+    # the ranks of one node share the host cores for their FEED threads
+    local_world = int(os.environ.get("LOCAL_WORLD_SIZE", str(world)))
+    feed_threads = max(1, (os.cpu_count() or 1) // max(1, local_world))
 
     def barrier():
         if world > 1:
@@ -185,7 +188,8 @@ def run_ours(args, rank, world, local_rank):
         return float(t.item())
 
     # ---- K-mode: bits resident in HBM, one prng_fill per step
-    g = Generator(walkers=W_PER_GPU, seed=SEED, walker_base=rank * W_PER_GPU, device=local_rank)
+    g = Generator(walkers=W_PER_GPU, seed=SEED, walker_base=rank * W_PER_GPU, device=local_rank,
+                  host_threads=feed_threads)
     g.prefetch(DRAWS_PER_STEP)
     g.mark()
     out = torch.empty(U32_PER_STEP, dtype=torch.int32, device=dev)
@@ -301,14 +305,14 @@ def run_ours(args, rank, world, local_rank):
 
     # ---- on-demand consumers of the paper at full size (C3, C4), one run each
     if not args.no_apps:
-        res["apps"] = run_apps(args, rank, world, local_rank, max_over_ranks)
+        res["apps"] = run_apps(args, rank, world, local_rank, max_over_ranks, feed_threads)
         torch.cuda.empty_cache()
 
     # ---- e2e: host buffers through prng_fill_host (FEED + H2D + walk + D2H)
     if not args.no_e2e:
         e2e_steps = max(1, min(args.steps, args.e2e_steps))
         g = Generator(walkers=W_PER_GPU, seed=SEED, walker_base=rank * W_PER_GPU,
-                      device=local_rank, epoch_draws=16)
+                      device=local_rank, epoch_draws=16, host_threads=feed_threads)
         host = torch.empty(U32_PER_STEP, dtype=torch.int32).pin_memory()
         g.fill_host(host, n=W_PER_GPU * 2 * 16)  # warm (allocations, feed threads)
         g.mark()
@@ -329,13 +333,13 @@ def run_ours(args, rank, world, local_rank):
             "steps": e2e_steps,
             "feed_s_per_step": (s1["feed_seconds"] - s0["feed_seconds"]) / e2e_steps,
             "api": "prng_fill_host (host FEED threads -> pinned -> H2D -> walk -> D2H to pinned)",
-            "host_threads": os.cpu_count(),
+            "host_threads": feed_threads,
         }
         g.close()
     return res
 
 
-def run_apps(args, rank, world, local_rank, max_over_ranks):
+def run_apps(args, rank, world, local_rank, max_over_ranks, feed_threads=0):
     """C3 list ranking (2^24 nodes, replica per GPU) and C4 Monte Carlo (2^20
     threads per GPU, 20 photons each, ~2^32 draws per GPU; integer tallies
     all-reduced over ranks).  Numbers are device-timed inside the C ABI."""
@@ -348,7 +352,7 @@ def run_apps(args, rank, world, local_rank, max_over_ranks):
     # C3: list ranking of a 2^24-node random list (every rank ranks its own copy)
     n = 1 << 24
     succ, pred, head = inputs.random_list(n, 0x5EED0003)
-    g = Generator(walkers=n, seed=0x5EED0003, device=local_rank)
+    g = Generator(walkers=n, seed=0x5EED0003, device=local_rank, host_threads=feed_threads)
     s_t, p_t = torch.from_numpy(succ).to(dev), torch.from_numpy(pred).to(dev)
     torch.cuda.synchronize()
     t = time.perf_counter()
@@ -373,7 +377,8 @@ def run_apps(args, rank, world, local_rank, max_over_ranks):
     from paper_conf_ipps_banerjeebk12_b200 import dist as gd
     thread0, T, T_total = gd.mc_shard(rank, world, W_PER_GPU)
     P_per = 20
-    g = Generator(walkers=T, seed=0x5EED0004, walker_base=thread0, device=local_rank)
+    g = Generator(walkers=T, seed=0x5EED0004, walker_base=thread0, device=local_rank,
+                  host_threads=feed_threads)
     layers = ((1.37, 1.0, 100.0, 0.9, 0.1), (1.37, 1.0, 10.0, 0.0, 0.1), (1.37, 2.0, 10.0, 0.7, 0.2))
     torch.cuda.synchronize()
     t = time.perf_counter()
@@ -416,6 +421,10 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    # test hooks: run the multi-rank path on one GPU (gloo, shared device)
+    backend = os.environ.get("GG_DIST_BACKEND", "nccl")
+    if "GG_FORCE_DEVICE" in os.environ:
+        local_rank = int(os.environ["GG_FORCE_DEVICE"])
 
     if args.impl == "reference":
         if rank != 0:
@@ -431,7 +440,10 @@ def main():
         import torch
         import torch.distributed as dist
         torch.cuda.set_device(local_rank)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        else:
+            dist.init_process_group(backend)
     res = run_ours(args, rank, world, local_rank)
     if rank == 0:
         line = {
