@@ -349,20 +349,25 @@ def run_apps(args, rank, world, local_rank, max_over_ranks, feed_threads=0):
     from paper_conf_ipps_banerjeebk12_b200 import Generator
     dev = torch.device("cuda", local_rank)
     out = {}
-    # C3: list ranking of a 2^24-node random list (every rank ranks its own copy)
+    # C3: list ranking of a 2^24-node random list.  With world > 1 the ranks
+    # share Phase II (sublist walks) and exchange the splitter records
+    # (allgather) and reduced-list ranks (allreduce) over NCCL.
+    from paper_conf_ipps_banerjeebk12_b200 import dist as gd_
+    coll = gd_.Collective(device=dev) if world > 1 else None
     n = 1 << 24
     succ, pred, head = inputs.random_list(n, 0x5EED0003)
     g = Generator(walkers=n, seed=0x5EED0003, device=local_rank, host_threads=feed_threads)
     s_t, p_t = torch.from_numpy(succ).to(dev), torch.from_numpy(pred).to(dev)
     torch.cuda.synchronize()
     t = time.perf_counter()
-    rank_t, info = g.list_rank(s_t, p_t, head)
+    rank_t, info = g.list_rank(s_t, p_t, head, collective=coll)
     torch.cuda.synchronize()
     wall = max_over_ranks(time.perf_counter() - t)
     ok = int(rank_t[head].item()) == 0 and int(rank_t.max().item()) == n - 1
     dev_us = info["phase1_us"] + info["phase2_us"] + info["phase3_us"]
     out["list_ranking"] = {
         "config": "C3: random list of 2^24 nodes, walker = active slot, b(u) = bit 63",
+        "splitter_exchange": world > 1,
         "rounds": info["rounds"], "reduced": info["reduced"], "splitters": info["splitters"],
         "draws": info["draws"], "ms_device": dev_us / 1e3, "ms_wall": wall * 1e3,
         "phase_ms": [info["phase1_us"] / 1e3, info["phase2_us"] / 1e3, info["phase3_us"] / 1e3],

@@ -38,6 +38,26 @@ int gg_consume(prng_t *h, uint64_t threads, const uint32_t *counts, uint32_t uni
                uint64_t *out, const uint64_t *offsets, uint64_t *xor_out, void *stream);
 
 /*
+ * Collectives supplied by the caller for multi-GPU runs (one process per
+ * GPU).  The library stays independent of any communication runtime: the
+ * Python layer implements these with torch.distributed (NCCL over
+ * NVLink/NVSwitch on the GPU box, gloo in tests).  Buffers are DEVICE
+ * pointers of the calling rank's GPU; each call is synchronous with respect
+ * to the device work enqueued before it (the library synchronises its
+ * stream first) and returns 0 on success.
+ *   allgather     : recv[r * bytes + i] = send_of_rank_r[i], i < bytes
+ *   allreduce_i32 : buf[i] = sum over ranks of buf_of_rank[i], i < count
+ */
+typedef int (*gg_allgather_fn)(void *ctx, const void *send, void *recv, size_t bytes);
+typedef int (*gg_allreduce_i32_fn)(void *ctx, int32_t *buf, size_t count);
+typedef struct {
+    int rank, world;
+    gg_allgather_fn allgather;
+    gg_allreduce_i32_fn allreduce_i32;
+    void *ctx;
+} gg_collective;
+
+/*
  * Randomised list ranking (§V): rank[v] = distance of node v
  * from the head (R17), computed by Alg.3 ReduceList (FIS rounds with
  * on-demand draws), Helman-JaJa [10] splitter ranking of the reduced
@@ -57,12 +77,22 @@ int gg_consume(prng_t *h, uint64_t threads, const uint32_t *counts, uint32_t uni
  *   is_splitter   : optional device int32[n]: 1 for Phase II splitters.
  *   info          : optional HOST int64[8]: rounds, reduced size, splitters,
  *                   draws, Phase I / II / III device microseconds, rounds.
+ *   coll          : NULL for one GPU.  With world > 1 every rank calls with the
+ *                   same list and a generator of the same seed and walker ids:
+ *                   Phase I is replicated (it is deterministic), Phase II walks
+ *                   only this rank's share of the splitters' sublists, the
+ *                   splitter records (sublist length, next splitter) are
+ *                   exchanged with one allgather (the north star's "splitter
+ *                   exchange"), the prefix over splitters is computed on every
+ *                   rank, the reduced-list ranks are combined with one int32
+ *                   allreduce, and Phase III runs replicated; every rank ends
+ *                   with the full rank array.
  * Synchronous (returns when rank is final).  Temporary device memory is
  * stream-ordered (cudaMallocAsync) on `stream`.
  */
 int gg_list_rank(prng_t *h, int64_t n, const int32_t *succ, const int32_t *pred, int64_t head,
                  int32_t *rank, int32_t *removed_round, int32_t *is_splitter, int64_t *info,
-                 void *stream);
+                 const gg_collective *coll, void *stream);
 
 /* ---------------------------------------------------------------------------
  * Monte Carlo photon migration (§VI, Alg.4): photons from a

@@ -164,17 +164,21 @@ class Generator:
         check(_lib.gg_consume(self._h, threads, ptr(counts), uniform, ptr(out), ptr(offsets),
                               ptr(xor_out), _stream_handle(stream)), "gg_consume")
 
-    def list_rank(self, succ, pred, head: int, removed_round=None, is_splitter=None, stream=None):
+    def list_rank(self, succ, pred, head: int, removed_round=None, is_splitter=None, stream=None,
+                  collective=None):
         """gg_list_rank: ranks (distance from head) of a linked list given as CUDA int32 arrays.
 
+        collective: None (one GPU) or a dist.Collective (multi-GPU splitter exchange).
         Returns (rank tensor, info dict)."""
         import torch
         n = succ.numel()
         rank = torch.empty(n, dtype=torch.int32, device=succ.device)
         info = (ctypes.c_int64 * 8)()
         ptr = lambda t: None if t is None else t.data_ptr()
+        coll = None if collective is None else ctypes.byref(collective.struct())
         check(_lib.gg_list_rank(self._h, n, succ.data_ptr(), pred.data_ptr(), head, rank.data_ptr(),
-                                ptr(removed_round), ptr(is_splitter), info, _stream_handle(stream)),
+                                ptr(removed_round), ptr(is_splitter), info, coll,
+                                _stream_handle(stream)),
               "gg_list_rank")
         keys = ("rounds", "reduced", "splitters", "draws", "phase1_us", "phase2_us", "phase3_us",
                 "rounds2")

@@ -68,6 +68,15 @@ class gg_mc_config(ctypes.Structure):
                 ("threads", u64), ("epoch_draws", u32), ("w_threshold", ctypes.c_double)]
 
 
+GG_ALLGATHER_FN = ctypes.CFUNCTYPE(c_int, vp, vp, vp, sz)
+GG_ALLREDUCE_I32_FN = ctypes.CFUNCTYPE(c_int, vp, vp, sz)
+
+
+class gg_collective(ctypes.Structure):
+    _fields_ = [("rank", c_int), ("world", c_int), ("allgather", GG_ALLGATHER_FN),
+                ("allreduce_i32", GG_ALLREDUCE_I32_FN), ("ctx", vp)]
+
+
 class prng_view(ctypes.Structure):
     """Mirror of struct prng_view (include/prng_device.cuh)."""
     _fields_ = [("bits", vp), ("wmap", vp), ("x", vp), ("y", vp), ("j", vp), ("flags", vp), ("pitch", u64),
@@ -101,7 +110,8 @@ _SIGS = {
     "prng_destroy": (c_int, [vp]),
     # include/gg_apps.h
     "gg_consume": (c_int, [vp, u64, vp, u32, vp, vp, vp, vp]),
-    "gg_list_rank": (c_int, [vp, ctypes.c_int64, vp, vp, ctypes.c_int64, vp, vp, vp, vp, vp]),
+    "gg_list_rank": (c_int, [vp, ctypes.c_int64, vp, vp, ctypes.c_int64, vp, vp, vp, vp,
+                             ctypes.POINTER(gg_collective), vp]),
     "gg_mc_run": (c_int, [vp, ctypes.POINTER(gg_mc_config), vp, vp, vp, vp]),
 }
 

@@ -117,12 +117,12 @@ __global__ void lr_splitter_index(const int32_t *spl, int64_t ns, int32_t *spl_i
     if (k < ns) spl_idx[spl[k]] = (int32_t)k;
 }
 
-// Sublist walk: splitter k follows succ to the next splitter.
-__global__ void lr_sublist(const int32_t *spl, int64_t ns, const int32_t *succ, const int32_t *w,
-                           const uint8_t *spl_node, const int32_t *spl_idx, int32_t *local,
-                           int32_t *sub, int32_t *len, int32_t *nextk) {
-    const int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (k >= ns) return;
+// Sublist walk: splitter k in [k0, k1) follows succ to the next splitter.
+__global__ void lr_sublist(const int32_t *spl, int64_t k0, int64_t k1, const int32_t *succ,
+                           const int32_t *w, const uint8_t *spl_node, const int32_t *spl_idx,
+                           int32_t *local, int32_t *sub, int32_t *len, int32_t *nextk) {
+    const int64_t k = k0 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (k >= k1) return;
     int32_t v = spl[k], off = 0;
     for (;;) {
         local[v] = off;
@@ -153,15 +153,50 @@ __global__ void lr_jump(int64_t ns, const int32_t *val_in, const int32_t *nxt_in
     }
 }
 
-// rank = (total - suffix of own sublist) + local offset.
+// rank = (total - suffix of own sublist) + local offset, for nodes whose
+// sublist this rank walked (sub >= 0); slot_rank[i] gets the same value (0
+// for nodes of other ranks) for the cross-rank sum.
 __global__ void lr_fixup(const int32_t *act, int64_t A, const int32_t *sub, const int32_t *local,
                          const int32_t *suffix, const int32_t *spl_idx, int32_t head,
-                         int32_t *rank) {
+                         int32_t *rank, int32_t *slot_rank) {
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= A) return;
     const int32_t v = act[i];
-    const int32_t total = suffix[spl_idx[head]];
-    rank[v] = total - suffix[sub[v]] + local[v];
+    const int32_t sb = sub[v];
+    int32_t r = 0;
+    if (sb >= 0) {
+        const int32_t total = suffix[spl_idx[head]];
+        r = total - suffix[sb] + local[v];
+        rank[v] = r;
+    }
+    if (slot_rank) slot_rank[i] = r;
+}
+
+// Rebuild the full splitter tables from the allgathered per-rank chunks:
+// rank q contributed splitters [q*ns/G, (q+1)*ns/G) at offset q*chunk.
+__global__ void lr_unpack(const int2 *recv, int64_t ns, int world, int64_t chunk, int32_t *len,
+                          int32_t *nextk) {
+    const int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (k >= ns) return;
+    int q = (int)((k * world) / ns);
+    while (q + 1 < world && (q + 1) * ns / world <= k) q++;
+    while (q > 0 && q * ns / world > k) q--;
+    const int64_t k0 = q * ns / world;
+    const int2 rec = recv[q * chunk + (k - k0)];
+    len[k] = rec.x;
+    nextk[k] = rec.y;
+}
+
+__global__ void lr_pack(const int32_t *len, const int32_t *nextk, int64_t k0, int64_t k1,
+                        int2 *send) {
+    const int64_t k = k0 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (k < k1) send[k - k0] = make_int2(len[k], nextk[k]);
+}
+
+__global__ void lr_scatter_slot_rank(const int32_t *act, int64_t A, const int32_t *slot_rank,
+                                     int32_t *rank) {
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < A) rank[act[i]] = slot_rank[i];
 }
 
 __global__ void lr_reinsert(const int32_t *list, int64_t cnt, const int32_t *rem_pred,
@@ -178,8 +213,14 @@ inline unsigned nblk(int64_t n, int t = 256) { return (unsigned)((n + t - 1) / t
 
 extern "C" int gg_list_rank(prng_t *h, int64_t n, const int32_t *succ, const int32_t *pred,
                             int64_t head, int32_t *rank, int32_t *removed_round,
-                            int32_t *is_splitter, int64_t *info, void *stream) {
+                            int32_t *is_splitter, int64_t *info, const gg_collective *coll,
+                            void *stream) {
     if (!h || n <= 0 || !succ || !pred || !rank || head < 0 || head >= n) return PRNG_E_INVALID;
+    const int world = coll ? coll->world : 1;
+    const int me = coll ? coll->rank : 0;
+    if (world < 1 || me < 0 || me >= world ||
+        (world > 1 && (!coll->allgather || !coll->allreduce_i32)))
+        return PRNG_E_INVALID;
     if (n > (1ll << 24)) return PRNG_E_UNSUPPORTED;
     cudaStream_t s = (cudaStream_t)stream;
     std::vector<void *> bufs;
@@ -292,9 +333,26 @@ extern "C" int gg_list_rank(prng_t *h, int64_t n, const int32_t *succ, const int
         int32_t *local = (int32_t *)alloc(n4), *sub = (int32_t *)alloc(n4);
         int32_t *va = (int32_t *)alloc((size_t)ns * 4), *na = (int32_t *)alloc((size_t)ns * 4);
         int32_t *vb = (int32_t *)alloc((size_t)ns * 4), *nb = (int32_t *)alloc((size_t)ns * 4);
+        LCK(cudaMemsetAsync(sub, 0xFF, n4, s));  // -1: not in a sublist walked here
         lr_splitter_index<<<nblk(ns), 256, 0, s>>>(spl, ns, spl_idx);
-        lr_sublist<<<nblk(ns, 128), 128, 0, s>>>(spl, ns, d_succ, w, spl_node, spl_idx, local, sub,
-                                                va, na);
+        // this rank's share of the sublists (all of them on one GPU)
+        const int64_t k0 = (int64_t)me * ns / world, k1 = (int64_t)(me + 1) * ns / world;
+        if (k1 > k0)
+            lr_sublist<<<nblk(k1 - k0, 128), 128, 0, s>>>(spl, k0, k1, d_succ, w, spl_node, spl_idx,
+                                                         local, sub, va, na);
+        int32_t *slot_rank = nullptr;
+        if (world > 1) {
+            // splitter exchange: one allgather of (sublist length, next splitter)
+            const int64_t chunk = (ns + world - 1) / world;
+            int2 *send = (int2 *)alloc((size_t)chunk * 8);
+            int2 *recv = (int2 *)alloc((size_t)chunk * 8 * world);
+            if (k1 > k0) lr_pack<<<nblk(k1 - k0), 256, 0, s>>>(va, na, k0, k1, send);
+            LCK(cudaStreamSynchronize(s));
+            if (coll->allgather(coll->ctx, send, recv, (size_t)chunk * 8) != 0)
+                throw Fail{PRNG_E_CUDA};
+            lr_unpack<<<nblk(ns), 256, 0, s>>>(recv, ns, world, chunk, va, na);
+            slot_rank = (int32_t *)alloc((size_t)A * 4);
+        }
         int iters = 0;
         while ((1ll << iters) < (int64_t)ns) iters++;
         for (int it = 0; it <= iters; it++) {
@@ -302,7 +360,14 @@ extern "C" int gg_list_rank(prng_t *h, int64_t n, const int32_t *succ, const int
             std::swap(va, vb);
             std::swap(na, nb);
         }
-        lr_fixup<<<nblk(A), 256, 0, s>>>(act, A, sub, local, va, spl_idx, (int32_t)head, rank);
+        lr_fixup<<<nblk(A), 256, 0, s>>>(act, A, sub, local, va, spl_idx, (int32_t)head, rank,
+                                        slot_rank);
+        if (world > 1) {
+            // every reduced node was ranked by exactly one rank: sum the slot arrays
+            LCK(cudaStreamSynchronize(s));
+            if (coll->allreduce_i32(coll->ctx, slot_rank, (size_t)A) != 0) throw Fail{PRNG_E_CUDA};
+            lr_scatter_slot_rank<<<nblk(A), 256, 0, s>>>(act, A, slot_rank, rank);
+        }
         LCK(cudaEventRecord(ev[2], s));
         // ---------------- Phase III
         for (int64_t r = rounds - 1; r >= 0; r--) {

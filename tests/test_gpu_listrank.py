@@ -80,3 +80,97 @@ def test_c3_full_size_ranks_and_fis_invariants():
         lab = int(O.walker_draws(M32, 64, 64, 0x5EED0003, i, info["rounds"], 1)[0])
         v = reduced[i]
         assert bool(spl[v]) == (v == order[0] or (lab >> 58) == 0), i
+
+
+class _FakeCollective:
+    """Two ranks as two host threads of this process sharing one GPU: the
+    gg_collective callbacks exchange through host copies behind a barrier.
+    Exercises the sharded Phase II and the splitter exchange without NCCL."""
+
+    def __init__(self, world):
+        import threading
+        self.world = world
+        self.bar = threading.Barrier(world)
+        self.slots = [None] * world
+
+    def member(self, rank):
+        import ctypes
+        import torch
+        from paper_conf_ipps_banerjeebk12_b200 import _lib
+        from paper_conf_ipps_banerjeebk12_b200.dist import _device_view
+        fc = self
+        dev = torch.device("cuda", 0)
+
+        def allgather(ctx, send, recv, nbytes):
+            fc.slots[rank] = _device_view(send, nbytes, dev).cpu()
+            fc.bar.wait()
+            _device_view(recv, nbytes * fc.world, dev).copy_(torch.cat(fc.slots))
+            torch.cuda.synchronize()
+            fc.bar.wait()
+            return 0
+
+        def allreduce(ctx, buf, count):
+            fc.slots[rank] = _device_view(buf, count * 4, dev).view(torch.int32).cpu()
+            fc.bar.wait()
+            tot = sum(s.to(torch.int64) for s in fc.slots).to(torch.int32)
+            fc.bar.wait()
+            _device_view(buf, count * 4, dev).view(torch.int32).copy_(tot)
+            torch.cuda.synchronize()
+            return 0
+
+        class M:
+            def __init__(self):
+                self._ag = _lib.GG_ALLGATHER_FN(allgather)
+                self._ar = _lib.GG_ALLREDUCE_I32_FN(allreduce)
+
+            def struct(self):
+                return _lib.gg_collective(rank, fc.world, self._ag, self._ar, None)
+        return M()
+
+
+@pytest.mark.parametrize("n,world", [(2, 2), (1000, 2), (1 << 16, 2), (1 << 16, 3), (200000, 4)])
+def test_sharded_splitter_exchange(n, world):
+    """world > 1: every rank ends with the exact ranks; FIS and splitter sets
+    equal the one-GPU run (Phase I and the splitter choice are replicated)."""
+    import threading
+    import torch
+    from paper_conf_ipps_banerjeebk12_b200 import Generator
+    succ, pred, head = inputs.random_list(n, 7 + n)
+    seed = 0x5EED0003
+    single = run_gpu(succ, pred, head, seed)
+    fc = _FakeCollective(world)
+    res = [None] * world
+    errs = []
+
+    def worker(r):
+        try:
+            torch.cuda.set_device(0)
+            st = torch.cuda.Stream()
+            with torch.cuda.stream(st):
+                g = Generator(walkers=n, seed=seed)
+                s = torch.from_numpy(succ).cuda()
+                p = torch.from_numpy(pred).cuda()
+                rr = torch.empty(n, dtype=torch.int32, device="cuda")
+                sp = torch.empty(n, dtype=torch.int32, device="cuda")
+                rank, info = g.list_rank(s, p, head, removed_round=rr, is_splitter=sp,
+                                         stream=st, collective=fc.member(r))
+                st.synchronize()
+                res[r] = (rank.cpu().numpy(), rr.cpu().numpy(), sp.cpu().numpy().astype(bool), info)
+                g.close()
+        except Exception as e:  # pragma: no cover - surfaced below
+            errs.append(e)
+            fc.bar.abort()
+
+    th = [threading.Thread(target=worker, args=(r,)) for r in range(world)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join(timeout=300)
+    assert not errs, errs
+    ref = O.lr_rank_seq(succ, head)
+    for r in range(world):
+        rank, rr, sp, info = res[r]
+        assert np.array_equal(rank, ref), r
+        assert np.array_equal(rr, single["removed_round"]), r
+        assert np.array_equal(sp, single["is_splitter"]), r
+        assert info["splitters"] == single["info"]["splitters"]
