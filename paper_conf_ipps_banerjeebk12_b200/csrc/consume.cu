@@ -19,6 +19,10 @@ __global__ void __launch_bounds__(128) consume_kernel(prng_view v, uint64_t thre
     const uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= threads) return;
     const uint32_t c = counts ? counts[t] : uniform;
+    if (c == 0) {  // idle this launch: the walker's state is untouched
+        if (xor_out) xor_out[t] = 0;
+        return;
+    }
     prng_state st = prng_state_load(&v, (uint32_t)t);
     uint64_t acc = 0;
     const uint64_t base = out ? (offsets ? offsets[t] : t * (uint64_t)uniform) : 0;

@@ -63,4 +63,8 @@ void feed_randr_rows(uint64_t seed, uint64_t tg0, uint64_t count, uint64_t k0, u
 void feed_randr_rows_ids(uint64_t seed, uint64_t base, const uint32_t *ids, uint64_t count,
                          uint64_t k0, uint32_t nrows, uint32_t *out, uint64_t pitch);
 
+// Library-owned stream-ordered scratch pool of the current device (listrank.cu):
+// keeps its memory between calls; nullptr on CUDA failure.
+cudaMemPool_t scratch_pool();
+
 }  // namespace gg

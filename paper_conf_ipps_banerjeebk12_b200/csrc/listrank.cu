@@ -19,12 +19,15 @@
 #include <cstdint>
 #include <cstdio>
 #include <cstdlib>
+#include <map>
+#include <mutex>
 #include <vector>
 
 #include <cub/cub.cuh>
 #include <cuda_runtime.h>
 
 #include "gg_apps.h"
+#include "gg_internal.h"
 #include "prng.h"
 #include "prng_device.cuh"
 
@@ -211,6 +214,30 @@ inline unsigned nblk(int64_t n, int t = 256) { return (unsigned)((n + t - 1) / t
 
 }  // namespace
 
+// Stream-ordered scratch pool of this library, one per device, that keeps its
+// memory between calls (release threshold = max): the default pool returns
+// freed memory to the driver at every synchronisation, and re-mapping the
+// ~0.7 GB of C3 scratch made repeated calls' wall time erratic.
+cudaMemPool_t gg::scratch_pool() {
+    static std::mutex mu;
+    static std::map<int, cudaMemPool_t> pools;
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) return nullptr;
+    std::lock_guard<std::mutex> lk(mu);
+    auto it = pools.find(dev);
+    if (it != pools.end()) return it->second;
+    cudaMemPoolProps props{};
+    props.allocType = cudaMemAllocationTypePinned;
+    props.location.type = cudaMemLocationTypeDevice;
+    props.location.id = dev;
+    cudaMemPool_t p = nullptr;
+    if (cudaMemPoolCreate(&p, &props) != cudaSuccess) return nullptr;
+    uint64_t thr = UINT64_MAX;
+    cudaMemPoolSetAttribute(p, cudaMemPoolAttrReleaseThreshold, &thr);
+    pools[dev] = p;
+    return p;
+}
+
 extern "C" int gg_list_rank(prng_t *h, int64_t n, const int32_t *succ, const int32_t *pred,
                             int64_t head, int32_t *rank, int32_t *removed_round,
                             int32_t *is_splitter, int64_t *info, const gg_collective *coll,
@@ -224,9 +251,11 @@ extern "C" int gg_list_rank(prng_t *h, int64_t n, const int32_t *succ, const int
     if (n > (1ll << 24)) return PRNG_E_UNSUPPORTED;
     cudaStream_t s = (cudaStream_t)stream;
     std::vector<void *> bufs;
+    cudaMemPool_t pool = gg::scratch_pool();
+    if (!pool) return PRNG_E_CUDA;
     auto alloc = [&](size_t bytes) -> void * {
         void *p = nullptr;
-        LCK(cudaMallocAsync(&p, bytes ? bytes : 1, s));
+        LCK(cudaMallocFromPoolAsync(&p, bytes ? bytes : 1, pool, s));
         bufs.push_back(p);
         return p;
     };

@@ -24,6 +24,7 @@
 #include <cuda_runtime.h>
 
 #include "gg_apps.h"
+#include "gg_internal.h"
 #include "prng.h"
 #include "prng_device.cuh"
 
@@ -325,9 +326,11 @@ extern "C" int gg_mc_run(prng_t *h, const gg_mc_config *cfg, int64_t *tallies, i
     const int nt = kFixed + P.nl;
 
     std::vector<void *> bufs;
+    cudaMemPool_t pool = gg::scratch_pool();
+    if (!pool) return PRNG_E_CUDA;
     auto alloc = [&](size_t bytes) -> void * {
         void *p = nullptr;
-        MCK(cudaMallocAsync(&p, bytes, s));
+        MCK(cudaMallocFromPoolAsync(&p, bytes, pool, s));
         bufs.push_back(p);
         return p;
     };

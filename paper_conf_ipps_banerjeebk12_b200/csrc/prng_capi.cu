@@ -298,9 +298,13 @@ void stage_rows(prng_s *h, uint64_t k0, uint64_t nrows, uint64_t Wv, uint32_t *d
             h->chunk_next = (b + 1) % prng_s::kChunks;
             CK(cudaEventSynchronize(h->chunk_done[b]));
             const uint64_t cw = wb - wa;
-            feed_chunk(h, wa, wb, k0 + r, (uint32_t)nr, h->chunk[b], ids, cw, bursty);
+            // rows start 32-B aligned in the chunk, so the streaming-store path
+            // (feed.cpp nt_ok) covers the ragged last segment too: cached
+            // stores there halved the DMA rate of whole rounds (LR trace)
+            const uint64_t cp = round_up(cw, 8);
+            feed_chunk(h, wa, wb, k0 + r, (uint32_t)nr, h->chunk[b], ids, cp, bursty);
             for (uint64_t i = 0; i < nr; i++)  // one contiguous DMA per row segment
-                CK(cudaMemcpyAsync(dst + (r + i) * dpitch + wa, h->chunk[b] + i * cw, cw * 4,
+                CK(cudaMemcpyAsync(dst + (r + i) * dpitch + wa, h->chunk[b] + i * cp, cw * 4,
                                    cudaMemcpyHostToDevice, h->copy_stream));
             CK(cudaEventRecord(h->chunk_done[b], h->copy_stream));
             h->stats.h2d_bytes += (uint64_t)nr * cw * 4;

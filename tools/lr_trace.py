@@ -12,7 +12,7 @@ from paper_conf_ipps_banerjeebk12_b200 import Generator  # noqa: E402
 n = 1 << 24
 succ, pred, head = inputs.random_list(n, 0x5EED0003)
 s, p = torch.from_numpy(succ).cuda(), torch.from_numpy(pred).cuda()
-for rep in range(2):
+for rep in range(int(os.environ.get("REPS", "3"))):
     g = Generator(walkers=n, seed=0x5EED0003)
     torch.cuda.synchronize()
     t = time.perf_counter()
