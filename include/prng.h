@@ -195,6 +195,17 @@ int prng_epoch_begin_list(prng_t *h, const uint32_t *walkers, uint64_t count, ui
 int prng_epoch_end(prng_t *h, void *stream);
 
 /*
+ * Pre-allocate both device window slots (epochs are double-buffered) for
+ * windows of up to `active_walkers` x `draws`, so that later
+ * prng_epoch_begin calls within that size never allocate (no allocation or
+ * device synchronisation jitter inside a timed or latency-sensitive loop).
+ * Blocks until slots in use by earlier epochs are free.  Returns
+ * PRNG_E_INVALID for zero sizes or active_walkers > walkers, PRNG_E_STATE
+ * inside an open epoch.
+ */
+int prng_epoch_reserve(prng_t *h, uint64_t active_walkers, uint32_t draws);
+
+/*
  * Fill *view (a struct prng_view from prng_device.cuh, view_bytes =
  * sizeof(struct prng_view)) for the open epoch.  The view holds device
  * pointers; pass it by value to kernels.

@@ -146,6 +146,10 @@ class Generator:
         check(_lib.prng_epoch_begin_list(self._h, ids.ctypes.data, ids.size, draws,
                                          _stream_handle(stream)), "prng_epoch_begin_list")
 
+    def epoch_reserve(self, active_walkers: int, draws: int) -> None:
+        """prng_epoch_reserve: pre-allocate both window slots up to this size."""
+        check(_lib.prng_epoch_reserve(self._h, active_walkers, draws), "prng_epoch_reserve")
+
     def epoch_end(self, stream=None) -> None:
         check(_lib.prng_epoch_end(self._h, _stream_handle(stream)), "prng_epoch_end")
 

@@ -104,6 +104,7 @@ _SIGS = {
     "prng_epoch_begin": (c_int, [vp, u64, u32, vp]),
     "prng_epoch_begin_list": (c_int, [vp, vp, u64, u32, vp]),
     "prng_epoch_end": (c_int, [vp, vp]),
+    "prng_epoch_reserve": (c_int, [vp, ctypes.c_uint64, ctypes.c_uint32]),
     "prng_device_view": (c_int, [vp, vp, sz]),
     "prng_check": (c_int, [vp]),
     "prng_get_stats": (c_int, [vp, ctypes.POINTER(prng_stats)]),

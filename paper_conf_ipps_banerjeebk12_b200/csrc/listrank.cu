@@ -295,6 +295,9 @@ extern "C" int gg_list_rank(prng_t *h, int64_t n, const int32_t *succ, const int
         int64_t A = n, rounds = 0, draws = 0, log_off = 0;
         std::vector<int64_t> round_off, round_cnt;
         prng_view view;
+        // both window slots sized for the first (largest) round: the slot
+        // parity flips between calls (rounds + 1 epochs per call)
+        LRC(prng_epoch_reserve(h, (uint64_t)n, 1));
         // ---------------- Phase I
         static const bool trace = getenv("GG_LR_TRACE") != nullptr;
         while (A > target && rounds < 1000) {

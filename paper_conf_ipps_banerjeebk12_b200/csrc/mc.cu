@@ -382,6 +382,7 @@ extern "C" int gg_mc_run(prng_t *h, const gg_mc_config *cfg, int64_t *tallies, i
         MCK(cudaEventCreate(&k1));
         MCK(cudaEventCreateWithFlags(&kc, cudaEventDisableTiming));
         try {
+            MRC(prng_epoch_reserve(h, n, cfg->epoch_draws));  // no allocation inside the loop
             MRC(prng_epoch_begin(h, n, cfg->epoch_draws, s));
             uint64_t wslots = n;
             for (;;) {

@@ -834,6 +834,25 @@ int prng_epoch_begin_list(prng_t *h, const uint32_t *walkers, uint64_t count, ui
     return epoch_begin_impl(h, count, walkers, draws, stream);
 }
 
+int prng_epoch_reserve(prng_t *h, uint64_t active_walkers, uint32_t draws) {
+    if (!h) return PRNG_E_INVALID;
+    if (active_walkers == 0 || active_walkers > h->W || draws == 0) return PRNG_E_INVALID;
+    if (h->od_open) return PRNG_E_STATE;
+    return guard(h, [&] {
+        const size_t bytes = (size_t)draws * h->R * round_up(active_walkers, 32) * 4;
+        for (int slot = 0; slot < 2; slot++) {
+            if (bytes <= h->od_cap[slot]) continue;
+            CK(cudaEventSynchronize(h->od_free[slot]));
+            if (h->od_buf[slot]) CK(cudaFree(h->od_buf[slot]));
+            h->od_buf[slot] = nullptr;
+            h->od_cap[slot] = 0;
+            CK(cudaMalloc(&h->od_buf[slot], bytes));
+            h->od_cap[slot] = bytes;
+        }
+        return PRNG_OK;
+    });
+}
+
 int prng_epoch_end(prng_t *h, void *stream) {
     if (!h) return PRNG_E_INVALID;
     if (!h->od_open) return PRNG_E_STATE;

@@ -140,3 +140,35 @@ def test_epoch_with_walker_list():
         assert int(z2[t]) == ow.draw(3)
     ow = OracleWalker(M32, seed, 7)   # not listed: skipped draws 0..2
     assert int(z2[7]) == ow.draw(3)
+
+
+def test_epoch_reserve_same_numbers_and_errors():
+    """prng_epoch_reserve only pre-allocates: the numbers are unchanged, and
+    it is refused inside an open epoch or for empty / oversized windows."""
+    import torch
+    from paper_conf_ipps_banerjeebk12_b200 import Generator, PrngError
+    W, seed = 4096, 33
+    res = []
+    for reserve in (False, True):
+        g = Generator(walkers=W, seed=seed)
+        if reserve:
+            g.epoch_reserve(W, 3)
+        outs = []
+        for A, D in ((W, 3), (W // 2, 2), (W, 1), (100, 3)):
+            g.epoch_begin(A, D)
+            o = torch.empty(A * D, dtype=torch.int64, device="cuda")
+            g.consume(A, uniform=D, out=o)
+            g.epoch_end()
+            outs.append(o.cpu().numpy())
+        res.append(np.concatenate(outs))
+        if reserve:
+            with pytest.raises(PrngError):
+                g.epoch_reserve(0, 1)
+            with pytest.raises(PrngError):
+                g.epoch_reserve(W + 1, 1)
+            g.epoch_begin(10, 1)
+            with pytest.raises(PrngError):
+                g.epoch_reserve(10, 1)
+            g.epoch_end()
+        g.close()
+    assert np.array_equal(res[0], res[1])

@@ -69,3 +69,21 @@ def test_negative_control_l16_serial_parity_fails():
     par = lambda v: (v & 1) | (((v >> 32) & 1) << 1)
     cell = par(a) * 4 + par(c)
     assert chi2_p(torch.bincount(cell, minlength=16), cell.numel() / 16) < 1e-10
+
+
+def test_battery_on_gpu_output():
+    """SmallCrush-style battery (tests/battery.py) on 2^23 labels of the C2
+    generator computed on the GPU, bulk order and walker-major order."""
+    import battery as B
+    z = gen(64, n_draws=64, W=1 << 17).cpu().numpy()  # [draw, walker] int64
+    for name, arr in (("bulk", z), ("walker-major", z.T.copy())):
+        res = B.run(np.ascontiguousarray(arr).reshape(-1).view(np.uint32))
+        bad = {k: v for k, v in res.items() if v < 1e-4}
+        assert not bad, (name, bad)
+
+
+def test_battery_negative_control_l1_on_gpu():
+    import battery as B
+    z = gen(1, n_draws=1024, W=1 << 12).cpu().numpy()
+    res = B.run(np.ascontiguousarray(z.T).reshape(-1).view(np.uint32))
+    assert sum(v < 1e-10 for v in res.values()) >= 3, res
