@@ -91,3 +91,14 @@ def test_c4_full_size_conservation_and_sampled_parity():
         o = O.mc_run(nthreads=1, walker0=tg, threads_total=T, photons_total=P, D=192,
                      seed=0x5EED0004)
         assert np.array_equal(pt[tg], o["tallies"]), tg
+
+
+@pytest.mark.parametrize("T,P,D", [(1, 1, 3), (1, 5, 6), (100, 7, 3), (33, 1000, 9), (4096, 4095, 192)])
+def test_degenerate_sizes_exact_parity(T, P, D):
+    """Fewer photons than threads (idle threads), one thread, tiny epochs
+    (one iteration per epoch), photon counts not divisible by threads."""
+    g = gpu_mc(T, P, D=D, per_thread=True)
+    o = O.mc_run(nthreads=T, photons_total=P, D=D, seed=0x5EED0004, per_thread=True)
+    assert_tallies_match(g["tallies"], o["tallies"])
+    assert g["photons"] == P
+    assert np.array_equal(g["per_thread"], o["per_thread"])
