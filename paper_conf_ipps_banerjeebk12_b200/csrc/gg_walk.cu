@@ -352,7 +352,15 @@ __global__ void __launch_bounds__(64) gg_fill64x2_tma_kernel(const __grid_consta
 // ~10 instructions: the bound is HBM, not the integer pipes.  Each warp owns
 // 32 walkers; lane 0 streams 32-draw x 32-walker tiles (4 KB) by TMA into two
 // smem stages; lanes step through their column and store coalesced.
-constexpr int kL1Draws = 32;
+constexpr int kL1Draws = 16;
+
+// One l = 1 step for m = 2^k (wrapped): b -> sigma_{b mod 7} (§III-A).
+__device__ __forceinline__ void gg_step_l1(uint32_t b, uint32_t &x, uint32_t &y) {
+    const uint32_t cy = b - 1u, cx = b - 4u;
+    const uint32_t ty = y + 2u * x + cy, tx = x + 2u * y + cx;
+    y = (cy < 3u) ? ty : y;
+    x = (cx < 3u) ? tx : x;
+}
 
 template <int EMIT>
 __global__ void __launch_bounds__(64) gg_fill_l1_tma_kernel(const __grid_constant__ CUtensorMap tmap,
@@ -383,6 +391,9 @@ __global__ void __launch_bounds__(64) gg_fill_l1_tma_kernel(const __grid_constan
         const uint32_t jlo = __reduce_min_sync(0xFFFFFFFFu, j0);
         const uint32_t jhi = __reduce_max_sync(0xFFFFFFFFu, j1);
         if (jlo >= jhi) continue;
+        // draws every lane of the warp emits (empty if some lane is idle)
+        const uint32_t jin0 = __reduce_max_sync(0xFFFFFFFFu, j0);
+        const uint32_t jin1 = __reduce_min_sync(0xFFFFFFFFu, j1);
         const uint32_t ntiles = (jhi - jlo + kL1Draws - 1) / kL1Draws;
         uint32_t x = 0, y = 0;
         if (t < a.W) {
@@ -402,12 +413,25 @@ __global__ void __launch_bounds__(64) gg_fill_l1_tma_kernel(const __grid_constan
             if (sidx) ph1 ^= 1u; else ph0 ^= 1u;
             const uint32_t *buf = tiles[wib][sidx];
             const uint32_t jt = jlo + q * kL1Draws;
-#pragma unroll 8
-            for (uint32_t d = 0; d < kL1Draws; d++) {
-                const uint32_t j = jt + d;
-                if (j >= j0 && j < j1) {
-                    gg_step_generic(buf[d * 32 + lane] & 7u, x, y, 0, true);
-                    emit_label<EMIT>(a, (uint64_t)j * a.W + t - a.g_origin, x, y);
+            if (jt >= jin0 && jt + kL1Draws <= jin1) {
+                // interior tile (warp-uniform): all loads first, no per-draw tests
+                uint32_t b[kL1Draws];
+#pragma unroll
+                for (int d = 0; d < kL1Draws; d++) b[d] = buf[d * 32 + lane];
+                const uint64_t i0 = (uint64_t)jt * a.W + t - a.g_origin;
+#pragma unroll
+                for (int d = 0; d < kL1Draws; d++) {
+                    gg_step_l1(b[d] & 7u, x, y);
+                    emit_label<EMIT>(a, i0 + (uint64_t)d * a.W, x, y);
+                }
+            } else {
+#pragma unroll 4
+                for (uint32_t d = 0; d < kL1Draws; d++) {
+                    const uint32_t j = jt + d;
+                    if (j >= j0 && j < j1) {
+                        gg_step_l1(buf[d * 32 + lane] & 7u, x, y);
+                        emit_label<EMIT>(a, (uint64_t)j * a.W + t - a.g_origin, x, y);
+                    }
                 }
             }
             __syncwarp();
