@@ -81,7 +81,25 @@ def build(force: bool = False, verbose: bool = False) -> str:
         ["-lpthread", "-cudart", "static"]
     subprocess.check_call(cmd)
     os.replace(tmp, LIB)
+    build_examples()
     return LIB
+
+
+EXAMPLES = os.path.join(ROOT, "examples")
+
+
+def build_examples() -> None:
+    """C/CUDA programs that use only include/ and libggprng.so (no Python)."""
+    if not os.path.isdir(EXAMPLES):
+        return
+    for f in sorted(os.listdir(EXAMPLES)):
+        if not f.endswith(".cu"):
+            continue
+        exe = os.path.join(EXAMPLES, f[:-3])
+        cmd = [NVCC] + ARCH + ["-O2", "-std=c++17", "-I", INCLUDE, os.path.join(EXAMPLES, f),
+                               "-o", exe, "-L", PKG, "-lggprng", "-Xlinker",
+                               "-rpath,$ORIGIN/../" + os.path.basename(PKG)]
+        subprocess.check_call(cmd)
 
 
 if __name__ == "__main__":
