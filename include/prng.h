@@ -70,7 +70,9 @@ enum {
 /* Graph parameters (§III-A/B).  Paper defaults in comments. */
 typedef struct {
     uint64_t m;          /* modulus: 2^32 (n = 2^65 vertices, §III-B).  Allowed:
-                            any power of two 2..2^32, or any m in [2, 2^30] */
+                            any m in [2, 2^32]; powers of two take the fast
+                            wrapped-arithmetic kernels, other m the generic one
+                            (conditional-subtract reduction, 64-bit above 2^30) */
     uint32_t degree;     /* must be 7 (Gabber–Galil), else PRNG_E_UNSUPPORTED */
     uint32_t walk_len;   /* l = 64 steps per number (Alg.2, R6); 1..4096 */
     uint32_t burnin_len; /* l0 = 64 steps of Alg.1 ("initial walk of length 64"); 0..4096 */

@@ -171,8 +171,11 @@ __device__ __forceinline__ void gg_walk64x2(const uint32_t a[6], const uint32_t 
     gg_word10x2<4>(a[5] >> 20, b[5] >> 20, xa, ya, xb, yb);
 }
 
-/* One step, any m (generic path).  Non power-of-two m requires m <= 2^30 and
- * x, y < m: every pre-reduction value is < 4m and fits in 32 bits.
+/* One step, any m (generic path), x, y < m.  m = 2^k: wrapped 32-bit
+ * arithmetic.  Other m <= 2^30: every pre-reduction value is < 4m < 2^32, so
+ * two conditional subtracts reduce it.  Other m < 2^32 ("wide"): the same in
+ * 64 bits (2x + y + c <= 3m - 1 needs 34 bits).  A multiply-shift (Barrett)
+ * reduction is not needed: the quotient is at most 3.
  * inv: apply sigma_k^{-1} (variant 1, odd steps): y - 2x - c / x - 2y - c. */
 __device__ __forceinline__ uint32_t gg_reduce(uint32_t t, uint32_t m, bool pow2)
 {
@@ -183,17 +186,32 @@ __device__ __forceinline__ uint32_t gg_reduce(uint32_t t, uint32_t m, bool pow2)
     return t;
 }
 
+__device__ __forceinline__ uint32_t gg_reduce64(uint64_t t, uint32_t m)  /* t < 4m */
+{
+    const uint64_t mm = m;
+    t = (t >= 2u * mm) ? t - 2u * mm : t;
+    t = (t >= mm) ? t - mm : t;
+    return (uint32_t)t;
+}
+
 __device__ __forceinline__ void gg_step_generic(uint32_t b, uint32_t &x, uint32_t &y,
                                                 uint32_t m, bool pow2, bool inv = false)
 {
     const uint32_t cy = b - 1u, cx = b - 4u;
+    const bool wide = !pow2 && m > (1u << 30);
     if (cy < 3u) {
-        if (!inv)
+        if (wide)
+            y = inv ? gg_reduce64((uint64_t)y + 3ull * m - 2ull * x - cy, m)
+                    : gg_reduce64((uint64_t)y + 2ull * x + cy, m);
+        else if (!inv)
             y = gg_reduce(y + 2u * x + cy, m, pow2);
         else
             y = pow2 ? y - 2u * x - cy : gg_reduce(y + 3u * m - 2u * x - cy, m, false);
     } else if (cx < 3u) {
-        if (!inv)
+        if (wide)
+            x = inv ? gg_reduce64((uint64_t)x + 3ull * m - 2ull * y - cx, m)
+                    : gg_reduce64((uint64_t)x + 2ull * y + cx, m);
+        else if (!inv)
             x = gg_reduce(x + 2u * y + cx, m, pow2);
         else
             x = pow2 ? x - 2u * y - cx : gg_reduce(x + 3u * m - 2u * y - cx, m, false);

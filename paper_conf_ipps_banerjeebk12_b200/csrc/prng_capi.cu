@@ -475,7 +475,6 @@ int prng_create(prng_t **out, const prng_graph_params *g, uint64_t walkers, uint
     if (g->degree != 7 || g->variant > 1) return PRNG_E_UNSUPPORTED;
     if (g->m < 2 || g->m > (1ull << 32)) return PRNG_E_INVALID;
     const bool pow2 = (g->m & (g->m - 1)) == 0;
-    if (!pow2 && g->m > (1ull << 30)) return PRNG_E_UNSUPPORTED;
     if (g->walk_len < 1 || g->walk_len > 4096 || g->burnin_len > 4096) return PRNG_E_INVALID;
     if (walkers + o.walker_base > (1ull << 24)) return PRNG_E_INVALID;
     if (o.bit_source != PRNG_BITS_SPLITMIX && o.bit_source != PRNG_BITS_RANDR &&

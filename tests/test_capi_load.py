@@ -63,8 +63,10 @@ def test_host_only_calls(lib):
     p.degree = 5
     assert lib.prng_create(ctypes.byref(h), ctypes.byref(p), 16, 0, None) == lib.PRNG_E_UNSUPPORTED
     p.degree = 7
-    p.m = 3 << 30  # not a power of two and > 2^30
-    assert lib.prng_create(ctypes.byref(h), ctypes.byref(p), 16, 0, None) == lib.PRNG_E_UNSUPPORTED
+    p.m = (1 << 32) + 1  # beyond the 64-bit label space (m^2 <= 2^64)
+    assert lib.prng_create(ctypes.byref(h), ctypes.byref(p), 16, 0, None) == lib.PRNG_E_INVALID
+    p.m = 1
+    assert lib.prng_create(ctypes.byref(h), ctypes.byref(p), 16, 0, None) == lib.PRNG_E_INVALID
     p.m = 1 << 32
     assert lib.prng_create(ctypes.byref(h), ctypes.byref(p), 0, 0, None) == lib.PRNG_E_INVALID
     assert lib.prng_create(ctypes.byref(h), ctypes.byref(p), (1 << 24) + 1, 0, None) == lib.PRNG_E_INVALID

@@ -105,7 +105,10 @@ def test_u32_words_of_full_size_labels(torch_cuda):
 
 @pytest.mark.parametrize("m,l,l0", [(1000, 64, 64), (7, 64, 64), (1 << 16, 64, 64),
                                     ((1 << 30) - 35, 64, 64), (M32, 1, 64), (M32, 16, 8),
-                                    (256, 11, 0), (M32, 100, 64), (2, 64, 64)])
+                                    (256, 11, 0), (M32, 100, 64), (2, 64, 64),
+                                    # m above 2^30, not a power of two: 64-bit reduction
+                                    ((1 << 32) - 5, 64, 64), ((1 << 31) + 11, 11, 7),
+                                    ((3 << 30) + 1, 64, 64), ((1 << 30) + 3, 1, 64)])
 def test_generic_m_and_l_parity(torch_cuda, m, l, l0):
     # General modulus (mod-m reduction each step) and walk lengths other
     # than 64 take the generic kernel; still bit-exact.
@@ -224,7 +227,8 @@ def test_invalid_calls_have_no_side_effects(torch_cuda):
 
 
 # ------------------------------------------------------------ f1 walk variants
-@pytest.mark.parametrize("m,l", [(M32, 64), (256, 64), (1000, 64), (M32, 1), (1000, 1), (M32, 11)])
+@pytest.mark.parametrize("m,l", [(M32, 64), (256, 64), (1000, 64), (M32, 1), (1000, 1), (M32, 11),
+                                 ((1 << 32) - 5, 64), ((3 << 30) + 1, 3)])
 def test_bipartite_variant_parity(torch_cuda, m, l):
     torch = torch_cuda
     W, seed = 320, 13
@@ -257,6 +261,22 @@ def test_l1_fast_kernel_parity_ragged(torch_cuda, m):
         o32 = torch.empty(total, dtype=torch.int32, device="cuda")
         h.fill(o32)
         assert np.array_equal(o32.cpu().numpy().view(np.uint32).astype(np.uint64), want)
+
+
+def test_wide_modulus_on_demand_and_u32(torch_cuda):
+    """m = 2^32 - 5 through prng_next (on demand) and the u32 word format."""
+    torch = torch_cuda
+    m, W, D, seed = (1 << 32) - 5, 200, 3, 91
+    g = G(walkers=W, seed=seed, m=m)
+    o32 = torch.empty(2 * W, dtype=torch.int32, device="cuda")
+    g.fill(o32)  # draw 0 of every walker, 2 words per label (R12)
+    g.epoch_begin(W, D)
+    o = torch.empty(W * D, dtype=torch.int64, device="cuda")
+    g.consume(W, uniform=D, out=o)
+    g.epoch_end()
+    want = O.bulk(m, 64, 64, seed, W, 0, W * (D + 1)).reshape(D + 1, W)
+    assert np.array_equal(o32.cpu().numpy().view(np.uint64), want[0])
+    assert np.array_equal(o.view(W, D).cpu().numpy().view(np.uint64), want[1:].T)
 
 
 def test_bipartite_on_demand(torch_cuda):
