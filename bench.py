@@ -595,7 +595,7 @@ def run_reference(args, world):
     cores = os.cpu_count() or 1
     import multiprocessing as mp
     ctx = mp.get_context("spawn")
-    walkers, draws = 512, 64
+    walkers, draws = 4096, 64  # ~0.3-0.6 s of oracle work per step (pool overhead < 1%)
     with ctx.Pool(cores) as pool:
         pool.map(_oracle_worker, [(0, 1, 1)] * cores)
         for _ in range(args.warmup):
