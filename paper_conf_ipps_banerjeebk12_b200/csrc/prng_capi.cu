@@ -120,10 +120,11 @@ struct prng_s {
     bool have_mark = false, od_started_mark = false;
 
     // pinned staging chunks
-    static const int kChunks = 4;
-    uint32_t *chunk[kChunks] = {};
+    static const int kMaxChunks = 8;
+    int kChunks = 4;
+    uint32_t *chunk[kMaxChunks] = {};
     size_t chunk_bytes = 0;
-    cudaEvent_t chunk_done[kChunks] = {};
+    cudaEvent_t chunk_done[kMaxChunks] = {};
     int chunk_next = 0;
 
     // resident (prefetched) window: draws [res_J, res_J + res_D) of all walkers
@@ -171,7 +172,7 @@ void free_all(prng_s *h) {
         if (p) cudaFree(p);
     for (auto p : h->hout)
         if (p) cudaFree(p);
-    for (int i = 0; i < prng_s::kChunks; i++) {
+    for (int i = 0; i < h->kChunks; i++) {
         if (h->chunk[i]) cudaFreeHost(h->chunk[i]);
         if (h->chunk_done[i]) cudaEventDestroy(h->chunk_done[i]);
     }
@@ -235,6 +236,8 @@ void feed_chunk(prng_s *h, uint64_t wa, uint64_t wb, uint64_t k0, uint32_t nrows
 void stage_rows(prng_s *h, uint64_t k0, uint64_t nrows, uint64_t Wv, uint32_t *dst,
                 uint64_t dpitch, const uint32_t *ids = nullptr, bool bursty = false) {
     if (nrows == 0 || Wv == 0) return;
+    static const bool nt_all = getenv("GG_FEED_NT_ALL") != nullptr;  // A/B hook
+    bursty = bursty || nt_all;
     const uint64_t chunk_words = h->chunk_bytes / 4;
     // Chunks hold an even number of rows (>= 2) so each 64-bit SplitMix word
     // feeds two rows (k even, k+1) with one hash.  Full-width chunks are
@@ -277,7 +280,7 @@ void stage_rows(prng_s *h, uint64_t k0, uint64_t nrows, uint64_t Wv, uint32_t *d
             uint64_t nr = std::min<uint64_t>(rows_per, nrows - r);
             if (((k0 + r) & 1) && nr > 1) nr -= 1;  // keep later chunks pair-aligned
             const int b = h->chunk_next;
-            h->chunk_next = (b + 1) % prng_s::kChunks;
+            h->chunk_next = (b + 1) % h->kChunks;
             CK(cudaEventSynchronize(h->chunk_done[b]));  // pinned chunk free again
             feed_chunk(h, 0, Wv, k0 + r, (uint32_t)nr, h->chunk[b], ids, dpitch, bursty);
             CK(cudaMemcpyAsync(dst + r * dpitch, h->chunk[b], nr * dpitch * 4,
@@ -295,7 +298,7 @@ void stage_rows(prng_s *h, uint64_t k0, uint64_t nrows, uint64_t Wv, uint32_t *d
         for (uint64_t wa = 0; wa < Wv; wa += walkers_per) {
             const uint64_t wb = std::min<uint64_t>(Wv, wa + walkers_per);
             const int b = h->chunk_next;
-            h->chunk_next = (b + 1) % prng_s::kChunks;
+            h->chunk_next = (b + 1) % h->kChunks;
             CK(cudaEventSynchronize(h->chunk_done[b]));
             const uint64_t cw = wb - wa;
             // rows start 32-B aligned in the chunk, so the streaming-store path
@@ -508,8 +511,11 @@ int prng_create(prng_t **out, const prng_graph_params *g, uint64_t walkers, uint
         CK(cudaStreamCreateWithFlags(&h->d2h_stream, cudaStreamNonBlocking));
         CK(cudaStreamCreateWithFlags(&h->work_stream, cudaStreamNonBlocking));
         CK(cudaEventCreateWithFlags(&h->ev_tmp, cudaEventDisableTiming));
-        h->chunk_bytes = 32ull << 20;
-        for (int i = 0; i < prng_s::kChunks; i++) {
+        static const int chunk_mb = getenv("GG_FEED_CHUNK_MB") ? atoi(getenv("GG_FEED_CHUNK_MB")) : 16;
+        static const int nchunks = getenv("GG_FEED_CHUNKS") ? atoi(getenv("GG_FEED_CHUNKS")) : 4;
+        h->chunk_bytes = (size_t)(chunk_mb > 0 ? chunk_mb : 32) << 20;
+        h->kChunks = std::min(prng_s::kMaxChunks, std::max(2, nchunks));
+        for (int i = 0; i < h->kChunks; i++) {
             CK(cudaHostAlloc((void **)&h->chunk[i], h->chunk_bytes, cudaHostAllocPortable));
             CK(cudaEventCreateWithFlags(&h->chunk_done[i], cudaEventDisableTiming));
         }
