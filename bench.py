@@ -96,50 +96,107 @@ def cpu_baseline_block(target_seconds: float = 8.0):
 
 # ------------------------------------------------------------------ clocks
 class ClockSampler:
-    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
-              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
-              "clocks_event_reasons.sw_power_cap")
+    """SM clock, power and throttle reasons sampled every ~5 ms by NVML in a
+    thread (nvidia-smi -lms 20 as the fallback).  start() before the warm-up,
+    mark(True/False) around the timed region: summary() keeps the samples
+    taken inside it (the recipe's clocks line), falling back to every sample
+    under load if the region is shorter than the sampling period."""
+    REASONS = (("hw_slowdown", 0x8), ("hw_thermal_slowdown", 0x40), ("sw_thermal_slowdown", 0x20),
+               ("sw_power_cap", 0x4), ("hw_power_brake_slowdown", 0x80))
 
-    def __init__(self, gpu_id: str):
-        self.gpu_id, self.rows, self.proc = gpu_id, [], None
+    def __init__(self, gpu_id: str, index: int = 0):
+        self.gpu_id, self.index = gpu_id, index
+        self.rows = []  # (t, sm_mhz, max_mhz, power_w, reasons bitmask)
+        self.t0 = self.t1 = None
+        self.stop = threading.Event()
+        self.th = None
+        self.backend = None
 
     def __enter__(self):
         try:
-            self.proc = subprocess.Popen(
-                ["nvidia-smi", "-i", self.gpu_id, f"--query-gpu={self.FIELDS}",
-                 "--format=csv,noheader,nounits", "-lms", "20"],
-                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
-            self.th = threading.Thread(target=self._read, daemon=True)
+            import pynvml
+            pynvml.nvmlInit()
+            try:
+                h = pynvml.nvmlDeviceGetHandleByUUID(self.gpu_id)
+            except Exception:
+                h = pynvml.nvmlDeviceGetHandleByIndex(self.index)
+            self.backend = "nvml"
+
+            def run():
+                mx = pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM)
+                while not self.stop.is_set():
+                    try:
+                        sm = pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM)
+                        pw = pynvml.nvmlDeviceGetPowerUsage(h) / 1000.0
+                        rs = pynvml.nvmlDeviceGetCurrentClocksEventReasons(h)
+                        self.rows.append((time.perf_counter(), float(sm), float(mx), pw, int(rs)))
+                    except Exception:
+                        pass
+                    time.sleep(0.005)
+            self.th = threading.Thread(target=run, daemon=True)
             self.th.start()
-        except OSError:
-            self.proc = None
+        except Exception:
+            self._smi()
         return self
 
-    def _read(self):
-        for line in self.proc.stdout:
-            parts = [p.strip() for p in line.split(",")]
-            if len(parts) == 7:
-                self.rows.append(parts)
+    def _smi(self):
+        fields = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+                  "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+                  "clocks_event_reasons.sw_power_cap")
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", self.gpu_id, f"--query-gpu={fields}",
+                 "--format=csv,noheader,nounits", "-lms", "20"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except OSError:
+            return
+        self.backend = "nvidia-smi"
+        bits = (0x8, 0x40, 0x20, 0x4)
+
+        def run():
+            for line in self.proc.stdout:
+                p = [x.strip() for x in line.split(",")]
+                if len(p) == 7:
+                    try:
+                        rs = sum(b for b, v in zip(bits, p[3:]) if v == "Active")
+                        self.rows.append((time.perf_counter(), float(p[0]), float(p[1]),
+                                          float(p[2]), rs))
+                    except ValueError:
+                        pass
+        self.th = threading.Thread(target=run, daemon=True)
+        self.th.start()
+
+    def mark(self, start: bool):
+        if start:
+            self.t0 = time.perf_counter()
+        else:
+            self.t1 = time.perf_counter()
 
     def __exit__(self, *exc):
-        if self.proc:
+        self.stop.set()
+        if self.backend == "nvidia-smi":
             self.proc.terminate()
             try:
                 self.proc.wait(timeout=5)
             except subprocess.TimeoutExpired:
                 self.proc.kill()
+        elif self.th:
+            self.th.join(timeout=1)
 
     def summary(self):
-        if not self.rows:
+        rows = list(self.rows)
+        inside = [r for r in rows if self.t0 is not None and self.t1 is not None
+                  and self.t0 <= r[0] <= self.t1]
+        use = inside if len(inside) >= 3 else rows
+        if not use:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"], "samples": 0}
-        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
-        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        reasons = sorted({names[i] for r in self.rows for i in range(4) if r[3 + i] == "Active"})
-        pw = [float(r[2]) for r in self.rows if r[2].replace(".", "").isdigit()]
-        return {"sm_mhz": statistics.median(sm) if sm else None,
-                "sm_max_mhz": max(mx) if mx else None, "reasons": reasons,
-                "power_w_max": max(pw) if pw else None, "samples": len(self.rows)}
+        reasons = sorted({n for r in use for n, b in self.REASONS if r[4] & b})
+        return {"sm_mhz": statistics.median(r[1] for r in use),
+                "sm_max_mhz": max(r[2] for r in use), "reasons": reasons,
+                "power_w_max": max(r[3] for r in use), "samples": len(use),
+                "samples_in_timed_region": len(inside),
+                "window": "timed region" if use is inside else "whole K-mode section (region < 3 samples)",
+                "source": self.backend}
 
 
 def committed_traffic():
@@ -194,6 +251,9 @@ def run_ours(args, rank, world, local_rank):
     g.prefetch(DRAWS_PER_STEP)
     g.mark()
     out = torch.empty(U32_PER_STEP, dtype=torch.int32, device=dev)
+    gpu_id = getattr(props, "uuid", None)
+    gpu_id = f"GPU-{gpu_id}" if gpu_id is not None else str(local_rank)
+    clk = ClockSampler(gpu_id, local_rank).__enter__()  # running before the warm-up
     for _ in range(args.warmup):
         g.rewind()
         g.fill(out)
@@ -201,20 +261,20 @@ def run_ours(args, rank, world, local_rank):
     ev0 = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
     ev1 = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
     start, end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    gpu_id = getattr(props, "uuid", None)
-    gpu_id = f"GPU-{gpu_id}" if gpu_id is not None else str(local_rank)
     launches0 = g.stats()["kernel_launches"]
     barrier()
     torch.cuda.synchronize()
-    with ClockSampler(gpu_id) as clk:
-        start.record(stream)
-        for i in range(args.steps):
-            g.rewind()
-            ev0[i].record(stream)
-            g.fill(out)
-            ev1[i].record(stream)
-        end.record(stream)
-        torch.cuda.synchronize()
+    clk.mark(True)
+    start.record(stream)
+    for i in range(args.steps):
+        g.rewind()
+        ev0[i].record(stream)
+        g.fill(out)
+        ev1[i].record(stream)
+    end.record(stream)
+    torch.cuda.synchronize()
+    clk.mark(False)
+    clk.__exit__(None, None, None)
     barrier()
     launches = g.stats()["kernel_launches"] - launches0
     ms = max_over_ranks(start.elapsed_time(end))
