@@ -1,0 +1,83 @@
+"""Every diagnostic / A-B kernel and feed variant (DESIGN.md §8 hooks) is
+bit-exact with the oracle: the hooks are read once per process, so each
+runs in a subprocess on small C2-type inputs (ragged walker count, fills that
+stop mid-draw, an on-demand epoch with a walker list, a tiny MC run)."""
+import json
+import os
+import subprocess
+import sys
+
+import numpy as np
+import pytest
+
+import oracle as O
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+M32 = 1 << 32
+
+SNIPPET = r"""
+import json, sys
+import numpy as np, torch
+sys.path.insert(0, %(root)r)
+from paper_conf_ipps_banerjeebk12_b200 import Generator
+W, seed = 1000, 0x5EED00F0
+g = Generator(walkers=W, seed=seed, epoch_draws=3)
+outs = []
+for n in (7, 3 * W + 5, 2 * W):
+    o = torch.empty(n, dtype=torch.int64, device="cuda")
+    g.fill(o)
+    outs.append(o.cpu().numpy().view(np.uint64))
+bulk = np.concatenate(outs)
+ids = np.arange(0, W, 7, dtype=np.uint32)
+g.epoch_begin_list(ids, 2)
+od = torch.empty(ids.size * 2, dtype=torch.int64, device="cuda")
+g.consume(ids.size, uniform=2, out=od)
+g.epoch_end()
+layers = [(1.37, 1.0, 100.0, 0.9, 0.1), (1.37, 1.0, 10.0, 0.0, 0.1), (1.37, 2.0, 10.0, 0.7, 0.2)]
+g2 = Generator(walkers=512, seed=0x5EED0004)
+mc = g2.mc_run(layers, 2000, threads=512, epoch_draws=48)
+print(json.dumps({"bulk": [int(v) for v in bulk], "od": [int(v) for v in od.cpu().numpy().view(np.uint64)],
+                  "tallies": [int(v) for v in mc["tallies"]]}))
+"""
+
+VARIANTS = ["GG_FILL_NO_TMA=1", "GG_FILL_X1=1", "GG_FILL_MINB=1", "GG_FILL_MINB=28",
+            "GG_FILL_BPS=3", "GG_FILL_KPW=2", "GG_FEED_NT_ALL=1", "GG_FEED_NO_NT=1",
+            "GG_FEED_CHUNK_MB=1", "GG_FEED_CHUNKS=2", "GG_MC_MINB=4"]
+
+
+@pytest.fixture(scope="module")
+def want():
+    W, seed = 1000, 0x5EED00F0
+    n = 7 + 3 * W + 5 + 2 * W
+    bulk = O.bulk(M32, 64, 64, seed, W, 0, n)
+    J0 = -(-n // W)  # first epoch starts at the next whole draw (R10)
+    ids = np.arange(0, W, 7)
+    lib = O.lib()
+    od = []
+    for t in ids:  # R10: walk the bulk draws, skip the rest of draw J0-1, then J0, J0+1
+        x, y = O.walker_init(M32, 64, seed, int(t))
+        xa, ya = np.array([x], np.uint64), np.array([y], np.uint64)
+        for j in range((n - int(t) + W - 1) // W):
+            lib.or_walker_draw(M32, 64, 64, seed, int(t), j, xa.ctypes.data, ya.ctypes.data)
+        od.append([int(lib.or_walker_draw(M32, 64, 64, seed, int(t), J0 + i, xa.ctypes.data,
+                                          ya.ctypes.data)) for i in range(2)])
+    od = np.array(od, dtype=np.uint64)
+    mc = O.mc_run(nthreads=512, photons_total=2000, D=48, seed=0x5EED0004)
+    return bulk, od, mc["tallies"]
+
+
+@pytest.mark.parametrize("var", VARIANTS)
+def test_variant_bit_exact(var, want):
+    env = dict(os.environ)
+    k, v = var.split("=")
+    env[k] = v
+    out = subprocess.run([sys.executable, "-c", SNIPPET % {"root": ROOT}], env=env,
+                         capture_output=True, text=True, timeout=300)
+    assert out.returncode == 0, out.stderr[-2000:]
+    got = json.loads(out.stdout.strip().splitlines()[-1])
+    bulk, od, tallies = want
+    assert np.array_equal(np.array(got["bulk"], dtype=np.uint64), bulk), var
+    # consume(): slot k's draws at [2k, 2k+1] (offsets = k * uniform)
+    assert np.array_equal(np.array(got["od"], dtype=np.uint64).reshape(-1, 2), od), var
+    assert got["tallies"] == [int(t) for t in tallies], var
