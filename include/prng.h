@@ -123,7 +123,9 @@ int prng_create(prng_t **out, const prng_graph_params *g, uint64_t walkers,
  * sequence Z[N .. N+n) (R11: Z[g] = label of walker g mod W, draw g div W;
  * N advances by the labels written) to dev_ptr, in format fmt.
  *   dev_ptr : caller-owned device memory, >= n * (fmt==U64 ? 8 : 4) bytes,
- *             aligned to 8 (U64) / 4 (U32) bytes.
+ *             aligned to 8 bytes (labels are stored whole), or to 4 bytes
+ *             for U32 with m <= 2^16 (one word per label); else
+ *             PRNG_E_INVALID.
  *   n       : count in units of fmt.  For U32 with m > 2^16, n must be even.
  *   stream  : the kernels (and any copies of bits not already resident) are
  *             ordered on this stream; the call returns after enqueueing, but

@@ -581,7 +581,9 @@ int prng_fill(prng_t *h, void *dev_ptr, uint64_t n, int fmt, void *stream) {
     int rc = check_fmt(h, n, fmt);
     if (rc != PRNG_OK) return rc;
     if (n == 0) return PRNG_OK;
-    if (!dev_ptr || ((uintptr_t)dev_ptr % (fmt == PRNG_FMT_U64 ? 8 : 4))) return PRNG_E_INVALID;
+    // labels are stored whole: 8-byte alignment unless one u32 word per label
+    const uintptr_t align = (fmt == PRNG_FMT_U32 && h->g.m <= 65536ull) ? 4 : 8;
+    if (!dev_ptr || ((uintptr_t)dev_ptr % align)) return PRNG_E_INVALID;
     if (h->od_open) return PRNG_E_STATE;
     return guard(h, [&] {
         cudaStream_t s = (cudaStream_t)stream;

@@ -98,6 +98,23 @@ def test_u32_words_ragged_and_small_m():
     assert np.array_equal(o.cpu().numpy().view(np.uint32).astype(np.uint64), want)
 
 
+def test_misaligned_output_is_refused_without_side_effects():
+    """Labels are stored whole: a u32 buffer for m = 2^32 must be 8-B aligned."""
+    import torch
+    from paper_conf_ipps_banerjeebk12_b200 import PrngError
+    g = G(walkers=64, seed=5)
+    buf = torch.empty(2 * 64 + 1, dtype=torch.int32, device="cuda")
+    with pytest.raises(PrngError):
+        g.fill(buf[1:], n=2 * 64)
+    assert g.tell() == 0
+    g.fill(buf[:-1])  # still usable, sequence unchanged
+    assert np.array_equal(buf[:-1].cpu().numpy().view(np.uint64), O.bulk(M32, 64, 64, 5, 64, 0, 64))
+    g2 = G(walkers=64, seed=5, m=1 << 16)  # one word per label: 4-B alignment is enough
+    g2.fill(buf[1:], n=64)
+    want = O.bulk(1 << 16, 64, 64, 5, 64, 0, 64)
+    assert np.array_equal(buf[1:65].cpu().numpy().view(np.uint32).astype(np.uint64), want)
+
+
 def test_smallest_modulus():
     """m = 2: a 4-vertex graph; still the oracle's sequence."""
     import torch
