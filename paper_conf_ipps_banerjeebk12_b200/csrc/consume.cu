@@ -56,6 +56,8 @@ extern "C" int gg_consume(prng_t *h, uint64_t threads, const uint32_t *counts, u
     if (rc != PRNG_OK) return rc;
     if (threads == 0) return PRNG_OK;
     if (threads > v.Wv) return PRNG_E_INVALID;
+    auto mis = [](const void *p, uintptr_t a) { return p && ((uintptr_t)p % a) != 0; };
+    if (mis(counts, 4) || mis(out, 8) || mis(offsets, 8) || mis(xor_out, 8)) return PRNG_E_INVALID;
     const uint32_t tpb = 128;
     const uint64_t blocks = (threads + tpb - 1) / tpb;
     consume_kernel<<<(unsigned)blocks, tpb, 0, (cudaStream_t)stream>>>(v, threads, counts, uniform,

@@ -249,6 +249,9 @@ extern "C" int gg_list_rank(prng_t *h, int64_t n, const int32_t *succ, const int
         (world > 1 && (!coll->allgather || !coll->allreduce_i32)))
         return PRNG_E_INVALID;
     if (n > (1ll << 24)) return PRNG_E_UNSUPPORTED;
+    for (const void *p : {(const void *)succ, (const void *)pred, (const void *)rank,
+                          (const void *)removed_round, (const void *)is_splitter})
+        if (((uintptr_t)p % 4) != 0) return PRNG_E_INVALID;
     cudaStream_t s = (cudaStream_t)stream;
     std::vector<void *> bufs;
     cudaMemPool_t pool = gg::scratch_pool();

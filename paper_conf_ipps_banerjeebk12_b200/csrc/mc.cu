@@ -296,6 +296,7 @@ extern "C" int gg_mc_run(prng_t *h, const gg_mc_config *cfg, int64_t *tallies, i
         cfg->threads_total == 0 || cfg->epoch_draws < 3 || cfg->epoch_draws % 3 != 0 ||
         cfg->thread0 + cfg->threads > cfg->threads_total)
         return PRNG_E_INVALID;
+    if (per_thread && ((uintptr_t)per_thread % 8) != 0) return PRNG_E_INVALID;
     cudaStream_t s = (cudaStream_t)stream;
     McParams P{};
     P.nl = cfg->nlayers;
