@@ -599,6 +599,7 @@ int prng_fill(prng_t *h, void *dev_ptr, uint64_t n, int fmt, void *stream) {
                        h->stats.kernel_launches++;
                    });
         h->N = N + nl;
+        h->od_started = false;  // the next epoch starts at the next whole draw after N (R10)
         h->stats.labels_generated += nl;
         return PRNG_OK;
     });
@@ -657,6 +658,7 @@ int prng_fill_host(prng_t *h, void *host_ptr, uint64_t n, int fmt) {
         CK(cudaStreamSynchronize(h->d2h_stream));
         CK(cudaStreamSynchronize(s));
         h->N = N + nl;
+        h->od_started = false;  // the next epoch starts at the next whole draw after N (R10)
         h->stats.labels_generated += nl;
         return PRNG_OK;
     });

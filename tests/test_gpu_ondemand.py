@@ -172,3 +172,37 @@ def test_epoch_reserve_same_numbers_and_errors():
             g.epoch_end()
         g.close()
     assert np.array_equal(res[0], res[1])
+
+
+def test_on_demand_bulk_on_demand_keeps_one_sequence():
+    """epoch -> ragged bulk fill -> epoch: the second epoch starts at the next
+    whole draw after the fill (R10/R11); no draw is emitted twice."""
+    import torch
+    from paper_conf_ipps_banerjeebk12_b200 import Generator
+    W, seed = 300, 23
+    g = Generator(walkers=W, seed=seed)
+    g.epoch_begin(W, 2)
+    a = torch.empty(W * 2, dtype=torch.int64, device="cuda")
+    g.consume(W, uniform=2, out=a)
+    g.epoch_end()
+    n = 3 * W + 5
+    b = torch.empty(n, dtype=torch.int64, device="cuda")
+    g.fill(b)
+    g.epoch_begin(W, 1)
+    c = torch.empty(W, dtype=torch.int64, device="cuda")
+    g.consume(W, uniform=1, out=c)
+    g.epoch_end()
+    a = a.view(W, 2).cpu().numpy().view(np.uint64)
+    b = b.cpu().numpy().view(np.uint64)
+    c = c.cpu().numpy().view(np.uint64)
+    N = 2 * W + n          # bulk positions consumed so far
+    J1 = -(-N // W)        # second epoch's first draw
+    for t in (0, 4, 5, 150, W - 1):
+        ow = OracleWalker(M32, seed, t)
+        assert [ow.draw(0), ow.draw(1)] == [int(v) for v in a[t]]
+        for j in range(2, 6):
+            g_idx = j * W + t - 2 * W
+            if g_idx < n:
+                assert int(b[g_idx]) == ow.draw(j), (t, j)
+        assert int(c[t]) == ow.draw(J1), t
+    assert g.check() == 0
