@@ -171,6 +171,136 @@ __device__ __forceinline__ void gg_walk64x2(const uint32_t a[6], const uint32_t 
     gg_word10x2<4>(a[5] >> 20, b[5] >> 20, xa, ya, xb, yb);
 }
 
+/* ------------------------------------------------------------------------
+ * R2P form of the same step (default for l = 64, m = 2^k).  The per-step
+ * predicate tests (two LOP3.P per step above) are replaced by loading the
+ * predicate register file from one byte of a flag word: ptxas turns four
+ * single-bit tests of the same register that fall inside one byte into one
+ * R2P PR, F.Bn (measured, tools/step_bench2.cu).  Per 10-field word:
+ *   F = MY at field bit 0 (y-move) | MX at field bit 1 (x-move),  G = F >> 6
+ * and the 10 steps are grouped so that each group's flags sit in bits 0..6 of
+ * one byte of F or G:
+ *   F.B0 steps 0,1 | G.B0 step 2 | F.B1 steps 3,4 | G.B1 step 5 |
+ *   F.B2 steps 6,7 | F.B3 steps 8,9        (4-field tail word: F.B0 0,1 | G.B0 2,3)
+ * i.e. 6 R2P + 1 shift per 10 steps instead of 20 LOP3.P.  The arithmetic is
+ * unchanged (u = x + y + c; y' = u + x | x' = u + y), so both forms are the
+ * same evaluation of the paper's step.
+ * ------------------------------------------------------------------------ */
+#define GG_R2P_U(S)                                                                   \
+    "shl.b32 ct, %3, " S ";\n\tshr.b32 c, ct, 30;\n\tadd.u32 s, %0, %1;\n\tadd.u32 u, s, c;\n\t"
+
+/* Two steps: py/px of the first at bits B0/B0+1 of S, of the second at B1/B1+1;
+ * SH0/SH1 = 30 - 3k bring field k's constant to the top of C. */
+template <int B0, int B1, int SH0, int SH1>
+__device__ __forceinline__ void gg_r2p_two(uint32_t S, uint32_t C, uint32_t &x, uint32_t &y)
+{
+    asm volatile(
+        "{\n\t.reg .pred py0, px0, py1, px1;\n\t.reg .b32 t, ct, c, u, s;\n\t"
+        "and.b32 t, %2, %4;\n\tsetp.ne.b32 py0, t, 0;\n\t"
+        "and.b32 t, %2, %5;\n\tsetp.ne.b32 px0, t, 0;\n\t"
+        "and.b32 t, %2, %6;\n\tsetp.ne.b32 py1, t, 0;\n\t"
+        "and.b32 t, %2, %7;\n\tsetp.ne.b32 px1, t, 0;\n\t"
+        GG_R2P_U("%8") "@py0 add.u32 %1, u, %0;\n\t@px0 add.u32 %0, u, %1;\n\t"
+        GG_R2P_U("%9") "@py1 add.u32 %1, u, %0;\n\t@px1 add.u32 %0, u, %1;\n\t}"
+        : "+r"(x), "+r"(y)
+        : "r"(S), "r"(C), "n"(1u << B0), "n"(2u << B0), "n"(1u << B1), "n"(2u << B1), "n"(SH0),
+          "n"(SH1));
+}
+
+template <int B0, int SH0>
+__device__ __forceinline__ void gg_r2p_one(uint32_t S, uint32_t C, uint32_t &x, uint32_t &y)
+{
+    asm volatile(
+        "{\n\t.reg .pred py0, px0;\n\t.reg .b32 t, ct, c, u, s;\n\t"
+        "and.b32 t, %2, %4;\n\tsetp.ne.b32 py0, t, 0;\n\t"
+        "and.b32 t, %2, %5;\n\tsetp.ne.b32 px0, t, 0;\n\t"
+        GG_R2P_U("%6") "@py0 add.u32 %1, u, %0;\n\t@px0 add.u32 %0, u, %1;\n\t}"
+        : "+r"(x), "+r"(y)
+        : "r"(S), "r"(C), "n"(1u << B0), "n"(2u << B0), "n"(SH0));
+}
+
+/* Flag word F and constant word C of a 10-field word Q (fields at 3i). */
+__device__ __forceinline__ void gg_r2p_prep(uint32_t Q, uint32_t &C, uint32_t &F)
+{
+    const uint32_t f1 = Q >> 1, f2 = Q >> 2;
+    const uint32_t MY = ((f1 | Q) & 0x09249249u) & ~f2; /* b in {1,2,3}, at 3i  */
+    const uint32_t MX = f2 & ~(f1 & Q);                  /* b in {4,5,6}, at 3i (+garbage) */
+    C = Q - MY;
+    F = MY | ((MX << 1) & 0x12492492u);                  /* MX moved to 3i+1   */
+}
+
+#define GG_SH(k) (30 - 3 * (k))
+
+template <int NK>
+__device__ __forceinline__ void gg_word10_r2p(uint32_t Q, uint32_t &x, uint32_t &y)
+{
+    uint32_t C, F;
+    gg_r2p_prep(Q, C, F);
+    const uint32_t G = F >> 6;
+    gg_r2p_two<0, 3, GG_SH(0), GG_SH(1)>(F, C, x, y);
+    if (NK == 4) {
+        gg_r2p_two<0, 3, GG_SH(2), GG_SH(3)>(G, C, x, y);
+        return;
+    }
+    gg_r2p_one<0, GG_SH(2)>(G, C, x, y);
+    gg_r2p_two<9, 12, GG_SH(3), GG_SH(4)>(F, C, x, y);
+    gg_r2p_one<9, GG_SH(5)>(G, C, x, y);
+    gg_r2p_two<18, 21, GG_SH(6), GG_SH(7)>(F, C, x, y);
+    gg_r2p_two<24, 27, GG_SH(8), GG_SH(9)>(F, C, x, y);
+}
+
+template <int NK>
+__device__ __forceinline__ void gg_word10x2_r2p(uint32_t Qa, uint32_t Qb, uint32_t &xa, uint32_t &ya,
+                                                uint32_t &xb, uint32_t &yb)
+{
+    uint32_t Ca, Fa, Cb, Fb;
+    gg_r2p_prep(Qa, Ca, Fa);
+    gg_r2p_prep(Qb, Cb, Fb);
+    const uint32_t Ga = Fa >> 6, Gb = Fb >> 6;
+#define GG_R2P2(B0, B1, K0, K1, SA, SB)                                     \
+    gg_r2p_two<B0, B1, GG_SH(K0), GG_SH(K1)>(SA, Ca, xa, ya);                \
+    gg_r2p_two<B0, B1, GG_SH(K0), GG_SH(K1)>(SB, Cb, xb, yb);
+#define GG_R2P1(B0, K0, SA, SB)                                              \
+    gg_r2p_one<B0, GG_SH(K0)>(SA, Ca, xa, ya);                               \
+    gg_r2p_one<B0, GG_SH(K0)>(SB, Cb, xb, yb);
+    GG_R2P2(0, 3, 0, 1, Fa, Fb)
+    if (NK == 4) {
+        GG_R2P2(0, 3, 2, 3, Ga, Gb)
+        return;
+    }
+    GG_R2P1(0, 2, Ga, Gb)
+    GG_R2P2(9, 12, 3, 4, Fa, Fb)
+    GG_R2P1(9, 5, Ga, Gb)
+    GG_R2P2(18, 21, 6, 7, Fa, Fb)
+    GG_R2P2(24, 27, 8, 9, Fa, Fb)
+#undef GG_R2P2
+#undef GG_R2P1
+}
+
+/* 64 steps from a 6-word record (R2P form). */
+__device__ __forceinline__ void gg_walk64_r2p(const uint32_t w[6], uint32_t &x, uint32_t &y)
+{
+    gg_word10_r2p<10>(w[0], x, y);
+    gg_word10_r2p<10>(__funnelshift_r(w[0], w[1], 30), x, y);
+    gg_word10_r2p<10>(__funnelshift_r(w[1], w[2], 28), x, y);
+    gg_word10_r2p<10>(__funnelshift_r(w[2], w[3], 26), x, y);
+    gg_word10_r2p<10>(__funnelshift_r(w[3], w[4], 24), x, y);
+    gg_word10_r2p<10>(__funnelshift_r(w[4], w[5], 22), x, y);
+    gg_word10_r2p<4>(w[5] >> 20, x, y);
+}
+
+__device__ __forceinline__ void gg_walk64x2_r2p(const uint32_t a[6], const uint32_t b[6], uint32_t &xa,
+                                                uint32_t &ya, uint32_t &xb, uint32_t &yb)
+{
+    gg_word10x2_r2p<10>(a[0], b[0], xa, ya, xb, yb);
+    gg_word10x2_r2p<10>(__funnelshift_r(a[0], a[1], 30), __funnelshift_r(b[0], b[1], 30), xa, ya, xb, yb);
+    gg_word10x2_r2p<10>(__funnelshift_r(a[1], a[2], 28), __funnelshift_r(b[1], b[2], 28), xa, ya, xb, yb);
+    gg_word10x2_r2p<10>(__funnelshift_r(a[2], a[3], 26), __funnelshift_r(b[2], b[3], 26), xa, ya, xb, yb);
+    gg_word10x2_r2p<10>(__funnelshift_r(a[3], a[4], 24), __funnelshift_r(b[3], b[4], 24), xa, ya, xb, yb);
+    gg_word10x2_r2p<10>(__funnelshift_r(a[4], a[5], 22), __funnelshift_r(b[4], b[5], 22), xa, ya, xb, yb);
+    gg_word10x2_r2p<4>(a[5] >> 20, b[5] >> 20, xa, ya, xb, yb);
+}
+
 /* One step, any m (generic path), x, y < m.  m = 2^k: wrapped 32-bit
  * arithmetic.  Other m <= 2^30: every pre-reduction value is < 4m < 2^32, so
  * two conditional subtracts reduce it.  Other m < 2^32 ("wide"): the same in

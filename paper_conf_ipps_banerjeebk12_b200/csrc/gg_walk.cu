@@ -252,8 +252,9 @@ __global__ void __launch_bounds__(64, 32) gg_fill64_tma_kernel(const __grid_cons
 
 // Two walkers per lane: a warp owns 64 walkers (u*64 + lane, u*64 + 32 +
 // lane); one TMA box of 64 x 6 words (1.5 KB) per draw; the two walks are
-// interleaved step by step.
-template <int EMIT, int MINB = 1>
+// interleaved step by step.  STEP: 1 = R2P form of the walk step (default),
+// 0 = per-step LOP3.P predicates (A/B hook GG_FILL_STEP=0).
+template <int EMIT, int MINB = 1, int STEP = 1>
 __global__ void __launch_bounds__(64, MINB) gg_fill64x2_tma_kernel(const __grid_constant__ CUtensorMap tmap,
                                                          FillArgs a, uint32_t units64) {
     constexpr int kTile = 6 * 64;
@@ -318,7 +319,10 @@ __global__ void __launch_bounds__(64, MINB) gg_fill64x2_tma_kernel(const __grid_
                 wb[r] = buf[r * 64 + 32 + lane];
             }
             uint32_t nxa = xa, nya = ya, nxb = xb, nyb = yb;
-            gg_walk64x2(wa, wb, nxa, nya, nxb, nyb);
+            if (STEP)
+                gg_walk64x2_r2p(wa, wb, nxa, nya, nxb, nyb);
+            else
+                gg_walk64x2(wa, wb, nxa, nya, nxb, nyb);
             if (j >= ja0 && j < ja1) {
                 xa = nxa;
                 ya = nya;
@@ -568,7 +572,11 @@ cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count) {
                 // register budget (A/B hook GG_FILL_MINB; default 24 = 37 regs, 0.5% faster
                 // than ptxas' choice (1: 46 regs); 28 -> 32 regs is 5% slower; no spills)
                 static const int minb = getenv("GG_FILL_MINB") ? atoi(getenv("GG_FILL_MINB")) : 24;
-                if (minb == 24) {
+                static const bool r2p = !(getenv("GG_FILL_STEP") && atoi(getenv("GG_FILL_STEP")) == 0);
+                if (minb == 24 && !r2p) {
+                    plan_grid(gg_fill64x2_tma_kernel<0, 24, 0>, units64 * 2, sm_count, blocks, threads);
+                    gg_fill64x2_tma_kernel<0, 24, 0><<<blocks, threads, 0, s>>>(map, a, units64);
+                } else if (minb == 24) {
                     plan_grid(gg_fill64x2_tma_kernel<0, 24>, units64 * 2, sm_count, blocks, threads);
                     gg_fill64x2_tma_kernel<0, 24><<<blocks, threads, 0, s>>>(map, a, units64);
                 } else if (minb == 28) {
