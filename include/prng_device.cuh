@@ -426,7 +426,7 @@ __device__ __forceinline__ uint64_t prng_next(prng_state *st, const prng_view *v
 #pragma unroll
         for (int r = 0; r < 6; r++)
             w[r] = __ldg(rec + (uint64_t)r * v->pitch);
-        gg_walk64(w, x, y);
+        gg_walk64_r2p(w, x, y);
     } else {
         const uint64_t s0 = (uint64_t)v->l0 + (uint64_t)v->l * (v->J0 + st->used);
         gg_walk_generic(rec, v->pitch, v->l, x, y, (uint32_t)v->m, v->pow2 != 0, v->variant, s0);
@@ -460,7 +460,7 @@ __device__ __forceinline__ void prng_next_n(prng_state *st, const prng_view *v, 
     uint32_t x = st->x, y = st->y;
 #pragma unroll
     for (int k = 0; k < K; k++) {
-        gg_walk64(w[k], x, y);
+        gg_walk64_r2p(w[k], x, y);
         out[k] = gg_label(x, y, v->m, v->log2m, true);
     }
     st->x = x;

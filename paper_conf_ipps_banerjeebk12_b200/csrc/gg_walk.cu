@@ -36,7 +36,7 @@ __global__ void __launch_bounds__(128) gg_init_kernel(InitArgs a) {
         uint32_t w[6];
 #pragma unroll
         for (int r = 0; r < 6; r++) w[r] = rec[(uint64_t)(2 + r) * a.pitch];
-        gg_walk64(w, x, y);
+        gg_walk64_r2p(w, x, y);
     } else {
         gg_walk_generic(rec + 2 * a.pitch, a.pitch, a.l0, x, y, (uint32_t)a.m, a.pow2 != 0,
                         a.variant, 0);
@@ -177,7 +177,7 @@ __device__ __forceinline__ void emit_label(const FillArgs &a, uint64_t idx, uint
     }
 }
 
-template <int EMIT>
+template <int EMIT, int STEP = 1>
 __global__ void __launch_bounds__(64, 32) gg_fill64_tma_kernel(const __grid_constant__ CUtensorMap tmap,
                                                            FillArgs a, uint32_t units) {
     __shared__ __align__(128) uint32_t tiles[kFillWarps][2][kTileWords];
@@ -229,7 +229,10 @@ __global__ void __launch_bounds__(64, 32) gg_fill64_tma_kernel(const __grid_cons
 #pragma unroll
             for (int r = 0; r < 6; r++) w[r] = buf[r * 32 + lane];
             uint32_t nx = x, ny = y;
-            gg_walk64(w, nx, ny);
+            if (STEP)
+                gg_walk64_r2p(w, nx, ny);
+            else
+                gg_walk64(w, nx, ny);
             const bool active = j >= j0 && j < j1;
             if (active) {
                 x = nx;
@@ -254,7 +257,7 @@ __global__ void __launch_bounds__(64, 32) gg_fill64_tma_kernel(const __grid_cons
 // lane); one TMA box of 64 x 6 words (1.5 KB) per draw; the two walks are
 // interleaved step by step.  STEP: 1 = R2P form of the walk step (default),
 // 0 = per-step LOP3.P predicates (A/B hook GG_FILL_STEP=0).
-template <int EMIT, int MINB = 1, int STEP = 1>
+template <int EMIT, int MINB = 1, int STEP = 1, int U2 = 1>
 __global__ void __launch_bounds__(64, MINB) gg_fill64x2_tma_kernel(const __grid_constant__ CUtensorMap tmap,
                                                          FillArgs a, uint32_t units64) {
     constexpr int kTile = 6 * 64;
@@ -306,12 +309,9 @@ __global__ void __launch_bounds__(64, MINB) gg_fill64x2_tma_kernel(const __grid_
                 tma_load_tile(buf1, &tmap, bar1, (int32_t)(u * 64u), (int32_t)((jlo + 1 - a.Jw) * 6u));
             }
         }
-        for (uint32_t j = jlo; j < jhi; j++) {
-            const bool odd = ((j - jlo) & 1u) != 0;
-            uint32_t *buf = odd ? buf1 : buf0;
-            uint64_t *bar = odd ? bar1 : bar0;
-            mbar_wait(bar, odd ? ph1 : ph0);
-            if (odd) ph1 ^= 1u; else ph0 ^= 1u;
+        // One draw of both walkers from stage (buf, bar); refills the stage with draw j + 2.
+        auto draw = [&](uint32_t *buf, uint64_t *bar, uint32_t ph, uint32_t j) {
+            mbar_wait(bar, ph);
             uint32_t wa[6], wb[6];
 #pragma unroll
             for (int r = 0; r < 6; r++) {
@@ -338,6 +338,23 @@ __global__ void __launch_bounds__(64, MINB) gg_fill64x2_tma_kernel(const __grid_
                 asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
                 mbar_expect_tx(bar, kBytes);
                 tma_load_tile(buf, &tmap, bar, (int32_t)(u * 64u), (int32_t)((j + 2 - a.Jw) * 6u));
+            }
+        };
+        if (U2) {
+            // two draws per iteration: stage 0 holds even, stage 1 odd offsets from jlo
+            for (uint32_t j = jlo; j < jhi; j += 2) {
+                draw(buf0, bar0, ph0, j);
+                ph0 ^= 1u;
+                if (j + 1 < jhi) {
+                    draw(buf1, bar1, ph1, j + 1);
+                    ph1 ^= 1u;
+                }
+            }
+        } else {
+            for (uint32_t j = jlo; j < jhi; j++) {
+                const bool odd = ((j - jlo) & 1u) != 0;
+                draw(odd ? buf1 : buf0, odd ? bar1 : bar0, odd ? ph1 : ph0, j);
+                if (odd) ph1 ^= 1u; else ph0 ^= 1u;
             }
         }
         if (ta < a.W) {
@@ -569,23 +586,30 @@ cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count) {
                 plan_grid(gg_fill64x2_tma_kernel<2>, units64 * 2, sm_count, blocks, threads);
                 gg_fill64x2_tma_kernel<2><<<blocks, threads, 0, s>>>(map, a, units64);
             } else if (a.log2m == 32) {
-                // register budget (A/B hook GG_FILL_MINB; default 24 = 37 regs, 0.5% faster
-                // than ptxas' choice (1: 46 regs); 28 -> 32 regs is 5% slower; no spills)
-                static const int minb = getenv("GG_FILL_MINB") ? atoi(getenv("GG_FILL_MINB")) : 24;
+                // A/B hooks (measured on B200, C2 fill, profiles/r01_*):
+                //   GG_FILL_STEP=0  per-step LOP3.P predicates instead of R2P (8.93 vs 8.13 ms)
+                //   GG_FILL_U2=0    one draw per loop iteration instead of two (8.17 vs 8.13)
+                //   GG_FILL_MINB=24 37-40 registers / 48 warps per SM instead of ptxas' 55 /
+                //                   36 warps (8.39 vs 8.13: the R2P step wants the registers)
+                static const int minb = getenv("GG_FILL_MINB") ? atoi(getenv("GG_FILL_MINB")) : 1;
                 static const bool r2p = !(getenv("GG_FILL_STEP") && atoi(getenv("GG_FILL_STEP")) == 0);
-                if (minb == 24 && !r2p) {
-                    plan_grid(gg_fill64x2_tma_kernel<0, 24, 0>, units64 * 2, sm_count, blocks, threads);
-                    gg_fill64x2_tma_kernel<0, 24, 0><<<blocks, threads, 0, s>>>(map, a, units64);
-                } else if (minb == 24) {
-                    plan_grid(gg_fill64x2_tma_kernel<0, 24>, units64 * 2, sm_count, blocks, threads);
-                    gg_fill64x2_tma_kernel<0, 24><<<blocks, threads, 0, s>>>(map, a, units64);
-                } else if (minb == 28) {
-                    plan_grid(gg_fill64x2_tma_kernel<0, 28>, units64 * 2, sm_count, blocks, threads);
-                    gg_fill64x2_tma_kernel<0, 28><<<blocks, threads, 0, s>>>(map, a, units64);
-                } else {
-                    plan_grid(gg_fill64x2_tma_kernel<0>, units64 * 2, sm_count, blocks, threads);
-                    gg_fill64x2_tma_kernel<0><<<blocks, threads, 0, s>>>(map, a, units64);
-                }
+                static const bool u2 = !(getenv("GG_FILL_U2") && atoi(getenv("GG_FILL_U2")) == 0);
+#define GG_LAUNCH_X2(...)                                                                   \
+    do {                                                                                    \
+        plan_grid(gg_fill64x2_tma_kernel<__VA_ARGS__>, units64 * 2, sm_count, blocks, threads); \
+        gg_fill64x2_tma_kernel<__VA_ARGS__><<<blocks, threads, 0, s>>>(map, a, units64);    \
+    } while (0)
+                if (!r2p)
+                    GG_LAUNCH_X2(0, 24, 0, 0);
+                else if (minb == 24 && !u2)
+                    GG_LAUNCH_X2(0, 24, 1, 0);
+                else if (minb == 24)
+                    GG_LAUNCH_X2(0, 24, 1, 1);
+                else if (!u2)
+                    GG_LAUNCH_X2(0, 1, 1, 0);
+                else
+                    GG_LAUNCH_X2(0, 1, 1, 1);
+#undef GG_LAUNCH_X2
             } else {
                 plan_grid(gg_fill64x2_tma_kernel<1>, units64 * 2, sm_count, blocks, threads);
                 gg_fill64x2_tma_kernel<1><<<blocks, threads, 0, s>>>(map, a, units64);

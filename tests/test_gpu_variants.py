@@ -41,7 +41,8 @@ print(json.dumps({"bulk": [int(v) for v in bulk], "od": [int(v) for v in od.cpu(
                   "tallies": [int(v) for v in mc["tallies"]]}))
 """
 
-VARIANTS = ["GG_FILL_NO_TMA=1", "GG_FILL_X1=1", "GG_FILL_MINB=1", "GG_FILL_MINB=28",
+VARIANTS = ["GG_FILL_NO_TMA=1", "GG_FILL_X1=1", "GG_FILL_MINB=24", "GG_FILL_STEP=0", "GG_FILL_U2=0",
+            "GG_FILL_MINB=24 GG_FILL_U2=0",
             "GG_FILL_BPS=3", "GG_FILL_KPW=2", "GG_FEED_NT_ALL=1", "GG_FEED_NO_NT=1",
             "GG_FEED_CHUNK_MB=1", "GG_FEED_CHUNKS=2", "GG_MC_MINB=4"]
 
@@ -70,8 +71,9 @@ def want():
 @pytest.mark.parametrize("var", VARIANTS)
 def test_variant_bit_exact(var, want):
     env = dict(os.environ)
-    k, v = var.split("=")
-    env[k] = v
+    for kv in var.split():
+        k, v = kv.split("=")
+        env[k] = v
     out = subprocess.run([sys.executable, "-c", SNIPPET % {"root": ROOT}], env=env,
                          capture_output=True, text=True, timeout=300)
     assert out.returncode == 0, out.stderr[-2000:]

@@ -462,6 +462,93 @@ float run1(const uint32_t* bits, uint64_t pitch, uint32_t W, uint32_t D, uint32_
   float ms; cudaEventElapsedTime(&ms, a, b);
   return ms / reps;
 }
+
+// NW walkers per thread (t = u*32*NW + k*32 + lane), R2P step; groups interleaved across walkers.
+template <int NW, int NK>
+__device__ __forceinline__ void wordN(const uint32_t (&Q)[NW], uint32_t (&x)[NW], uint32_t (&y)[NW]) {
+  uint32_t C[NW], F[NW], G[NW];
+#pragma unroll
+  for (int k = 0; k < NW; k++) { prep12(Q[k], C[k], F[k]); G[k] = F[k] >> 6; }
+#define AW2(B0, B1, K0, K1, S) _Pragma("unroll") for (int k = 0; k < NW; k++) two13<B0, B1, SH(K0), SH(K1)>(S[k], C[k], x[k], y[k]);
+#define AW1(B0, K0, S) _Pragma("unroll") for (int k = 0; k < NW; k++) one13<B0, SH(K0)>(S[k], C[k], x[k], y[k]);
+  AW2(0, 3, 0, 1, F)
+  if (NK == 4) { AW2(0, 3, 2, 3, G) return; }
+  AW1(0, 2, G) AW2(9, 12, 3, 4, F) AW1(9, 5, G) AW2(18, 21, 6, 7, F) AW2(24, 27, 8, 9, F)
+#undef AW2
+#undef AW1
+}
+template <int NW>
+__device__ __forceinline__ void walkN(const uint32_t (&w)[NW][6], uint32_t (&x)[NW], uint32_t (&y)[NW]) {
+  uint32_t Q[NW];
+#pragma unroll
+  for (int k = 0; k < NW; k++) Q[k] = w[k][0];
+  wordN<NW, 10>(Q, x, y);
+#pragma unroll
+  for (int i = 1; i < 6; i++) {
+#pragma unroll
+    for (int k = 0; k < NW; k++) Q[k] = __funnelshift_r(w[k][i - 1], w[k][i], 32 - 2 * i);
+    wordN<NW, 10>(Q, x, y);
+  }
+#pragma unroll
+  for (int k = 0; k < NW; k++) Q[k] = w[k][5] >> 20;
+  wordN<NW, 4>(Q, x, y);
+}
+template <int NW, int MINB>
+__global__ void __launch_bounds__(64, MINB) kfillN(const uint32_t* __restrict__ bits, uint64_t pitch, uint32_t W, uint32_t D,
+                                             uint32_t* xs, uint32_t* ys, uint64_t* out, uint32_t units, uint32_t four) {
+  const uint32_t lane = threadIdx.x & 31u, warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+  for (uint32_t u = warp; u < units / NW; u += nwarps) {
+    uint32_t x[NW], y[NW], w0[NW][6], w1[NW][6];
+#pragma unroll
+    for (int k = 0; k < NW; k++) {
+      const uint32_t t = u * 32u * NW + k * 32u + lane;
+      x[k] = xs[t]; y[k] = ys[t];
+#pragma unroll
+      for (int r = 0; r < 6; r++) { w0[k][r] = __ldg(bits + t + (uint64_t)r * pitch); w1[k][r] = __ldg(bits + t + (uint64_t)(6 + r) * pitch); }
+    }
+    for (uint32_t j = 0; j < D; j++) {
+      uint32_t w2[NW][6];
+      const uint32_t jn = (j + 2 < D) ? j + 2 : j;
+#pragma unroll
+      for (int k = 0; k < NW; k++) {
+        const uint32_t t = u * 32u * NW + k * 32u + lane;
+#pragma unroll
+        for (int r = 0; r < 6; r++) w2[k][r] = __ldg(bits + t + ((uint64_t)jn * 6 + r) * pitch);
+      }
+      walkN<NW>(w0, x, y);
+#pragma unroll
+      for (int k = 0; k < NW; k++) {
+        const uint32_t t = u * 32u * NW + k * 32u + lane;
+        out[(uint64_t)j * W + t] = ((uint64_t)y[k] << 32) | x[k];
+#pragma unroll
+        for (int r = 0; r < 6; r++) { w0[k][r] = w1[k][r]; w1[k][r] = w2[k][r]; }
+      }
+    }
+#pragma unroll
+    for (int k = 0; k < NW; k++) { const uint32_t t = u * 32u * NW + k * 32u + lane; xs[t] = x[k]; ys[t] = y[k]; }
+  }
+}
+template <int NW, int MINB>
+float runN(const uint32_t* bits, uint64_t pitch, uint32_t W, uint32_t D, uint32_t* xs, uint32_t* ys, uint64_t* out,
+           int reps) {
+  uint32_t units = W / 32;
+  int per_sm = 0;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kfillN<NW, MINB>, 64, 0);
+  uint32_t max_warps = 148u * per_sm * 2;
+  uint32_t k = (units / NW + max_warps - 1) / max_warps;
+  uint32_t warps = (units / NW + k - 1) / k;
+  uint32_t blocks = (warps + 1) / 2;
+  cudaEvent_t a, b; cudaEventCreate(&a); cudaEventCreate(&b);
+  cudaEventRecord(a);
+  for (int r = 0; r < reps; r++) {
+    kinit<<<1184, 256>>>(xs, W); kinit<<<1184, 256>>>(ys, W);
+    kfillN<NW, MINB><<<blocks, 64>>>(bits, pitch, W, D, xs, ys, out, units, 4u);
+  }
+  cudaEventRecord(b); cudaEventSynchronize(b);
+  float ms; cudaEventElapsedTime(&ms, a, b);
+  return ms / reps;
+}
 int main(int argc, char** argv) {
   const uint32_t W = 1u << 20, D = 128;
   const int reps = argc > 1 ? atoi(argv[1]) : 5;
@@ -492,6 +579,11 @@ int main(int argc, char** argv) {
     printf("x1 warps/SM %d: V6 %.3f (%.1f) %s  V13 %.3f (%.1f) %s\n", wps, t6, labels / t6 / 1e6, ok6 ? "ok" : "MISMATCH",
            t13, labels / t13 / 1e6, got == ref ? "ok" : "MISMATCH");
   }
+#define RN(NW, MB) { float t = runN<NW, MB>(bits, pitch, W, D, xs, ys, out, reps); \
+    cudaMemcpy(got.data(), out + (size_t)(D - 1) * W, W * 8, cudaMemcpyDeviceToHost); \
+    int per_sm = 0; cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kfillN<NW, MB>, 64, 0); \
+    printf("N=%d minb=%d (%d blk/SM): %.3f ms (%.1f G/s) %s\n", NW, MB, per_sm, t, labels / t / 1e6, got == ref ? "ok" : "MISMATCH"); }
+  RN(1, 1) RN(2, 1) RN(2, 16) RN(2, 24) RN(3, 1) RN(3, 12) RN(4, 1) RN(4, 8)
   printf("err: %s\n", cudaGetErrorString(cudaGetLastError()));
   return 0;
 }
