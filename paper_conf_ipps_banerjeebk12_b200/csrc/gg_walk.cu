@@ -531,12 +531,17 @@ __global__ void __launch_bounds__(64) gg_fill_generic_kernel(FillArgs a, uint32_
     }
 }
 
-// One full wave: as many 64-thread blocks as can be resident on every SM at
-// once (occupancy API for the actual kernel), never more than the units need.
-// Units (32 walkers) go round-robin over all warps, so every SM gets the same
-// number of units +-1 and there is no partially filled second wave.
+// Grid of 64-thread blocks (2 warps each); `units` = work items a warp takes
+// round-robin (32 walkers; 64 for the x2 kernels).
+//  - spread = false: one wave, never more warps than can be resident at once
+//    (occupancy API for the actual kernel);
+//  - spread = true (the l = 64 walk kernels): one item per warp and let the block
+//    scheduler start a new block wherever one finishes.  A C2 fill has 16384 x2
+//    items for 5328 resident warps; any static split leaves SMs idle at the end
+//    (one wave: 8.15 ms; 2 items/warp: 7.98; 1 item/warp: 7.77).
 template <class K>
-static void plan_grid(K kernel, uint32_t units, int sm_count, uint32_t &blocks, uint32_t &threads) {
+static void plan_grid(K kernel, uint32_t units, int sm_count, uint32_t &blocks, uint32_t &threads,
+                      bool spread = false) {
     threads = 64;
     int per_sm = 0;
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, (int)threads, 0) !=
@@ -546,12 +551,12 @@ static void plan_grid(K kernel, uint32_t units, int sm_count, uint32_t &blocks, 
     static const int bps_env = getenv("GG_FILL_BPS") ? atoi(getenv("GG_FILL_BPS")) : 0;
     if (bps_env > 0 && bps_env < per_sm) per_sm = bps_env;
     const uint32_t cap = (uint32_t)sm_count * (uint32_t)per_sm;
-    const uint32_t need = (units + 1) / 2;  // 2 warps per block, >= 1 unit per warp
-    blocks = need < cap ? need : cap;
+    const uint32_t need = (units + 1) / 2;
+    blocks = (spread || need < cap) ? need : cap;
     static const int kpw = getenv("GG_FILL_KPW") ? atoi(getenv("GG_FILL_KPW")) : 0;
-    if (kpw > 0) {  // experiment: exactly kpw units per warp (may exceed one wave)
-        const uint32_t warps = (units + kpw - 1) / kpw;
-        blocks = (warps + 1) / 2;
+    if (kpw > 0) {  // experiment: exactly kpw units per warp
+        const uint32_t w = (units + kpw - 1) / kpw;
+        blocks = (w + 1) / 2;
     }
     if (blocks == 0) blocks = 1;
 }
@@ -583,7 +588,7 @@ cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count) {
         const uint32_t units64 = (a.W + 63u) / 64u;
         if (use_tma && use_x2 && a.rows && make_window_map(&map, a.bits, a.pitch, a.rows, 64)) {
             if (a.out_u32) {
-                plan_grid(gg_fill64x2_tma_kernel<2>, units64 * 2, sm_count, blocks, threads);
+                plan_grid(gg_fill64x2_tma_kernel<2>, units64, sm_count, blocks, threads, true);
                 gg_fill64x2_tma_kernel<2><<<blocks, threads, 0, s>>>(map, a, units64);
             } else if (a.log2m == 32) {
                 // A/B hooks (measured on B200, C2 fill, profiles/r01_*):
@@ -596,7 +601,7 @@ cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count) {
                 static const bool u2 = !(getenv("GG_FILL_U2") && atoi(getenv("GG_FILL_U2")) == 0);
 #define GG_LAUNCH_X2(...)                                                                   \
     do {                                                                                    \
-        plan_grid(gg_fill64x2_tma_kernel<__VA_ARGS__>, units64 * 2, sm_count, blocks, threads); \
+        plan_grid(gg_fill64x2_tma_kernel<__VA_ARGS__>, units64, sm_count, blocks, threads, true); \
         gg_fill64x2_tma_kernel<__VA_ARGS__><<<blocks, threads, 0, s>>>(map, a, units64);    \
     } while (0)
                 if (!r2p)
@@ -611,18 +616,18 @@ cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count) {
                     GG_LAUNCH_X2(0, 1, 1, 1);
 #undef GG_LAUNCH_X2
             } else {
-                plan_grid(gg_fill64x2_tma_kernel<1>, units64 * 2, sm_count, blocks, threads);
+                plan_grid(gg_fill64x2_tma_kernel<1>, units64, sm_count, blocks, threads, true);
                 gg_fill64x2_tma_kernel<1><<<blocks, threads, 0, s>>>(map, a, units64);
             }
         } else if (use_tma && a.rows && make_window_map(&map, a.bits, a.pitch, a.rows)) {
             if (a.out_u32) {
-                plan_grid(gg_fill64_tma_kernel<2>, units, sm_count, blocks, threads);
+                plan_grid(gg_fill64_tma_kernel<2>, units, sm_count, blocks, threads, true);
                 gg_fill64_tma_kernel<2><<<blocks, threads, 0, s>>>(map, a, units);
             } else if (a.log2m == 32) {
-                plan_grid(gg_fill64_tma_kernel<0>, units, sm_count, blocks, threads);
+                plan_grid(gg_fill64_tma_kernel<0>, units, sm_count, blocks, threads, true);
                 gg_fill64_tma_kernel<0><<<blocks, threads, 0, s>>>(map, a, units);
             } else {
-                plan_grid(gg_fill64_tma_kernel<1>, units, sm_count, blocks, threads);
+                plan_grid(gg_fill64_tma_kernel<1>, units, sm_count, blocks, threads, true);
                 gg_fill64_tma_kernel<1><<<blocks, threads, 0, s>>>(map, a, units);
             }
         } else if (a.out_u32) {
