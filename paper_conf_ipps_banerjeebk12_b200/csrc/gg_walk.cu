@@ -532,29 +532,28 @@ __global__ void __launch_bounds__(64) gg_fill_generic_kernel(FillArgs a, uint32_
 }
 
 // Grid of 64-thread blocks (2 warps each); `units` = work items a warp takes
-// round-robin (32 walkers; 64 for the x2 kernels).
-//  - spread = false: one wave, never more warps than can be resident at once
-//    (occupancy API for the actual kernel);
-//  - spread = true (the l = 64 walk kernels): one item per warp and let the block
-//    scheduler start a new block wherever one finishes.  A C2 fill has 16384 x2
-//    items for 5328 resident warps; any static split leaves SMs idle at the end
-//    (one wave: 8.15 ms; 2 items/warp: 7.98; 1 item/warp: 7.77).
+// round-robin (32 walkers; 64 for the x2 kernels).  One item per warp: the
+// block scheduler starts a new block wherever one finishes, so SMs stay busy to
+// the end.  A one-wave grid (A/B hook GG_FILL_ONEWAVE=1: as many warps as are
+// resident at once, items round-robin) leaves most warps idle during the last
+// partial round: C2 (16384 x2 items, 5328 resident warps) 8.15 -> 7.77 ms;
+// l = 1 fill (32768 items) 2.56 -> 2.22 ms.
 template <class K>
-static void plan_grid(K kernel, uint32_t units, int sm_count, uint32_t &blocks, uint32_t &threads,
-                      bool spread = false) {
+static void plan_grid(K kernel, uint32_t units, int sm_count, uint32_t &blocks, uint32_t &threads) {
     threads = 64;
-    int per_sm = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, (int)threads, 0) !=
-            cudaSuccess ||
-        per_sm <= 0)
-        per_sm = 16;
-    static const int bps_env = getenv("GG_FILL_BPS") ? atoi(getenv("GG_FILL_BPS")) : 0;
-    if (bps_env > 0 && bps_env < per_sm) per_sm = bps_env;
-    const uint32_t cap = (uint32_t)sm_count * (uint32_t)per_sm;
-    const uint32_t need = (units + 1) / 2;
-    blocks = (spread || need < cap) ? need : cap;
+    blocks = (units + 1) / 2;
+    static const bool onewave = getenv("GG_FILL_ONEWAVE") != nullptr;
+    if (onewave) {
+        int per_sm = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, (int)threads, 0) !=
+                cudaSuccess ||
+            per_sm <= 0)
+            per_sm = 16;
+        const uint32_t cap = (uint32_t)sm_count * (uint32_t)per_sm;
+        if (blocks > cap) blocks = cap;
+    }
     static const int kpw = getenv("GG_FILL_KPW") ? atoi(getenv("GG_FILL_KPW")) : 0;
-    if (kpw > 0) {  // experiment: exactly kpw units per warp
+    if (kpw > 0) {  // experiment: exactly kpw items per warp
         const uint32_t w = (units + kpw - 1) / kpw;
         blocks = (w + 1) / 2;
     }
@@ -588,7 +587,7 @@ cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count) {
         const uint32_t units64 = (a.W + 63u) / 64u;
         if (use_tma && use_x2 && a.rows && make_window_map(&map, a.bits, a.pitch, a.rows, 64)) {
             if (a.out_u32) {
-                plan_grid(gg_fill64x2_tma_kernel<2>, units64, sm_count, blocks, threads, true);
+                plan_grid(gg_fill64x2_tma_kernel<2>, units64, sm_count, blocks, threads);
                 gg_fill64x2_tma_kernel<2><<<blocks, threads, 0, s>>>(map, a, units64);
             } else if (a.log2m == 32) {
                 // A/B hooks (measured on B200, C2 fill, profiles/r01_*):
@@ -601,7 +600,7 @@ cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count) {
                 static const bool u2 = !(getenv("GG_FILL_U2") && atoi(getenv("GG_FILL_U2")) == 0);
 #define GG_LAUNCH_X2(...)                                                                   \
     do {                                                                                    \
-        plan_grid(gg_fill64x2_tma_kernel<__VA_ARGS__>, units64, sm_count, blocks, threads, true); \
+        plan_grid(gg_fill64x2_tma_kernel<__VA_ARGS__>, units64, sm_count, blocks, threads); \
         gg_fill64x2_tma_kernel<__VA_ARGS__><<<blocks, threads, 0, s>>>(map, a, units64);    \
     } while (0)
                 if (!r2p)
@@ -616,18 +615,18 @@ cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count) {
                     GG_LAUNCH_X2(0, 1, 1, 1);
 #undef GG_LAUNCH_X2
             } else {
-                plan_grid(gg_fill64x2_tma_kernel<1>, units64, sm_count, blocks, threads, true);
+                plan_grid(gg_fill64x2_tma_kernel<1>, units64, sm_count, blocks, threads);
                 gg_fill64x2_tma_kernel<1><<<blocks, threads, 0, s>>>(map, a, units64);
             }
         } else if (use_tma && a.rows && make_window_map(&map, a.bits, a.pitch, a.rows)) {
             if (a.out_u32) {
-                plan_grid(gg_fill64_tma_kernel<2>, units, sm_count, blocks, threads, true);
+                plan_grid(gg_fill64_tma_kernel<2>, units, sm_count, blocks, threads);
                 gg_fill64_tma_kernel<2><<<blocks, threads, 0, s>>>(map, a, units);
             } else if (a.log2m == 32) {
-                plan_grid(gg_fill64_tma_kernel<0>, units, sm_count, blocks, threads, true);
+                plan_grid(gg_fill64_tma_kernel<0>, units, sm_count, blocks, threads);
                 gg_fill64_tma_kernel<0><<<blocks, threads, 0, s>>>(map, a, units);
             } else {
-                plan_grid(gg_fill64_tma_kernel<1>, units, sm_count, blocks, threads, true);
+                plan_grid(gg_fill64_tma_kernel<1>, units, sm_count, blocks, threads);
                 gg_fill64_tma_kernel<1><<<blocks, threads, 0, s>>>(map, a, units);
             }
         } else if (a.out_u32) {
