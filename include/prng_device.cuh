@@ -249,13 +249,12 @@ __device__ __forceinline__ void gg_word10_r2p(uint32_t Q, uint32_t &x, uint32_t 
     gg_r2p_two<24, 27, GG_SH(8), GG_SH(9)>(F, C, x, y);
 }
 
+/* Steps of one 10-field word (NK = 10) or of the 4-field tail word (NK = 4) for
+ * two walkers, from prepared (C, F) of each. */
 template <int NK>
-__device__ __forceinline__ void gg_word10x2_r2p(uint32_t Qa, uint32_t Qb, uint32_t &xa, uint32_t &ya,
-                                                uint32_t &xb, uint32_t &yb)
+__device__ __forceinline__ void gg_steps10x2_r2p(uint32_t Ca, uint32_t Fa, uint32_t Cb, uint32_t Fb,
+                                                 uint32_t &xa, uint32_t &ya, uint32_t &xb, uint32_t &yb)
 {
-    uint32_t Ca, Fa, Cb, Fb;
-    gg_r2p_prep(Qa, Ca, Fa);
-    gg_r2p_prep(Qb, Cb, Fb);
     const uint32_t Ga = Fa >> 6, Gb = Fb >> 6;
 #define GG_R2P2(B0, B1, K0, K1, SA, SB)                                     \
     gg_r2p_two<B0, B1, GG_SH(K0), GG_SH(K1)>(SA, Ca, xa, ya);                \
@@ -275,6 +274,16 @@ __device__ __forceinline__ void gg_word10x2_r2p(uint32_t Qa, uint32_t Qb, uint32
     GG_R2P2(24, 27, 8, 9, Fa, Fb)
 #undef GG_R2P2
 #undef GG_R2P1
+}
+
+template <int NK>
+__device__ __forceinline__ void gg_word10x2_r2p(uint32_t Qa, uint32_t Qb, uint32_t &xa, uint32_t &ya,
+                                                uint32_t &xb, uint32_t &yb)
+{
+    uint32_t Ca, Fa, Cb, Fb;
+    gg_r2p_prep(Qa, Ca, Fa);
+    gg_r2p_prep(Qb, Cb, Fb);
+    gg_steps10x2_r2p<NK>(Ca, Fa, Cb, Fb, xa, ya, xb, yb);
 }
 
 /* 64 steps from a 6-word record (R2P form). */
