@@ -362,7 +362,9 @@ def run_ours(args, rank, world, local_rank):
         od_ms = max_over_ranks(a.elapsed_time(b))
         res["on_demand"] = {"uniform_S100": world * W_PER_GPU * S / (od_ms / 1e3) / 1e9,
                             "unit": UNIT, "draws": world * W_PER_GPU * S, "ms": od_ms,
-                            "what": "gg_consume: 2^20 threads/GPU x 100 prng_next each, bits resident"}
+                            "what": "gg_consume: 2^20 threads/GPU x 100 prng_next each, bits resident",
+                            "roofline_frac_uniform": (W_PER_GPU * S * OPS_PER_LABEL / (od_ms / 1e3))
+                            / (props.multi_processor_count * 128 * sm_max * 1e6)}
         g.close()
         torch.cuda.empty_cache()
         res["on_demand"].update(ondemand_shaped(rank, world, local_rank, stream, max_over_ranks))
