@@ -64,3 +64,71 @@ def test_swar_recipe_every_field_value_at_every_position():
             w = [(bits >> (32 * r)) & M for r in range(6)]
             x0, y0 = (int(v) for v in rng.integers(0, 2 ** 32, 2, dtype=np.uint64))
             assert walk64_swar(w, x0, y0) == O.walk(1 << 32, x0, y0, np.array(w, np.uint32), 64)
+
+
+# ---------------------------------------------------------------------------
+# R2P form (gg_word10_r2p / gg_word10x2_r2p): the step predicates are not
+# tested bit by bit; R2P PR, S.Bn, mask loads predicate register P_i from bit
+# i (i = 0..6) of byte n of S.  Model exactly that: for each group the kernel
+# names a source (F or G = F >> 6), a byte and the bit offsets of py/px inside
+# the byte; the step then reads P[bit] of that byte only.  A wrong byte, a
+# flag outside bits 0..6 of its byte, or a wrong G shift fails here.
+
+def _r2p_load(S, byte):
+    v = (S >> (8 * byte)) & 0xFF
+    return [(v >> i) & 1 for i in range(7)]  # P0..P6 (bit 7 is not loadable)
+
+
+# (source, step k, bit of py within S) for the 10-field word, as in
+# gg_word10_r2p: F.B0 0,1 | G.B0 2 | F.B1 3,4 | G.B1 5 | F.B2 6,7 | F.B3 8,9
+R2P_GROUPS_10 = [("F", 0, 0), ("F", 1, 3), ("G", 2, 0), ("F", 3, 9), ("F", 4, 12),
+                 ("G", 5, 9), ("F", 6, 18), ("F", 7, 21), ("F", 8, 24), ("F", 9, 27)]
+R2P_GROUPS_4 = [("F", 0, 0), ("F", 1, 3), ("G", 2, 0), ("G", 3, 3)]
+
+
+def _word10_r2p(Q, nk, x, y):
+    f1, f2 = Q >> 1, Q >> 2
+    MY = ((f1 | Q) & 0x09249249) & ~f2 & M
+    MX = (f2 & ~(f1 & Q)) & M
+    C = (Q - MY) & M
+    F = (MY | ((MX << 1) & 0x12492492)) & M
+    G = F >> 6
+    for src, k, bit in (R2P_GROUPS_10 if nk == 10 else R2P_GROUPS_4):
+        S = F if src == "F" else G
+        byte, off = bit // 8, bit % 8
+        assert off + 1 <= 6, "flag outside the 7 loadable bits of the byte"
+        P = _r2p_load(S, byte)
+        py, px = P[off], P[off + 1]
+        c = ((C << (30 - 3 * k)) & M) >> 30
+        u = (x + y + c) & M
+        if py:
+            y = (u + x) & M
+        if px:
+            x = (u + y) & M
+    return x, y
+
+
+def walk64_r2p(w, x, y):
+    x, y = _word10_r2p(w[0], 10, x, y)
+    for a, s in [(0, 30), (1, 28), (2, 26), (3, 24), (4, 22)]:
+        x, y = _word10_r2p(_fsr(w[a], w[a + 1], s), 10, x, y)
+    return _word10_r2p(w[5] >> 20, 4, x, y)
+
+
+def test_r2p_groups_cover_each_step_once_in_order():
+    for groups, nk in ((R2P_GROUPS_10, 10), (R2P_GROUPS_4, 4)):
+        assert [k for _, k, _ in groups] == list(range(nk))
+        for src, k, bit in groups:  # the flags of step k sit at 3k (F) or 3k - 6 (G)
+            assert bit == (3 * k if src == "F" else 3 * k - 6)
+
+
+def test_r2p_recipe_every_field_value_at_every_position():
+    rng = np.random.default_rng(11)
+    for i in range(64):
+        for b in range(8):
+            bits = int.from_bytes(rng.bytes(24), "little")
+            bits &= ~(7 << (3 * i))
+            bits |= b << (3 * i)
+            w = [(bits >> (32 * r)) & M for r in range(6)]
+            x0, y0 = (int(v) for v in rng.integers(0, 2 ** 32, 2, dtype=np.uint64))
+            assert walk64_r2p(w, x0, y0) == O.walk(1 << 32, x0, y0, np.array(w, np.uint32), 64)
