@@ -17,6 +17,12 @@ walks the same 12 GiB of bits (larger than L2: no flush needed) and writes
 threads generate every bit, H2D copies, the walk, D2H of all numbers.
 `--impl reference` times the CPU oracle (the paper's method as plain C) on
 the host cores instead.
+
+`--workload c5` runs config C5 instead (BJ:configs "2^34 numbers sharded over
+1/2/4/8 B200"): 2^34 labels in total from 2^23 walkers split over
+the ranks (strong scaling), each rank filling a reused 2 GiB buffer; value =
+labels / summed fill time with each fill's bits prefetched (K-mode), e2e =
+the same job with the host FEED streaming the bits during the walk (E-mode).
 """
 from __future__ import annotations
 
@@ -406,6 +412,133 @@ def run_ours(args, rank, world, local_rank):
     return res
 
 
+# ------------------------------------------------------- C5 scaling sweep
+C5_LABELS = 1 << 34          # BJ:configs "2^34 numbers sharded over 1/2/4/8 B200"
+C5_WALKERS = 1 << 23         # W = 2^23 in total, split G ways (strong scaling)
+C5_CHUNK = 1 << 28           # labels per fill: a 2 GiB reused u64 buffer per GPU
+C5_SEED = 0x5EED0005
+C5_WORKLOAD = ("C5 scaling sweep: 2^34 64-bit labels in total (m=2^32, l=l0=64), 2^23 walkers "
+               "split over the GPUs (global walker ids, disjoint seed-bit streams), each GPU "
+               "filling a reused 2 GiB buffer (2^28 labels per prng_fill)")
+
+
+def run_c5(args, rank, world, local_rank):
+    """One step = the whole C5 job.  K-mode (value): per chunk the chunk's bits
+    are made resident by prng_prefetch (host FEED + H2D, untimed), then the
+    fill is timed with CUDA events; time = max over ranks of the summed fill
+    times.  E-mode (e2e): a second generator on the same seed runs the same
+    job through prng_fill with the host FEED and H2D overlapped with the
+    walk (the paper's regime), wall time between device synchronisations,
+    max over ranks; the last label is read back to the host."""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_ipps_banerjeebk12_b200 import Generator
+
+    if C5_WALKERS % world or (C5_LABELS // world) % C5_CHUNK:
+        raise SystemExit(f"C5 needs world in (1, 2, 4, 8, ...); got {world}")
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    props = torch.cuda.get_device_properties(dev)
+    stream = torch.cuda.current_stream()
+    local_world = int(os.environ.get("LOCAL_WORLD_SIZE", str(world)))
+    feed_threads = max(1, (os.cpu_count() or 1) // max(1, local_world))
+    Wr = C5_WALKERS // world
+    base = rank * Wr
+    Lr = C5_LABELS // world
+    chunks = Lr // C5_CHUNK
+    draws_per_chunk = C5_CHUNK // Wr
+
+    def max_over_ranks(v: float) -> float:
+        if world == 1:
+            return v
+        t = torch.tensor([v], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    out = torch.empty(C5_CHUNK, dtype=torch.int64, device=dev)
+    gpu_id = getattr(props, "uuid", None)
+    gpu_id = f"GPU-{gpu_id}" if gpu_id is not None else str(local_rank)
+    clk = ClockSampler(gpu_id, local_rank).__enter__()
+
+    def k_job(timed: bool):
+        g = Generator(walkers=Wr, seed=C5_SEED, walker_base=base, device=local_rank,
+                      host_threads=feed_threads)
+        kms, launches = 0.0, 0
+        for c in range(chunks):
+            g.prefetch(draws_per_chunk)
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            l0 = g.stats()["kernel_launches"]
+            a.record(stream)
+            g.fill(out)
+            b.record(stream)
+            b.synchronize()
+            launches += g.stats()["kernel_launches"] - l0
+            kms += a.elapsed_time(b)
+        g.close()
+        return kms, launches
+
+    # warm-up: one chunk's worth of work per warm-up step (allocations, feed threads, clocks)
+    for _ in range(args.warmup):
+        g = Generator(walkers=Wr, seed=C5_SEED, walker_base=base, device=local_rank,
+                      host_threads=feed_threads)
+        g.prefetch(draws_per_chunk)
+        g.fill(out)
+        g.close()
+    torch.cuda.synchronize()
+    barrier()
+    clk.mark(True)
+    k_ms, launches = [], 0
+    for _ in range(args.steps):
+        ms, n = k_job(True)
+        k_ms.append(max_over_ranks(ms))
+        launches += n
+    clk.mark(False)
+    clk.__exit__(None, None, None)
+    ms = sum(k_ms)
+    value = C5_LABELS * args.steps / (ms / 1e3) / 1e9
+    peaks = measured_peaks()
+    sm_max = float(peaks.get("sm_max_mhz", 1965.0))
+    peak_ops = props.multi_processor_count * 128 * sm_max * 1e6
+    per_fill_ms = statistics.mean(k_ms) / chunks
+    achieved = C5_CHUNK * OPS_PER_LABEL / (per_fill_ms / 1e3)
+    roofline = {
+        "bound": "alu", "achieved": achieved / 1e12, "peak": peak_ops / 1e12,
+        "unit": "Tops/s (32-bit integer ops)", "frac": achieved / peak_ops, "traffic": None,
+        "kernel": "gg_fill64x2_tma_kernel", "kernel_ms": per_fill_ms, "ops_per_label": OPS_PER_LABEL,
+        "note": "per-launch time = summed fill time / fills (max over ranks)"}
+
+    # E-mode: the same job with the bits streamed by the host FEED during the walk
+    e2e = None
+    if not args.no_e2e:
+        g = Generator(walkers=Wr, seed=C5_SEED, walker_base=base, device=local_rank,
+                      epoch_draws=16, host_threads=feed_threads)
+        host_last = torch.empty(1, dtype=torch.int64).pin_memory()
+        s0 = g.stats()
+        barrier()
+        torch.cuda.synchronize()
+        t = time.perf_counter()
+        for c in range(chunks):
+            g.fill(out)
+        host_last.copy_(out[-1:], non_blocking=False)
+        torch.cuda.synchronize()
+        dt = max_over_ranks(time.perf_counter() - t)
+        s1 = g.stats()
+        g.close()
+        e2e = {"value": C5_LABELS / dt / 1e9, "unit": UNIT,
+               "h2d_bytes_per_step": s1["h2d_bytes"] - s0["h2d_bytes"],
+               "d2h_bytes_per_step": 8, "steps": 1, "ms_wall": dt * 1e3,
+               "feed_s": s1["feed_seconds"] - s0["feed_seconds"], "host_threads": feed_threads,
+               "api": "prng_fill into the reused device buffer, host FEED -> pinned -> H2D "
+                      "overlapped with the walk; last label read back"}
+    return {"value": value, "ms": ms, "roofline": roofline, "clocks": clk.summary(),
+            "launches": launches, "e2e": e2e, "walkers_per_gpu": Wr, "chunks_per_gpu": chunks,
+            "draws_per_chunk": draws_per_chunk}
+
+
 def host_info():
     """nproc and CPU model of the box (SURVEY §8(d) reporting rules)."""
     model = None
@@ -587,7 +720,10 @@ def run_apps(args, rank, world, local_rank, max_over_ranks, feed_threads=0):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--steps", type=int, default=None, help="default 10 (C2), 1 (C5)")
+    ap.add_argument("--workload", default="c2", choices=["c2", "c5"],
+                    help="c2: bulk fill per GPU (weak scaling, default); c5: 2^34 labels split "
+                         "over the GPUs (strong scaling)")
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--e2e-steps", type=int, default=2)
@@ -598,6 +734,8 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=8.0)
     args = ap.parse_args()
+    if args.steps is None:
+        args.steps = 1 if args.workload == "c5" else 10
     if args.warmup < 3:
         args.warmup = 3
 
@@ -627,6 +765,28 @@ def main():
             dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
         else:
             dist.init_process_group(backend)
+    if args.workload == "c5":
+        res = run_c5(args, rank, world, local_rank)
+        if rank == 0:
+            print(json.dumps({
+                "metric": METRIC, "value": res["value"], "unit": UNIT, "n_gpus": world,
+                "steps": args.steps, "warmup": args.warmup, "ms_per_step": res["ms"] / args.steps,
+                "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u64",
+                "data": "synthetic (SplitMix64 counter-hash seed bits, reading R9)",
+                "config": {"workload": C5_WORKLOAD, "number": "one 64-bit vertex label",
+                           "walkers_per_gpu": res["walkers_per_gpu"],
+                           "fills_per_gpu_per_step": res["chunks_per_gpu"],
+                           "draws_per_fill": res["draws_per_chunk"],
+                           "bits": "each fill's bits made resident by prng_prefetch (untimed); "
+                                   "value = labels / summed fill kernel time (K-mode)",
+                           "l2": "inputs larger than L2 (>= 6 GiB of bits per fill)",
+                           "parallelism": f"walker shards dp{world}, no data-path collective"},
+                "roofline": res["roofline"], "cpu_baseline": cpu, "e2e": res["e2e"],
+                "clocks": res["clocks"], "gpu_launches": res["launches"], "host": host_info()}))
+        if world > 1:
+            import torch.distributed as dist
+            dist.destroy_process_group()
+        return 0
     res = run_ours(args, rank, world, local_rank)
     if rank == 0:
         line = {
