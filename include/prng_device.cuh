@@ -177,12 +177,13 @@ __device__ __forceinline__ void gg_walk64x2(const uint32_t a[6], const uint32_t 
  * predicate register file from one byte of a flag word: ptxas turns four
  * single-bit tests of the same register that fall inside one byte into one
  * R2P PR, F.Bn (measured, tools/step_bench2.cu).  Per 10-field word:
- *   F = MY at field bit 0 (y-move) | MX at field bit 1 (x-move),  G = F >> 6
- * and the 10 steps are grouped so that each group's flags sit in bits 0..6 of
- * one byte of F or G:
- *   F.B0 steps 0,1 | G.B0 step 2 | F.B1 steps 3,4 | G.B1 step 5 |
- *   F.B2 steps 6,7 | F.B3 steps 8,9        (4-field tail word: F.B0 0,1 | G.B0 2,3)
- * i.e. 6 R2P + 1 shift per 10 steps instead of 20 LOP3.P.  The arithmetic is
+ *   F = MY at field bit 0 (y-move) | MX at field bit 1 (x-move),  G = F >> 4
+ * and the 10 steps are grouped in pairs so that each pair's four flags sit in
+ * bits 0..6 of one byte of F or G (step k's flags: F bits 3k, 3k+1):
+ *   F.B0 steps 0,1 | G.B0 steps 2,3 | G.B1 steps 4,5 | F.B2 steps 6,7 |
+ *   F.B3 steps 8,9                          (4-field tail word: F.B0 | G.B0)
+ * i.e. 5 R2P + 1 shift per 10 steps instead of 20 LOP3.P (with G = F >> 6 no
+ * pairing covers all ten steps: 6 R2P).  The arithmetic is
  * unchanged (u = x + y + c; y' = u + x | x' = u + y), so both forms are the
  * same evaluation of the paper's step.
  * ------------------------------------------------------------------------ */
@@ -207,18 +208,6 @@ __device__ __forceinline__ void gg_r2p_two(uint32_t S, uint32_t C, uint32_t &x, 
           "n"(SH1));
 }
 
-template <int B0, int SH0>
-__device__ __forceinline__ void gg_r2p_one(uint32_t S, uint32_t C, uint32_t &x, uint32_t &y)
-{
-    asm volatile(
-        "{\n\t.reg .pred py0, px0;\n\t.reg .b32 t, ct, c, u, s;\n\t"
-        "and.b32 t, %2, %4;\n\tsetp.ne.b32 py0, t, 0;\n\t"
-        "and.b32 t, %2, %5;\n\tsetp.ne.b32 px0, t, 0;\n\t"
-        GG_R2P_U("%6") "@py0 add.u32 %1, u, %0;\n\t@px0 add.u32 %0, u, %1;\n\t}"
-        : "+r"(x), "+r"(y)
-        : "r"(S), "r"(C), "n"(1u << B0), "n"(2u << B0), "n"(SH0));
-}
-
 /* Flag word F and constant word C of a 10-field word Q (fields at 3i). */
 __device__ __forceinline__ void gg_r2p_prep(uint32_t Q, uint32_t &C, uint32_t &F)
 {
@@ -236,15 +225,11 @@ __device__ __forceinline__ void gg_word10_r2p(uint32_t Q, uint32_t &x, uint32_t 
 {
     uint32_t C, F;
     gg_r2p_prep(Q, C, F);
-    const uint32_t G = F >> 6;
+    const uint32_t G = F >> 4;
     gg_r2p_two<0, 3, GG_SH(0), GG_SH(1)>(F, C, x, y);
-    if (NK == 4) {
-        gg_r2p_two<0, 3, GG_SH(2), GG_SH(3)>(G, C, x, y);
-        return;
-    }
-    gg_r2p_one<0, GG_SH(2)>(G, C, x, y);
-    gg_r2p_two<9, 12, GG_SH(3), GG_SH(4)>(F, C, x, y);
-    gg_r2p_one<9, GG_SH(5)>(G, C, x, y);
+    gg_r2p_two<2, 5, GG_SH(2), GG_SH(3)>(G, C, x, y);
+    if (NK == 4) return;
+    gg_r2p_two<8, 11, GG_SH(4), GG_SH(5)>(G, C, x, y);
     gg_r2p_two<18, 21, GG_SH(6), GG_SH(7)>(F, C, x, y);
     gg_r2p_two<24, 27, GG_SH(8), GG_SH(9)>(F, C, x, y);
 }
@@ -255,25 +240,17 @@ template <int NK>
 __device__ __forceinline__ void gg_steps10x2_r2p(uint32_t Ca, uint32_t Fa, uint32_t Cb, uint32_t Fb,
                                                  uint32_t &xa, uint32_t &ya, uint32_t &xb, uint32_t &yb)
 {
-    const uint32_t Ga = Fa >> 6, Gb = Fb >> 6;
+    const uint32_t Ga = Fa >> 4, Gb = Fb >> 4;
 #define GG_R2P2(B0, B1, K0, K1, SA, SB)                                     \
     gg_r2p_two<B0, B1, GG_SH(K0), GG_SH(K1)>(SA, Ca, xa, ya);                \
     gg_r2p_two<B0, B1, GG_SH(K0), GG_SH(K1)>(SB, Cb, xb, yb);
-#define GG_R2P1(B0, K0, SA, SB)                                              \
-    gg_r2p_one<B0, GG_SH(K0)>(SA, Ca, xa, ya);                               \
-    gg_r2p_one<B0, GG_SH(K0)>(SB, Cb, xb, yb);
     GG_R2P2(0, 3, 0, 1, Fa, Fb)
-    if (NK == 4) {
-        GG_R2P2(0, 3, 2, 3, Ga, Gb)
-        return;
-    }
-    GG_R2P1(0, 2, Ga, Gb)
-    GG_R2P2(9, 12, 3, 4, Fa, Fb)
-    GG_R2P1(9, 5, Ga, Gb)
+    GG_R2P2(2, 5, 2, 3, Ga, Gb)
+    if (NK == 4) return;
+    GG_R2P2(8, 11, 4, 5, Ga, Gb)
     GG_R2P2(18, 21, 6, 7, Fa, Fb)
     GG_R2P2(24, 27, 8, 9, Fa, Fb)
 #undef GG_R2P2
-#undef GG_R2P1
 }
 
 template <int NK>

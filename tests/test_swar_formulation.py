@@ -80,10 +80,11 @@ def _r2p_load(S, byte):
 
 
 # (source, step k, bit of py within S) for the 10-field word, as in
-# gg_word10_r2p: F.B0 0,1 | G.B0 2 | F.B1 3,4 | G.B1 5 | F.B2 6,7 | F.B3 8,9
-R2P_GROUPS_10 = [("F", 0, 0), ("F", 1, 3), ("G", 2, 0), ("F", 3, 9), ("F", 4, 12),
-                 ("G", 5, 9), ("F", 6, 18), ("F", 7, 21), ("F", 8, 24), ("F", 9, 27)]
-R2P_GROUPS_4 = [("F", 0, 0), ("F", 1, 3), ("G", 2, 0), ("G", 3, 3)]
+# gg_word10_r2p with G = F >> 4: F.B0 0,1 | G.B0 2,3 | G.B1 4,5 | F.B2 6,7 | F.B3 8,9
+G_SHIFT = 4
+R2P_GROUPS_10 = [("F", 0, 0), ("F", 1, 3), ("G", 2, 2), ("G", 3, 5), ("G", 4, 8),
+                 ("G", 5, 11), ("F", 6, 18), ("F", 7, 21), ("F", 8, 24), ("F", 9, 27)]
+R2P_GROUPS_4 = [("F", 0, 0), ("F", 1, 3), ("G", 2, 2), ("G", 3, 5)]
 
 
 def _word10_r2p(Q, nk, x, y):
@@ -92,7 +93,7 @@ def _word10_r2p(Q, nk, x, y):
     MX = (f2 & ~(f1 & Q)) & M
     C = (Q - MY) & M
     F = (MY | ((MX << 1) & 0x12492492)) & M
-    G = F >> 6
+    G = F >> G_SHIFT
     for src, k, bit in (R2P_GROUPS_10 if nk == 10 else R2P_GROUPS_4):
         S = F if src == "F" else G
         byte, off = bit // 8, bit % 8
@@ -118,8 +119,14 @@ def walk64_r2p(w, x, y):
 def test_r2p_groups_cover_each_step_once_in_order():
     for groups, nk in ((R2P_GROUPS_10, 10), (R2P_GROUPS_4, 4)):
         assert [k for _, k, _ in groups] == list(range(nk))
-        for src, k, bit in groups:  # the flags of step k sit at 3k (F) or 3k - 6 (G)
-            assert bit == (3 * k if src == "F" else 3 * k - 6)
+        for src, k, bit in groups:  # the flags of step k sit at 3k (F) or 3k - G_SHIFT (G)
+            assert bit == (3 * k if src == "F" else 3 * k - G_SHIFT)
+        # steps are paired: each R2P (source, byte) loads the flags of two steps
+        loads = {}
+        for src, k, bit in groups:
+            loads.setdefault((src, bit // 8), []).append(k)
+        assert all(len(v) == 2 for v in loads.values()), loads
+        assert len(loads) == nk // 2
 
 
 def test_r2p_recipe_every_field_value_at_every_position():
