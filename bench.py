@@ -102,7 +102,7 @@ def cpu_baseline_block(target_seconds: float = 8.0):
 
 # ------------------------------------------------------------------ clocks
 class ClockSampler:
-    """SM clock, power and throttle reasons sampled every ~5 ms by NVML in a
+    """SM clock and throttle reasons sampled every ~2 ms by NVML (power every 8th) in a
     thread (nvidia-smi -lms 20 as the fallback).  start() before the warm-up,
     mark(True/False) around the timed region: summary() keeps the samples
     taken inside it (the recipe's clocks line), falling back to every sample
@@ -129,16 +129,20 @@ class ClockSampler:
             self.backend = "nvml"
 
             def run():
+                # clock + reasons every ~2 ms; power (a slower query) every 8th sample
                 mx = pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM)
+                pw, i = 0.0, 0
                 while not self.stop.is_set():
                     try:
+                        if i % 8 == 0:
+                            pw = pynvml.nvmlDeviceGetPowerUsage(h) / 1000.0
+                        i += 1
                         sm = pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM)
-                        pw = pynvml.nvmlDeviceGetPowerUsage(h) / 1000.0
                         rs = pynvml.nvmlDeviceGetCurrentClocksEventReasons(h)
                         self.rows.append((time.perf_counter(), float(sm), float(mx), pw, int(rs)))
                     except Exception:
                         pass
-                    time.sleep(0.005)
+                    time.sleep(0.002)
             self.th = threading.Thread(target=run, daemon=True)
             self.th.start()
         except Exception:
