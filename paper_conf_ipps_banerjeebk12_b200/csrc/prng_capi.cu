@@ -539,7 +539,9 @@ int prng_create(prng_t **out, const prng_graph_params *g, uint64_t walkers, uint
             // stage_rows works on walkers [0, Wv) of the handle; shift the base.
             const uint64_t saved_base = h->o.walker_base;
             h->o.walker_base = saved_base + w0;
-            stage_rows(h, 0, 2 + h->R0, cnt, tmp, cpitch);
+            // one burst per chunk (<= 134 MB): streaming stores, like the on-demand
+            // windows (cached stores left dirty lines that slowed the DMA to 17 GB/s)
+            stage_rows(h, 0, 2 + h->R0, cnt, tmp, cpitch, nullptr, true);
             h->o.walker_base = saved_base;
             join_copies(h, h->work_stream);
             gg::InitArgs a{};
