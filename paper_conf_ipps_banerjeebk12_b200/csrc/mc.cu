@@ -115,6 +115,13 @@ __global__ void mc_init_state(McState s, uint64_t n, uint32_t *iota) {
     s.alive[i] = 0;
     s.launched[i] = 0;
     s.w[i] = 0;
+    // geometry of a thread without a photon is never used before launch sets
+    // it, but the epoch kernel loads it unconditionally: define it (initcheck)
+    s.x[i] = s.y[i] = s.z[i] = 0.0;
+    s.ux[i] = s.uy[i] = 0.0;
+    s.uz[i] = 1.0;
+    s.sleft[i] = 0.0;
+    s.layer[i] = 0;
     s.busy[i] = 1;
     iota[i] = (uint32_t)i;
 }
