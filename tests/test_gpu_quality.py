@@ -87,3 +87,20 @@ def test_battery_negative_control_l1_on_gpu():
     z = gen(1, n_draws=1024, W=1 << 12).cpu().numpy()
     res = B.run(np.ascontiguousarray(z.T).reshape(-1).view(np.uint32))
     assert sum(v < 1e-10 for v in res.values()) >= 3, res
+
+
+def test_nist_sp800_22_on_gpu_output():
+    """NIST SP 800-22 subset (tests/nist.py) on 16 sequences of 10^6 bits of
+    C2 output computed on the GPU, bulk and walker-major order.  NIST's
+    acceptance rule: the proportion of sequences passing at alpha = 0.01 must
+    exceed 0.99 - 3 sqrt(0.99 * 0.01 / k); for k = 16 at most one failure is
+    expected, allow three (P(>= 4 of 16) ~ 2e-6 per test)."""
+    import nist as N
+    z = gen(64, n_draws=16, W=1 << 16).cpu().numpy()  # 2^20 labels = 2^26 bits
+    for name, arr in (("bulk", z), ("walker-major", z.T.copy())):
+        bits = N.bits_of_words(np.ascontiguousarray(arr).reshape(-1).view(np.uint32))
+        fails = {}
+        for s in range(16):
+            for k, v in N.run(bits[s * 1_000_000:(s + 1) * 1_000_000]).items():
+                fails[k] = fails.get(k, 0) + (v < 0.01)
+        assert max(fails.values()) <= 3, (name, fails)
