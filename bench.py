@@ -833,14 +833,18 @@ def run_reference(args, world):
         dt = time.perf_counter() - t
     labels = args.steps * cores * walkers * draws
     value = labels / dt / 1e9
-    sample = (f"per step {cores * walkers * draws} labels of the C2 workload: {cores} "
-              f"single-threaded oracle processes x {walkers} walkers x {draws} draws")
+    wl = "C5" if args.workload == "c5" else "C2"
+    sample = (f"per step {cores * walkers * draws} labels of the {wl} workload (m=2^32, "
+              f"l=l0=64): {cores} single-threaded oracle processes x {walkers} walkers x "
+              f"{draws} draws")
     line = {
         "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt * 1e3 / args.steps,
-        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64",
+        "higher_is_better": True, "scaling": "strong" if args.workload == "c5" else "weak",
+        "vs_baseline": None, "dtype": "u64",
         "data": "synthetic (SplitMix64 counter-hash seed bits, reading R9)",
-        "config": {"workload": WORKLOAD, "number": "one 64-bit vertex label (the paper's unit)",
+        "config": {"workload": C5_WORKLOAD if args.workload == "c5" else WORKLOAD,
+                   "number": "one 64-bit vertex label (the paper's unit)",
                    "parallelism": "host cores"},
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle",
                          "sample": sample},
