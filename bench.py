@@ -89,11 +89,14 @@ def cpu_baseline_block(target_seconds: float = 8.0):
     # calibrate on one core, then size the sample to ~target_seconds wall
     r1, _, _ = oracle_rate(1, 64, 64)
     per_core = max(64 * 16, int(r1 * target_seconds))
+    # the plain oracle on one core, then on all cores
+    r1, l1, t1 = oracle_rate(1, max(1, int(r1 * 2.0) // 64), 64)
     draws = 64
     walkers = max(1, per_core // draws)
     rate, labels, dt = oracle_rate(cores, walkers, draws)
     return {
         "value": rate / 1e9, "unit": UNIT, "cores": cores, "kind": "oracle",
+        "value_1core": r1 / 1e9, "sample_1core": f"{l1} labels on one core, {t1:.1f} s",
         "sample": (f"{labels} labels of the C2 workload (m=2^32, l=l0=64, seed 0x5EED0002): "
                    f"{cores} single-threaded oracle processes x {walkers} walkers x draws 0..{draws-1} "
                    f"(Alg.1 burn-in included), {dt:.1f} s wall"),
