@@ -225,6 +225,16 @@ def committed_traffic():
         return None
 
 
+def measured_int_peak():
+    """Interleaved LOP3/IMAD lane-op rate measured by tools/int_peak.cu on this
+    pool's B200 (profiles/r01_measured_box.json), T ops/s, or None."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "r01_measured_box.json")) as f:
+            return float(json.load(f)["int_issue"]["lop3_imad_1to1_tops"])
+    except (OSError, KeyError, ValueError):
+        return None
+
+
 def measured_peaks():
     try:
         with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
@@ -312,6 +322,9 @@ def run_ours(args, rank, world, local_rank):
         "kernel_ms_median_min_max": [statistics.median(step_ms), min(step_ms), max(step_ms)],
         "peak_basis": (f"{props.multi_processor_count} SMs x 128 int lanes/clk (ALU 64 + FMA 64, "
                        f"issue 4x32) x {sm_max:.0f} MHz (MEASURED_PEAKS sm_max_mhz)"),
+        "peak_measured": measured_int_peak(),
+        "peak_measured_note": ("tools/int_peak.cu, LOP3/IMAD interleaved 1:1 "
+                               "(profiles/r01_measured_box.json); frac uses the derived peak"),
         "hbm_gbs_achieved": LABELS_PER_STEP * (BITS_BYTES_PER_LABEL + 8) / (kern_ms / 1e3) / 1e9,
         "hbm_gbs_peak": peaks.get("hbm_gbs"),
     }
