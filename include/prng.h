@@ -64,7 +64,15 @@ enum {
                                "the LCG present in the glibc library"); word k of walker t
                                = low 16 bits of outputs 2k, 2k+1 of the stream seeded with
                                low32(seed ^ (t+1)*0x9E3779B97F4A7C15) */
-    PRNG_BITS_CALLBACK = 2  /* user callback supplies the words (tests, fault injection) */
+    PRNG_BITS_CALLBACK = 2, /* user callback supplies the words (tests, fault injection) */
+    PRNG_BITS_GGCPU = 3     /* the generator itself run by the host feed threads (§IV-A
+                               "Our generator, working on a multicore CPU can be used in
+                               the place of rand()"; reading R23): word k of walker t = x
+                               (k even) or y (k odd) of label (k mod 64)/2 of walker t of
+                               the m = 2^32, l = l0 = 64 generator seeded with
+                               mix64(seed ^ (k/64 + 1) * 0xD1B54A32D192ED03), whose own
+                               seed bits are the SplitMix64 stream (R9).  Costs one host
+                               walk of 64 steps per two words. */
 };
 
 /* Graph parameters (§III-A/B).  Paper defaults in comments. */

@@ -70,6 +70,7 @@ def lib():
                 "or_sigma_inv": (None, [u64, ctypes.c_int, u64, u64, P, P]),
                 "or_rand_r": (ctypes.c_int32, [P]),
                 "or_stream_word32_randr": (u32, [u64, u64, u64]),
+                "or_stream_word32_ggcpu": (u32, [u64, u64, u64]),
                 "or_set_bit_source": (None, [ctypes.c_int]),
                 "or_walk_bipartite": (None, [u64, P, P, P, u32, u64]),
                 "or_walker_init_v": (ctypes.c_int, [u64, u32, u32, u64, u64, P, P]),

@@ -63,6 +63,18 @@ void feed_randr_rows(uint64_t seed, uint64_t tg0, uint64_t count, uint64_t k0, u
 void feed_randr_rows_ids(uint64_t seed, uint64_t base, const uint32_t *ids, uint64_t count,
                          uint64_t k0, uint32_t nrows, uint32_t *out, uint64_t pitch);
 
+// The generator on the host as the FEED (bit_source 3, reading R23; see
+// feed.cpp).  Per walker of the handle (index = global id - t0): the host
+// walk's state (x, y) after label nxt - 1 of block blk (nxt = 0: nothing
+// walked yet).  Column i is global walker base + l0 + i, or base + ids[i].
+struct GgCpuCache {
+    uint32_t *x, *y, *blk, *nxt;
+    uint64_t t0;
+};
+void feed_ggcpu_rows(uint64_t seed, uint64_t base, uint64_t l0, const uint32_t *ids,
+                     uint64_t count, uint64_t k0, uint32_t nrows, uint32_t *out, uint64_t pitch,
+                     GgCpuCache &cache);
+
 // Library-owned stream-ordered scratch pool of the current device (listrank.cu):
 // keeps its memory between calls; nullptr on CUDA failure.
 cudaMemPool_t scratch_pool();

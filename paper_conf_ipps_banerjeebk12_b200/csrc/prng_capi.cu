@@ -127,6 +127,10 @@ struct prng_s {
     cudaEvent_t chunk_done[kMaxChunks] = {};
     int chunk_next = 0;
 
+    // host walks of the generator-as-FEED bit source (PRNG_BITS_GGCPU, R23)
+    std::vector<uint32_t> gg_x, gg_y, gg_blk, gg_nxt;
+    uint64_t gg_t0 = 0;  // global id of cache slot 0 (the handle's walker_base)
+
     // resident (prefetched) window: draws [res_J, res_J + res_D) of all walkers
     uint32_t *res_bits = nullptr;
     size_t res_cap = 0;
@@ -202,6 +206,13 @@ void feed_chunk(prng_s *h, uint64_t wa, uint64_t wb, uint64_t k0, uint32_t nrows
         uint64_t per = round_up((cw + nt - 1) / nt, 16);
         uint64_t lo = std::min<uint64_t>(cw, per * ti), hi = std::min<uint64_t>(cw, lo + per);
         if (lo >= hi) return;
+        if (h->o.bit_source == PRNG_BITS_GGCPU) {
+            gg::GgCpuCache c{h->gg_x.data(), h->gg_y.data(), h->gg_blk.data(), h->gg_nxt.data(),
+                             h->gg_t0};
+            gg::feed_ggcpu_rows(h->seed, h->o.walker_base, wa + lo, ids ? ids + wa + lo : nullptr,
+                                hi - lo, k0, nrows, buf + lo, bpitch, c);
+            return;
+        }
         if (ids) {
             if (h->o.bit_source == PRNG_BITS_RANDR) {
                 gg::feed_randr_rows_ids(h->seed, h->o.walker_base, ids + wa + lo, hi - lo, k0,
@@ -481,7 +492,7 @@ int prng_create(prng_t **out, const prng_graph_params *g, uint64_t walkers, uint
     if (g->walk_len < 1 || g->walk_len > 4096 || g->burnin_len > 4096) return PRNG_E_INVALID;
     if (walkers + o.walker_base > (1ull << 24)) return PRNG_E_INVALID;
     if (o.bit_source != PRNG_BITS_SPLITMIX && o.bit_source != PRNG_BITS_RANDR &&
-        o.bit_source != PRNG_BITS_CALLBACK)
+        o.bit_source != PRNG_BITS_CALLBACK && o.bit_source != PRNG_BITS_GGCPU)
         return PRNG_E_INVALID;
     if (o.bit_source == PRNG_BITS_CALLBACK && !o.bits_fn) return PRNG_E_INVALID;
     if (o.epoch_draws == 0) o.epoch_draws = 16;
@@ -495,6 +506,15 @@ int prng_create(prng_t **out, const prng_graph_params *g, uint64_t walkers, uint
     h->o = o;
     h->W = walkers;
     h->seed = seed;
+    if (o.bit_source == PRNG_BITS_GGCPU) {
+        try {
+            for (auto *v : {&h->gg_x, &h->gg_y, &h->gg_blk, &h->gg_nxt}) v->assign(walkers, 0u);
+            h->gg_t0 = o.walker_base;
+        } catch (const std::bad_alloc &) {
+            delete h;
+            return PRNG_E_NOMEM;
+        }
+    }
     h->R = words_per_walk(g->walk_len);
     h->R0 = words_per_walk(g->burnin_len);
     h->pow2 = pow2 ? 1 : 0;

@@ -137,3 +137,81 @@ def test_randr_feed_jump_ahead_matches_plain_replay(randr_feed, k0, rows):
     for i, t in enumerate(ids):
         for r in range(rows):
             assert got[r, i] == O.lib().or_stream_word32_randr(seed, 100 + int(t), k0 + r)
+
+
+# ------------------------------------- f3: the generator itself as the FEED
+GGCPU_SHIM = r'''
+#include <cstdint>
+#include "gg_internal.h"
+extern "C" void run(uint64_t seed, uint64_t base, uint64_t l0, const uint32_t *ids, uint64_t n,
+                    uint64_t k0, uint32_t r, uint32_t *o, uint64_t p, uint32_t *cx, uint32_t *cy,
+                    uint32_t *cb, uint32_t *cn, uint64_t t0) {
+    gg::GgCpuCache c{cx, cy, cb, cn, t0};
+    gg::feed_ggcpu_rows(seed, base, l0, ids, n, k0, r, o, p, c);
+}
+'''
+
+
+@pytest.fixture(scope="module")
+def ggcpu_feed(tmp_path_factory):
+    d = tmp_path_factory.mktemp("ggcpu")
+    src, so = d / "shim.cpp", d / "shim.so"
+    src.write_text(GGCPU_SHIM)
+    feed_src = os.path.join(ROOT, "paper_conf_ipps_banerjeebk12_b200", "csrc", "feed.cpp")
+    subprocess.check_call(["g++", "-O2", "-std=c++17", "-shared", "-fPIC", "-I",
+                           os.path.join(ROOT, "paper_conf_ipps_banerjeebk12_b200", "csrc"),
+                           "-I", "/usr/local/cuda/include", "-o", str(so), str(src), feed_src])
+    return ctypes.CDLL(str(so))
+
+
+class _GgCache:
+    def __init__(self, n):
+        self.a = [np.zeros(n, np.uint32) for _ in range(4)]
+
+    def args(self):
+        return [ctypes.c_void_p(a.ctypes.data) for a in self.a]
+
+
+def _ggcpu_rows(feed, cache, seed, base, l0, n, k0, rows, ids=None, t0=0):
+    pitch = max(n, 1)
+    buf = np.zeros(rows * pitch, np.uint32)
+    feed.run(ctypes.c_uint64(seed), ctypes.c_uint64(base), ctypes.c_uint64(l0),
+             ctypes.c_void_p(None if ids is None else ids.ctypes.data), ctypes.c_uint64(n),
+             ctypes.c_uint64(k0), ctypes.c_uint32(rows), ctypes.c_void_p(buf.ctypes.data),
+             ctypes.c_uint64(pitch), *cache.args(), ctypes.c_uint64(t0))
+    return buf.reshape(rows, pitch)[:, :n]
+
+
+def test_ggcpu_oracle_is_the_generator_reseeded_per_block():
+    # R23 restated through the oracle's own Alg.1/Alg.2 (pinned elsewhere):
+    # word k = x or y of label (k mod 64)/2 of walker t under seed_b
+    seed, t = 0x5EED0001, 12
+    for k in (0, 1, 7, 62, 63, 64, 65, 200):
+        b, j = k // 64, (k % 64) // 2
+        sb = O.lib().or_mix64(seed ^ (((b + 1) * 0xD1B54A32D192ED03) & (2**64 - 1)))
+        lab = int(O.walker_draws(1 << 32, 64, 64, sb, t, 0, j + 1)[j])
+        want = lab & 0xFFFFFFFF if k % 2 == 0 else lab >> 32
+        assert O.lib().or_stream_word32_ggcpu(seed, t, k) == want
+
+
+def test_ggcpu_feed_matches_oracle_sequential_random_and_lists(ggcpu_feed):
+    seed, base, W = 0x5EED0007, 1000, 40
+    cache = _GgCache(W)
+    want = lambda t, k: O.lib().or_stream_word32_ggcpu(seed, base + t, k)  # noqa: E731
+    # sequential row ranges (the bulk feed), crossing the 64-word block edges
+    for k0, rows in ((0, 8), (8, 30), (38, 40), (78, 60)):
+        got = _ggcpu_rows(ggcpu_feed, cache, seed, base, 0, W, k0, rows, t0=base)
+        for t in (0, 5, W - 1):
+            assert [int(v) for v in got[:, t]] == [want(t, k0 + r) for r in range(rows)]
+    # backwards and odd starts (restart from the block's beginning)
+    for k0, rows in ((3, 5), (129, 2), (64, 1), (65, 1)):
+        got = _ggcpu_rows(ggcpu_feed, cache, seed, base, 0, W, k0, rows, t0=base)
+        for t in (1, 17):
+            assert [int(v) for v in got[:, t]] == [want(t, k0 + r) for r in range(rows)]
+    # a sub-range of walkers (l0) and an explicit walker list
+    got = _ggcpu_rows(ggcpu_feed, cache, seed, base, 20, 10, 140, 6, t0=base)
+    assert [int(v) for v in got[:, 3]] == [want(23, 140 + r) for r in range(6)]
+    ids = np.array([39, 0, 21, 7], np.uint32)
+    got = _ggcpu_rows(ggcpu_feed, cache, seed, base, 0, 4, 146, 6, ids=ids, t0=base)
+    for i, t in enumerate(ids):
+        assert [int(v) for v in got[:, i]] == [want(int(t), 146 + r) for r in range(6)]

@@ -302,3 +302,35 @@ def test_randr_bit_source_parity(torch_cuda):
     with O.bit_source(1):
         want = O.bulk(256, 64, 64, seed, W, 0, W * 4 + 3)
     assert np.array_equal(as_u64(o), want)
+
+
+def test_ggcpu_bit_source_parity(torch_cuda):
+    # f3: the generator itself, run by the host feed threads, supplies the
+    # seed bits (bit_source 3, R23): streamed and prefetched bulk fills across
+    # 64-word block edges, an on-demand epoch and an epoch over a walker list
+    torch = torch_cuda
+    W, seed = 300, 0x5EED0003
+    g = G(walkers=W, seed=seed, bit_source=3, epoch_draws=5)
+    n = W * 23 + 7  # draws 0..23: words 8..151, blocks 0..2
+    o = torch.empty(n, dtype=torch.int64, device="cuda")
+    g.fill(o[: W * 11 + 5])
+    g.fill(o[W * 11 + 5:])
+    with O.bit_source(3):
+        want = O.bulk(M32, 64, 64, seed, W, 0, n)
+    assert np.array_equal(as_u64(o), want)
+    g.close()
+    g = G(walkers=W, seed=seed, bit_source=3)
+    g.prefetch(12)
+    o2 = torch.empty(W * 12, dtype=torch.int64, device="cuda")
+    g.fill(o2)
+    assert np.array_equal(as_u64(o2), want[: W * 12])
+    # on demand: the next epoch starts at draw 12 (R10)
+    g.epoch_begin(W, 3)
+    od = torch.empty(W * 3, dtype=torch.int64, device="cuda")
+    g.consume(W, uniform=3, out=od)
+    g.epoch_end()
+    got = as_u64(od).reshape(W, 3) if od.numel() else None
+    with O.bit_source(3):
+        for t in (0, 1, 150, W - 1):
+            assert np.array_equal(got[t], O.walker_draws(M32, 64, 64, seed, t, 12, 3)), t
+    g.close()
