@@ -15,11 +15,11 @@ import ctypes
 from contextlib import contextmanager
 
 from . import _lib
-from ._lib import (PRNG_BITS_CALLBACK, PRNG_BITS_SPLITMIX, PRNG_FMT_U32, PRNG_FMT_U64,
-                   PrngError, check)
+from ._lib import (PRNG_BITS_CALLBACK, PRNG_BITS_GGCPU, PRNG_BITS_RANDR, PRNG_BITS_SPLITMIX,
+                   PRNG_FMT_U32, PRNG_FMT_U64, PrngError, check)
 
 __all__ = ["Generator", "PrngError", "PRNG_FMT_U32", "PRNG_FMT_U64", "PRNG_BITS_SPLITMIX",
-           "PRNG_BITS_CALLBACK", "params", "options"]
+           "PRNG_BITS_RANDR", "PRNG_BITS_CALLBACK", "PRNG_BITS_GGCPU", "params", "options"]
 
 
 def params(m: int = 1 << 32, walk_len: int = 64, burnin_len: int = 64, degree: int = 7,

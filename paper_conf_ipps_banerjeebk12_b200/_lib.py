@@ -36,6 +36,7 @@ PRNG_FMT_U32 = 1
 PRNG_BITS_SPLITMIX = 0
 PRNG_BITS_RANDR = 1
 PRNG_BITS_CALLBACK = 2
+PRNG_BITS_GGCPU = 3
 
 PRNG_BITS_FN = ctypes.CFUNCTYPE(None, vp, u64, u64, u64, u32, ctypes.POINTER(ctypes.c_uint32), u64)
 
