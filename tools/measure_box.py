@@ -36,6 +36,9 @@ def ev_time(fn, reps=5):
 def main():
     res = {}
     exe = os.path.join(ROOT, "tools", "int_peak")
+    if not os.path.exists(exe):
+        subprocess.run(["nvcc", "-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-o", exe,
+                        exe + ".cu"], check=False)
     if os.path.exists(exe):
         out = subprocess.run([exe], capture_output=True, text=True, timeout=300)
         res["int_issue"] = json.loads(out.stdout.strip().splitlines()[-1])
