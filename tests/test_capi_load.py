@@ -70,6 +70,13 @@ def test_host_only_calls(lib):
     p.m = 1 << 32
     assert lib.prng_create(ctypes.byref(h), ctypes.byref(p), 0, 0, None) == lib.PRNG_E_INVALID
     assert lib.prng_create(ctypes.byref(h), ctypes.byref(p), (1 << 24) + 1, 0, None) == lib.PRNG_E_INVALID
+    o = lib.prng_options()
+    assert lib.prng_default_options(ctypes.byref(o)) == 0
+    o.bit_source = 4  # PRNG_BITS_* ends at PRNG_BITS_GGCPU = 3
+    assert lib.prng_create(ctypes.byref(h), ctypes.byref(p), 16, 0, ctypes.byref(o)) == lib.PRNG_E_INVALID
+    o.bit_source = 2  # callback without a function
+    assert lib.prng_create(ctypes.byref(h), ctypes.byref(p), 16, 0, ctypes.byref(o)) == lib.PRNG_E_INVALID
+    assert not h.value  # nothing was created
     assert lib.prng_destroy(None) == 0
     assert lib.prng_fill(None, None, 1, 0, None) == lib.PRNG_E_INVALID
 
