@@ -405,7 +405,8 @@ def run_ours(args, rank, world, local_rank):
     if not args.no_e2e:
         e2e_steps = max(1, min(args.steps, args.e2e_steps))
         g = Generator(walkers=W_PER_GPU, seed=SEED, walker_base=rank * W_PER_GPU,
-                      device=local_rank, epoch_draws=16, host_threads=feed_threads)
+                      device=local_rank, epoch_draws=int(os.environ.get("GG_E2E_D", "16")),
+                      host_threads=feed_threads)
         host = torch.empty(U32_PER_STEP, dtype=torch.int32).pin_memory()
         g.fill_host(host, n=W_PER_GPU * 2 * 16)  # warm (allocations, feed threads)
         g.mark()
