@@ -206,3 +206,52 @@ def test_on_demand_bulk_on_demand_keeps_one_sequence():
                 assert int(b[g_idx]) == ow.draw(j), (t, j)
         assert int(c[t]) == ow.draw(J1), t
     assert g.check() == 0
+
+
+def test_full_size_uniform_and_mc_shaped_sampled_parity():
+    """The on-demand consumers in bench.py's launch configuration, at full
+    size: 2^20 threads x S = 100 prng_next per thread (Fig.4's batch; the
+    bench's uniform_S100 line, xor_out and out both checked) and the
+    MC-shaped demand (geometric counts, mean 200, cap 600, walker t's draws
+    at offsets[t]); sampled walkers against the oracle."""
+    import math
+
+    import torch
+    from paper_conf_ipps_banerjeebk12_b200 import Generator
+    W, S, seed = 1 << 20, 100, 0x5EED0003
+    g = Generator(walkers=W, seed=seed)
+    g.epoch_begin(W, S)
+    o = torch.empty(W * S, dtype=torch.int64, device="cuda")
+    xo = torch.empty(W, dtype=torch.int64, device="cuda")
+    g.consume(W, uniform=S, out=o)
+    g.epoch_end()
+    g.epoch_begin(W, S)
+    g.consume(W, uniform=S, xor_out=xo)
+    g.epoch_end()
+    assert g.check() == 0
+    z = o.view(W, S)
+    x = xo.cpu().numpy().view(np.uint64)
+    for t in list(range(0, W, 65521)) + [W - 1]:
+        want = O.walker_draws(M32, 64, 64, seed, t, 0, 2 * S)
+        assert np.array_equal(z[t].cpu().numpy().view(np.uint64), want[:S]), t
+        assert int(x[t]) == int(np.bitwise_xor.reduce(want[S:])), t
+    g.close()
+    del o, z
+    # MC-shaped counts, outputs packed at per-walker offsets
+    gen = torch.Generator(device="cpu").manual_seed(7)
+    u = torch.rand(W, generator=gen, dtype=torch.float64)
+    c = torch.clamp(torch.ceil(torch.log1p(-u) / math.log1p(-1 / 200)), 1, 600).to(torch.int32)
+    off = torch.zeros(W, dtype=torch.int64)
+    off[1:] = torch.cumsum(c.to(torch.int64), 0)[:-1]
+    total = int(c.sum().item())
+    g = Generator(walkers=W, seed=seed + 1)
+    g.epoch_begin(W, 600)
+    o = torch.empty(total, dtype=torch.int64, device="cuda")
+    g.consume(W, counts=c.cuda(), out=o, offsets=off.cuda())
+    g.epoch_end()
+    oc = o.cpu().numpy().view(np.uint64)
+    for t in list(range(3, W, 131071)) + [W - 1]:
+        n = int(c[t])
+        want = O.walker_draws(M32, 64, 64, seed + 1, t, 0, n)
+        assert np.array_equal(oc[int(off[t]):int(off[t]) + n], want), t
+    g.close()
