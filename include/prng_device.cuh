@@ -427,7 +427,7 @@ __device__ __forceinline__ uint64_t prng_next(prng_state *st, const prng_view *v
  * first walk, so a consumer that needs several numbers per iteration (the
  * Monte Carlo consumer takes three) waits for memory once, not K times.
  * Same numbers, same order, same overrun rule as K calls of prng_next. */
-template <int K>
+template <int K, bool ROLL = false>
 __device__ __forceinline__ void prng_next_n(prng_state *st, const prng_view *v, uint64_t (&out)[K])
 {
     if (!(v->l == 64u && v->pow2 && v->variant == 0) || st->used + K > v->D ||
@@ -444,10 +444,33 @@ __device__ __forceinline__ void prng_next_n(prng_state *st, const prng_view *v, 
         for (int r = 0; r < 6; r++) w[k][r] = __ldg(rec + (uint64_t)r * v->pitch);
     }
     uint32_t x = st->x, y = st->y;
+    if (!ROLL) {
 #pragma unroll
+        for (int k = 0; k < K; k++) {
+            gg_walk64_r2p(w[k], x, y);
+            out[k] = gg_label(x, y, v->m, v->log2m, true);
+        }
+        st->x = x;
+        st->y = y;
+        st->used += K;
+        return;
+    }
+    /* ROLL: one copy of the walk in a rolled loop (the records rotate through
+     * w[0] with register moves), for consumers whose hot loop would not fit
+     * the instruction cache with K unrolled walks (Monte Carlo: ncu "no
+     * instruction" stalls; 28.5 -> 30.9 G draws/s in-kernel).  Kernels with a
+     * small body keep the unrolled form (gg_consume: 65.7 vs 61.2 G/s rolled). */
+#pragma unroll 1
     for (int k = 0; k < K; k++) {
-        gg_walk64_r2p(w[k], x, y);
-        out[k] = gg_label(x, y, v->m, v->log2m, true);
+        gg_walk64_r2p(w[0], x, y);
+        uint64_t lab = gg_label(x, y, v->m, v->log2m, true);
+#pragma unroll
+        for (int q = 0; q < K; q++)
+            if (q == k) out[q] = lab;
+#pragma unroll
+        for (int q = 0; q + 1 < K; q++)
+#pragma unroll
+            for (int r = 0; r < 6; r++) w[q][r] = w[q + 1][r];
     }
     st->x = x;
     st->y = y;

@@ -161,7 +161,7 @@ __global__ void __launch_bounds__(128, MINB) mc_epoch(prng_view v, McParams P, M
             if (!alive && launched == budget) break;
             // three draws at a convergent point (R22), their loads in flight together
             uint64_t d3[3];
-            prng_next_n<3>(&st, &v, d3);
+            prng_next_n<3, true>(&st, &v, d3);
             const uint64_t la = d3[0], lb = d3[1], lc = d3[2];
             draws += 3;
             if (!alive) {
