@@ -161,3 +161,13 @@ def test_negative_controls_fail():
     rng = np.random.default_rng(9)
     biased = (rng.random(1_000_000) < 0.505).astype(np.uint8)
     assert "frequency" in _run_pass(biased)
+
+
+def test_host_generator_feed_words_pass():
+    # R23 (bit_source 3): the words the host generator feeds (x, y halves of
+    # its labels, reseeded per 64-word block) are themselves random-looking
+    seed, n_words = 0x5EED0008, 31250
+    f = O.lib().or_stream_word32_ggcpu
+    w = np.array([f(seed, t, k) for t in range(250) for k in range(125)], dtype=np.uint32)
+    assert w.size == n_words
+    assert not _run_pass(N.bits_of_words(w))
