@@ -3,6 +3,9 @@
 // staging pipeline (FEED -> TRANSFER, §IV-A Fig.4), resident and
 // streamed bit windows, on-demand epochs (R10), checkpoints.
 #include <algorithm>
+#include <cctype>
+#include <sched.h>
+#include <pthread.h>
 #include <chrono>
 #include <condition_variable>
 #include <cstdint>
@@ -26,8 +29,19 @@ namespace {
 // ------------------------------------------------------------ thread pool
 class ThreadPool {
   public:
-    explicit ThreadPool(unsigned n) : n_(n ? n : 1) {
-        for (unsigned i = 1; i < n_; i++) workers_.emplace_back([this, i] { loop(i); });
+    // cpus: if non-empty, worker i (i >= 1; index 0 is the calling thread,
+    // never pinned) is pinned to cpus[i % cpus.size()].
+    explicit ThreadPool(unsigned n, std::vector<int> cpus = {}) : n_(n ? n : 1) {
+        for (unsigned i = 1; i < n_; i++)
+            workers_.emplace_back([this, i, cpus] {
+                if (!cpus.empty()) {
+                    cpu_set_t set;
+                    CPU_ZERO(&set);
+                    CPU_SET(cpus[i % cpus.size()], &set);
+                    pthread_setaffinity_np(pthread_self(), sizeof(set), &set);
+                }
+                loop(i);
+            });
     }
     ~ThreadPool() {
         {
@@ -85,6 +99,39 @@ class ThreadPool {
     uint64_t gen_ = 0;
     bool stop_ = false;
 };
+
+// CPUs of the GPU's own NUMA node (feed threads next to
+// the GPU's PCIe root): /sys/bus/pci/devices/<bus id>/local_cpulist,
+// intersected with the process's allowed CPUs; empty if unknown.
+std::vector<int> gpu_local_cpus(int device) {
+    std::vector<int> out;
+    char bus[32] = {0};
+    if (cudaDeviceGetPCIBusId(bus, sizeof(bus), device) != cudaSuccess) return out;
+    for (char *c = bus; *c; c++) *c = (char)tolower(*c);
+    char path[128];
+    snprintf(path, sizeof(path), "/sys/bus/pci/devices/%s/local_cpulist", bus);
+    FILE *f = fopen(path, "r");
+    if (!f) return out;
+    char line[1024] = {0};
+    const bool ok = fgets(line, sizeof(line), f) != nullptr;
+    fclose(f);
+    if (!ok) return out;
+    cpu_set_t allowed;
+    CPU_ZERO(&allowed);
+    if (sched_getaffinity(0, sizeof(allowed), &allowed) != 0) return out;
+    for (char *tok = strtok(line, ",\n"); tok; tok = strtok(nullptr, ",\n")) {
+        int a = -1, b = -1;
+        if (sscanf(tok, "%d-%d", &a, &b) == 2) {
+        } else if (sscanf(tok, "%d", &a) == 1) {
+            b = a;
+        } else {
+            continue;
+        }
+        for (int c = a; c <= b && c < CPU_SETSIZE; c++)
+            if (c >= 0 && CPU_ISSET(c, &allowed)) out.push_back(c);
+    }
+    return out;
+}
 
 inline uint32_t words_per_walk(uint32_t nsteps) { return (3u * nsteps + 31u) / 32u; }
 inline uint64_t round_up(uint64_t v, uint64_t a) { return (v + a - 1) / a * a; }
@@ -526,7 +573,19 @@ int prng_create(prng_t **out, const prng_graph_params *g, uint64_t walkers, uint
         CK(cudaDeviceGetAttribute(&h->sm_count, cudaDevAttrMultiProcessorCount, o.device));
         unsigned nt = o.host_threads ? o.host_threads : std::thread::hardware_concurrency();
         if (nt == 0) nt = 1;
-        h->pool = new ThreadPool(nt);
+        // A/B hook GG_FEED_PIN=1: pin the feed threads to the GPU's NUMA-local
+        // CPUs, rank r of a node (walker_base = r * walkers) on its own slice
+        static const bool pin = getenv("GG_FEED_PIN") && atoi(getenv("GG_FEED_PIN")) == 1;
+        std::vector<int> cpus;
+        if (pin) {
+            std::vector<int> local = gpu_local_cpus(o.device);
+            if (!local.empty()) {
+                const size_t rank = (size_t)(o.walker_base / walkers);
+                for (unsigned i = 0; i < nt; i++)
+                    cpus.push_back(local[(rank * nt + i) % local.size()]);
+            }
+        }
+        h->pool = new ThreadPool(nt, cpus);
         CK(cudaStreamCreateWithFlags(&h->copy_stream, cudaStreamNonBlocking));
         CK(cudaStreamCreateWithFlags(&h->d2h_stream, cudaStreamNonBlocking));
         CK(cudaStreamCreateWithFlags(&h->work_stream, cudaStreamNonBlocking));
