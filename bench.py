@@ -235,6 +235,23 @@ def measured_int_peak():
         return None
 
 
+def pcie_bound(h2d_bytes: float, d2h_bytes: float, labels: float):
+    """Upper bound on e2e labels/s from the measured PCIe rates of this pool's
+    box (profiles/r01_measured_box.json): the D2H bytes share the link with
+    as many H2D bytes at the bidirectional rate, the rest of the H2D bytes
+    run at the one-way rate."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "r01_measured_box.json")) as f:
+            mb = json.load(f)
+        h2d, bi = float(mb["h2d_pinned_gbs"]) * 1e9, float(mb["h2d_plus_d2h_gbs"]) * 1e9
+    except (OSError, KeyError, ValueError):
+        return None
+    both = min(h2d_bytes, d2h_bytes)
+    t = 2 * both / bi + (h2d_bytes - both) / h2d + (d2h_bytes - both) / h2d
+    return {"kind": "pcie", "h2d_gbs": h2d / 1e9, "bidir_gbs": bi / 1e9,
+            "max_value": labels / t / 1e9, "source": "profiles/r01_measured_box.json"}
+
+
 def measured_peaks():
     try:
         with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
@@ -429,6 +446,11 @@ def run_ours(args, rank, world, local_rank):
             "api": "prng_fill_host (host FEED threads -> pinned -> H2D -> walk -> D2H to pinned)",
             "host_threads": feed_threads,
         }
+        b = pcie_bound(res["e2e"]["h2d_bytes_per_step"], res["e2e"]["d2h_bytes_per_step"],
+                       LABELS_PER_STEP)
+        if b:
+            b["frac"] = res["e2e"]["value"] / world / b["max_value"]
+            res["e2e"]["bound"] = b
         g.close()
     return res
 
@@ -555,6 +577,10 @@ def run_c5(args, rank, world, local_rank):
                "feed_s": s1["feed_seconds"] - s0["feed_seconds"], "host_threads": feed_threads,
                "api": "prng_fill into the reused device buffer, host FEED -> pinned -> H2D "
                       "overlapped with the walk; last label read back"}
+        b = pcie_bound(e2e["h2d_bytes_per_step"], 8, C5_LABELS / world)
+        if b:
+            b["frac"] = e2e["value"] / world / b["max_value"]
+            e2e["bound"] = b
     return {"value": value, "ms": ms, "roofline": roofline, "clocks": clk.summary(),
             "launches": launches, "e2e": e2e, "walkers_per_gpu": Wr, "chunks_per_gpu": chunks,
             "draws_per_chunk": draws_per_chunk}
