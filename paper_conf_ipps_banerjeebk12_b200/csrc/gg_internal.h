@@ -6,6 +6,8 @@
 
 #include <cuda_runtime.h>
 
+struct prng_s;
+
 namespace gg {
 
 // Alg.1 (§III-B) for walkers [w0, w0 + count): start vertex from stream
@@ -74,6 +76,10 @@ struct GgCpuCache {
 void feed_ggcpu_rows(uint64_t seed, uint64_t base, uint64_t l0, const uint32_t *ids,
                      uint64_t count, uint64_t k0, uint32_t nrows, uint32_t *out, uint64_t pitch,
                      GgCpuCache &cache);
+
+// Stage walkers [0, hi) of the next on-demand epoch's window (one draw, row
+// pitch `pitch`) ahead of prng_epoch_begin (prng_capi.cu); list ranking.
+int epoch_prefeed(prng_s *h, uint64_t hi, uint64_t pitch);
 
 // Library-owned stream-ordered scratch pool of the current device (listrank.cu):
 // keeps its memory between calls; nullptr on CUDA failure.

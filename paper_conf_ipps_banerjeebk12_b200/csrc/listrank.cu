@@ -16,6 +16,7 @@
 // Phase III: re-insert removed nodes in reverse round order,
 //   rank(u) = rank(pred at removal) + distance at removal.
 #include <chrono>
+#include <cmath>
 #include <cstdint>
 #include <cstdio>
 #include <cstdlib>
@@ -329,6 +330,18 @@ extern "C" int gg_list_rank(prng_t *h, int64_t n, const int32_t *succ, const int
             sync_t("decide+splice", tq);
             LCK(cub::DevicePartition::Flagged(tmp, tmp_bytes, act, keep, act2, d_num, (int)A, s));
             sync_t("partition", tq);
+            // While this round's kernels run, stage the next round's bits for the
+            // slots that certainly stay active: an interior node is removed with
+            // probability 1/8 (Alg.3 l.8-9), so the survivors are ~7/8 A with a
+            // standard deviation of sqrt(7A)/8; slots below 7/8 A - 8 sd (and the
+            // window pitch of this round, an upper bound) are safe.  Off with
+            // GG_LR_PREFEED=0.
+            static const bool prefeed = !(getenv("GG_LR_PREFEED") && atoi(getenv("GG_LR_PREFEED")) == 0);
+            if (prefeed && A > 4096) {
+                const double sd = std::sqrt(7.0 * (double)A) / 8.0;
+                const int64_t lo = (int64_t)(0.875 * (double)A - 8.0 * sd);
+                if (lo > 0) LRC(gg::epoch_prefeed(h, (uint64_t)lo, ((uint64_t)A + 31) / 32 * 32));
+            }
             int32_t kept = 0;
             LCK(cudaMemcpyAsync(&kept, d_num, 4, cudaMemcpyDeviceToHost, s));
             LCK(cudaStreamSynchronize(s));

@@ -203,6 +203,11 @@ struct prng_s {
     size_t od_cap[2] = {};
     cudaEvent_t od_free[2] = {};       // recorded at epoch_end: kernels done with the slot
     int od_slot = 1;
+    // prefed part of the next epoch's window (gg_epoch_prefeed): walkers
+    // [0, pf_hi) of draw pf_J0 already staged in od_buf[pf_slot] at pitch pf_pitch
+    bool pf_valid = false;
+    int pf_slot = 0;
+    uint64_t pf_J0 = 0, pf_hi = 0, pf_pitch = 0;
     uint32_t *od_wmap_buf[2] = {};     // slot -> walker maps (prng_epoch_begin_list)
     size_t od_wmap_cap[2] = {};
     const uint32_t *od_wmap = nullptr; // map of the open epoch, or nullptr
@@ -292,7 +297,8 @@ void feed_chunk(prng_s *h, uint64_t wa, uint64_t wb, uint64_t k0, uint32_t nrows
 // pinned chunk while the previous chunks are DMA'd on copy_stream.
 // On return every copy is enqueued on copy_stream.
 void stage_rows(prng_s *h, uint64_t k0, uint64_t nrows, uint64_t Wv, uint32_t *dst,
-                uint64_t dpitch, const uint32_t *ids = nullptr, bool bursty = false) {
+                uint64_t dpitch, const uint32_t *ids = nullptr, bool bursty = false,
+                bool row_segments = false) {
     if (nrows == 0 || Wv == 0) return;
     static const bool nt_all = getenv("GG_FEED_NT_ALL") != nullptr;  // A/B hook
     bursty = bursty || nt_all;
@@ -332,7 +338,9 @@ void stage_rows(prng_s *h, uint64_t k0, uint64_t nrows, uint64_t Wv, uint32_t *d
             cudaEventDestroy(b);
         }
     } trace_end{h, tr0, tr1, host_t0, h->stats.h2d_bytes};
-    if (2 * dpitch <= chunk_words) {
+    // row_segments: copy only columns [0, Wv) of every row (dst may point into
+    // the middle of a row); otherwise small windows go as whole-row chunks
+    if (2 * dpitch <= chunk_words && !row_segments) {
         uint64_t rows_per = std::max<uint64_t>(2, (chunk_words / dpitch) & ~1ull);
         for (uint64_t r = 0; r < nrows;) {
             uint64_t nr = std::min<uint64_t>(rows_per, nrows - r);
@@ -857,9 +865,13 @@ static int epoch_begin_impl(prng_t *h, uint64_t active_walkers, const uint32_t *
         cudaStream_t s = (cudaStream_t)stream;
         const uint64_t J0 = h->od_started ? h->od_J0 : (h->N + h->W - 1) / h->W;
         if (J0 + draws > 0xFFFFFFFFull) return PRNG_E_UNSUPPORTED;
-        const uint64_t pitch = round_up(active_walkers, 32);
-        const size_t bytes = (size_t)draws * h->R * pitch * 4;
         const int slot = h->od_slot ^ 1;
+        // walkers [0, pf_hi) of this window were staged ahead (gg_epoch_prefeed)
+        const bool pf = h->pf_valid && !ids && draws == 1 && h->pf_J0 == J0 &&
+                        h->pf_slot == slot && active_walkers <= h->pf_pitch;
+        h->pf_valid = false;
+        const uint64_t pitch = pf ? h->pf_pitch : round_up(active_walkers, 32);
+        const size_t bytes = (size_t)draws * h->R * pitch * 4;
         if (bytes > h->od_cap[slot] || (ids && active_walkers * 4 > h->od_wmap_cap[slot])) {
             CK(cudaEventSynchronize(h->od_free[slot]));
             if (bytes > h->od_cap[slot]) {
@@ -894,8 +906,18 @@ static int epoch_begin_impl(prng_t *h, uint64_t active_walkers, const uint32_t *
         // small windows are bursty (the consumer waits for the last chunk):
         // stream them past the CPU caches; large windows pipeline like bulk
         const bool bursty = bytes < (1ull << 30);
-        stage_rows(h, 2 + h->R0 + h->R * J0, (uint64_t)draws * h->R, active_walkers, h->od_bits,
-                   pitch, ids, bursty);
+        if (pf) {
+            if (active_walkers > h->pf_hi) {  // the rest: walkers [pf_hi, active)
+                const uint64_t lo = h->pf_hi, saved = h->o.walker_base;
+                h->o.walker_base = saved + lo;
+                stage_rows(h, 2 + h->R0 + h->R * J0, h->R, active_walkers - lo, h->od_bits + lo,
+                           pitch, nullptr, true, true);
+                h->o.walker_base = saved;
+            }
+        } else {
+            stage_rows(h, 2 + h->R0 + h->R * J0, (uint64_t)draws * h->R, active_walkers,
+                       h->od_bits, pitch, ids, bursty);
+        }
         join_copies(h, s);
         h->od_J0 = J0;
         h->od_D = draws;
@@ -906,6 +928,36 @@ static int epoch_begin_impl(prng_t *h, uint64_t active_walkers, const uint32_t *
         return PRNG_OK;
     });
 }
+
+extern "C++" {
+namespace gg {
+// Stage the next epoch's window ahead (one draw, walkers [0, hi), pitch
+// `pitch` >= the next epoch's active count) while the current epoch's
+// kernels run: list ranking knows the next round's active count only after
+// its kernels, but not fewer than ~7/8 of this round's nodes survive.  The
+// next prng_epoch_begin with draws = 1 and active <= pitch stages only the
+// walkers above hi.  No effect on the numbers: a walker's bits at a draw are
+// a pure function of (seed, walker, draw) (R9).
+int epoch_prefeed(prng_t *h, uint64_t hi, uint64_t pitch) {
+    if (!h || h->od_open || !h->od_started || hi == 0 || hi > pitch || pitch > round_up(h->W, 32))
+        return PRNG_E_INVALID;
+    return guard(h, [&] {
+        const int slot = h->od_slot ^ 1;
+        const uint64_t J0 = h->od_J0;
+        const size_t bytes = (size_t)h->R * pitch * 4;
+        if (bytes > h->od_cap[slot]) return PRNG_OK;  // not reserved: skip the prefeed
+        CK(cudaStreamWaitEvent(h->copy_stream, h->od_free[slot], 0));
+        stage_rows(h, 2 + h->R0 + h->R * J0, h->R, hi, h->od_buf[slot], pitch, nullptr, true);
+        h->pf_valid = true;
+        h->pf_slot = slot;
+        h->pf_J0 = J0;
+        h->pf_hi = hi;
+        h->pf_pitch = pitch;
+        return PRNG_OK;
+    });
+}
+}  // namespace gg
+}  // extern "C++"
 
 int prng_epoch_begin(prng_t *h, uint64_t active_walkers, uint32_t draws, void *stream) {
     if (!h) return PRNG_E_INVALID;
