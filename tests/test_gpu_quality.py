@@ -104,3 +104,14 @@ def test_nist_sp800_22_on_gpu_output():
             for k, v in N.run(bits[s * 1_000_000:(s + 1) * 1_000_000]).items():
                 fails[k] = fails.get(k, 0) + (v < 0.01)
         assert max(fails.values()) <= 3, (name, fails)
+
+
+def test_crush_style_on_gpu_output():
+    """Crush-style tests (tests/battery_crush.py) on 2^23 labels of the C2
+    generator computed on the GPU, bulk and walker-major order."""
+    import battery_crush as C
+    z = gen(64, n_draws=64, W=1 << 17).cpu().numpy()
+    for name, arr in (("bulk", z), ("walker-major", z.T.copy())):
+        res = C.run(np.ascontiguousarray(arr).reshape(-1).view(np.uint32))
+        bad = {k: v for k, v in res.items() if v < 1e-4}
+        assert not bad, (name, bad)

@@ -1,5 +1,5 @@
 """Battery report on GPU output (tool, Tables II-III):
-tests/battery.py on 2^24 labels (2^25 u32 words) of the C2 generator, in bulk
+tests/battery.py (+ the Crush-style tests of tests/battery_crush.py) on 2^24 labels (2^25 u32 words) of the C2 generator, in bulk
 and walker-major order, for l = 64 (the paper's walk), l = 16 and l = 1.
 
     python tools/quality_report.py > profiles/r01_battery.json
@@ -16,6 +16,7 @@ import numpy as np  # noqa: E402
 import torch  # noqa: E402
 
 import battery as B  # noqa: E402
+import battery_crush as C  # noqa: E402
 from paper_conf_ipps_banerjeebk12_b200 import Generator  # noqa: E402
 
 W, D = 1 << 18, 64
@@ -29,7 +30,9 @@ for l in (64, 16, 1):
     g.close()
     for order, arr in (("bulk", z), ("walker-major", z.T)):
         t = time.time()
-        res = B.run(np.ascontiguousarray(arr).reshape(-1).view(np.uint32))
+        words = np.ascontiguousarray(arr).reshape(-1).view(np.uint32)
+        res = B.run(words)
+        res.update({f"crush:{k}": v for k, v in C.run(words).items()})
         rep["runs"][f"l={l} {order}"] = {
             "p": {k: float(f"{v:.3g}") for k, v in res.items()},
             "failed": sorted(k for k, v in res.items() if v < 1e-4),
