@@ -1,6 +1,6 @@
 """Interleaved A/B timing of the bulk fill under different env configs (tool).
 
-    python tools/ab_fill.py "GG_FILL_BPS=28" "GG_FILL_KPW=4" ...
+    python tools/ab_fill.py "GG_FILL_MINB=24" "GG_FILL_KPW=2" ...
 Each config runs in its own subprocess (env is read once per process);
 configs are interleaved R times; prints the median kernel ms per config.
 """
