@@ -208,6 +208,31 @@ __device__ __forceinline__ void gg_r2p_two(uint32_t S, uint32_t C, uint32_t &x, 
           "n"(SH1));
 }
 
+/* Bipartite walk (variant 1): a pair of steps whose first
+ * (even global step) applies sigma_k and whose second (odd) applies
+ * sigma_k^{-1}: y' = y - 2x - c | x' = x - 2y - c, as r = 2x + c, v = 2y + c
+ * (IMAD), @py y -= r, @px x -= v: 6 SASS instead of 5, kept on the FMA-heavy
+ * pipe where it can be (the plain-add form put 2/3 of the kernel on the ALU). */
+#define GG_R2P_INV(S)                                                                      \
+    "shl.b32 ct, %3, " S ";\n\tshr.b32 c, ct, 30;\n\t"                                      \
+    "mad.lo.u32 r, %0, 2, c;\n\tmad.lo.u32 v, %1, 2, c;\n\t"
+
+template <int B0, int B1, int SH0, int SH1>
+__device__ __forceinline__ void gg_r2p_two_bip(uint32_t S, uint32_t C, uint32_t &x, uint32_t &y)
+{
+    asm volatile(
+        "{\n\t.reg .pred py0, px0, py1, px1;\n\t.reg .b32 t, ct, c, u, s, r, v;\n\t"
+        "and.b32 t, %2, %4;\n\tsetp.ne.b32 py0, t, 0;\n\t"
+        "and.b32 t, %2, %5;\n\tsetp.ne.b32 px0, t, 0;\n\t"
+        "and.b32 t, %2, %6;\n\tsetp.ne.b32 py1, t, 0;\n\t"
+        "and.b32 t, %2, %7;\n\tsetp.ne.b32 px1, t, 0;\n\t"
+        GG_R2P_U("%8") "@py0 add.u32 %1, u, %0;\n\t@px0 add.u32 %0, u, %1;\n\t"
+        GG_R2P_INV("%9") "@py1 sub.u32 %1, %1, r;\n\t@px1 sub.u32 %0, %0, v;\n\t}"
+        : "+r"(x), "+r"(y)
+        : "r"(S), "r"(C), "n"(1u << B0), "n"(2u << B0), "n"(1u << B1), "n"(2u << B1), "n"(SH0),
+          "n"(SH1));
+}
+
 /* Flag word F and constant word C of a 10-field word Q (fields at 3i). */
 __device__ __forceinline__ void gg_r2p_prep(uint32_t Q, uint32_t &C, uint32_t &F)
 {
@@ -220,30 +245,40 @@ __device__ __forceinline__ void gg_r2p_prep(uint32_t Q, uint32_t &C, uint32_t &F
 
 #define GG_SH(k) (30 - 3 * (k))
 
-template <int NK>
+/* A pair of steps (fields K, K+1 with flags at bits B0, B1 of S). */
+template <bool BIP, int B0, int B1, int K>
+__device__ __forceinline__ void gg_r2p_pair(uint32_t S, uint32_t C, uint32_t &x, uint32_t &y)
+{
+    if (BIP)
+        gg_r2p_two_bip<B0, B1, GG_SH(K), GG_SH(K + 1)>(S, C, x, y);
+    else
+        gg_r2p_two<B0, B1, GG_SH(K), GG_SH(K + 1)>(S, C, x, y);
+}
+
+template <int NK, bool BIP = false>
 __device__ __forceinline__ void gg_word10_r2p(uint32_t Q, uint32_t &x, uint32_t &y)
 {
     uint32_t C, F;
     gg_r2p_prep(Q, C, F);
     const uint32_t G = F >> 4;
-    gg_r2p_two<0, 3, GG_SH(0), GG_SH(1)>(F, C, x, y);
-    gg_r2p_two<2, 5, GG_SH(2), GG_SH(3)>(G, C, x, y);
+    gg_r2p_pair<BIP, 0, 3, 0>(F, C, x, y);
+    gg_r2p_pair<BIP, 2, 5, 2>(G, C, x, y);
     if (NK == 4) return;
-    gg_r2p_two<8, 11, GG_SH(4), GG_SH(5)>(G, C, x, y);
-    gg_r2p_two<18, 21, GG_SH(6), GG_SH(7)>(F, C, x, y);
-    gg_r2p_two<24, 27, GG_SH(8), GG_SH(9)>(F, C, x, y);
+    gg_r2p_pair<BIP, 8, 11, 4>(G, C, x, y);
+    gg_r2p_pair<BIP, 18, 21, 6>(F, C, x, y);
+    gg_r2p_pair<BIP, 24, 27, 8>(F, C, x, y);
 }
 
 /* Steps of one 10-field word (NK = 10) or of the 4-field tail word (NK = 4) for
  * two walkers, from prepared (C, F) of each. */
-template <int NK>
+template <int NK, bool BIP = false>
 __device__ __forceinline__ void gg_steps10x2_r2p(uint32_t Ca, uint32_t Fa, uint32_t Cb, uint32_t Fb,
                                                  uint32_t &xa, uint32_t &ya, uint32_t &xb, uint32_t &yb)
 {
     const uint32_t Ga = Fa >> 4, Gb = Fb >> 4;
 #define GG_R2P2(B0, B1, K0, K1, SA, SB)                                     \
-    gg_r2p_two<B0, B1, GG_SH(K0), GG_SH(K1)>(SA, Ca, xa, ya);                \
-    gg_r2p_two<B0, B1, GG_SH(K0), GG_SH(K1)>(SB, Cb, xb, yb);
+    gg_r2p_pair<BIP, B0, B1, K0>(SA, Ca, xa, ya);                            \
+    gg_r2p_pair<BIP, B0, B1, K0>(SB, Cb, xb, yb);
     GG_R2P2(0, 3, 0, 1, Fa, Fb)
     GG_R2P2(2, 5, 2, 3, Ga, Gb)
     if (NK == 4) return;
@@ -253,38 +288,43 @@ __device__ __forceinline__ void gg_steps10x2_r2p(uint32_t Ca, uint32_t Fa, uint3
 #undef GG_R2P2
 }
 
-template <int NK>
+template <int NK, bool BIP = false>
 __device__ __forceinline__ void gg_word10x2_r2p(uint32_t Qa, uint32_t Qb, uint32_t &xa, uint32_t &ya,
                                                 uint32_t &xb, uint32_t &yb)
 {
     uint32_t Ca, Fa, Cb, Fb;
     gg_r2p_prep(Qa, Ca, Fa);
     gg_r2p_prep(Qb, Cb, Fb);
-    gg_steps10x2_r2p<NK>(Ca, Fa, Cb, Fb, xa, ya, xb, yb);
+    gg_steps10x2_r2p<NK, BIP>(Ca, Fa, Cb, Fb, xa, ya, xb, yb);
 }
 
-/* 64 steps from a 6-word record (R2P form). */
+/* 64 steps from a 6-word record (R2P form).  BIP: the bipartite variant with
+ * an even first global step (steps 2i apply sigma, steps 2i+1 sigma^{-1}; every
+ * R2P pair is (even, odd) because 10-field words and pairs start at even
+ * field indices). */
+template <bool BIP = false>
 __device__ __forceinline__ void gg_walk64_r2p(const uint32_t w[6], uint32_t &x, uint32_t &y)
 {
-    gg_word10_r2p<10>(w[0], x, y);
-    gg_word10_r2p<10>(__funnelshift_r(w[0], w[1], 30), x, y);
-    gg_word10_r2p<10>(__funnelshift_r(w[1], w[2], 28), x, y);
-    gg_word10_r2p<10>(__funnelshift_r(w[2], w[3], 26), x, y);
-    gg_word10_r2p<10>(__funnelshift_r(w[3], w[4], 24), x, y);
-    gg_word10_r2p<10>(__funnelshift_r(w[4], w[5], 22), x, y);
-    gg_word10_r2p<4>(w[5] >> 20, x, y);
+    gg_word10_r2p<10, BIP>(w[0], x, y);
+    gg_word10_r2p<10, BIP>(__funnelshift_r(w[0], w[1], 30), x, y);
+    gg_word10_r2p<10, BIP>(__funnelshift_r(w[1], w[2], 28), x, y);
+    gg_word10_r2p<10, BIP>(__funnelshift_r(w[2], w[3], 26), x, y);
+    gg_word10_r2p<10, BIP>(__funnelshift_r(w[3], w[4], 24), x, y);
+    gg_word10_r2p<10, BIP>(__funnelshift_r(w[4], w[5], 22), x, y);
+    gg_word10_r2p<4, BIP>(w[5] >> 20, x, y);
 }
 
+template <bool BIP = false>
 __device__ __forceinline__ void gg_walk64x2_r2p(const uint32_t a[6], const uint32_t b[6], uint32_t &xa,
                                                 uint32_t &ya, uint32_t &xb, uint32_t &yb)
 {
-    gg_word10x2_r2p<10>(a[0], b[0], xa, ya, xb, yb);
-    gg_word10x2_r2p<10>(__funnelshift_r(a[0], a[1], 30), __funnelshift_r(b[0], b[1], 30), xa, ya, xb, yb);
-    gg_word10x2_r2p<10>(__funnelshift_r(a[1], a[2], 28), __funnelshift_r(b[1], b[2], 28), xa, ya, xb, yb);
-    gg_word10x2_r2p<10>(__funnelshift_r(a[2], a[3], 26), __funnelshift_r(b[2], b[3], 26), xa, ya, xb, yb);
-    gg_word10x2_r2p<10>(__funnelshift_r(a[3], a[4], 24), __funnelshift_r(b[3], b[4], 24), xa, ya, xb, yb);
-    gg_word10x2_r2p<10>(__funnelshift_r(a[4], a[5], 22), __funnelshift_r(b[4], b[5], 22), xa, ya, xb, yb);
-    gg_word10x2_r2p<4>(a[5] >> 20, b[5] >> 20, xa, ya, xb, yb);
+    gg_word10x2_r2p<10, BIP>(a[0], b[0], xa, ya, xb, yb);
+    gg_word10x2_r2p<10, BIP>(__funnelshift_r(a[0], a[1], 30), __funnelshift_r(b[0], b[1], 30), xa, ya, xb, yb);
+    gg_word10x2_r2p<10, BIP>(__funnelshift_r(a[1], a[2], 28), __funnelshift_r(b[1], b[2], 28), xa, ya, xb, yb);
+    gg_word10x2_r2p<10, BIP>(__funnelshift_r(a[2], a[3], 26), __funnelshift_r(b[2], b[3], 26), xa, ya, xb, yb);
+    gg_word10x2_r2p<10, BIP>(__funnelshift_r(a[3], a[4], 24), __funnelshift_r(b[3], b[4], 24), xa, ya, xb, yb);
+    gg_word10x2_r2p<10, BIP>(__funnelshift_r(a[4], a[5], 22), __funnelshift_r(b[4], b[5], 22), xa, ya, xb, yb);
+    gg_word10x2_r2p<4, BIP>(a[5] >> 20, b[5] >> 20, xa, ya, xb, yb);
 }
 
 /* One step, any m (generic path), x, y < m.  m = 2^k: wrapped 32-bit
@@ -407,12 +447,15 @@ __device__ __forceinline__ uint64_t prng_next(prng_state *st, const prng_view *v
     }
     const uint32_t *rec = v->bits + (uint64_t)st->used * v->R * v->pitch + st->slot;
     uint32_t x = st->x, y = st->y;
-    if (v->l == 64u && v->pow2 && v->variant == 0) {
+    if (v->l == 64u && v->pow2 && (v->variant == 0 || (v->variant == 1 && (v->l0 & 1u) == 0))) {
         uint32_t w[6];
 #pragma unroll
         for (int r = 0; r < 6; r++)
             w[r] = __ldg(rec + (uint64_t)r * v->pitch);
-        gg_walk64_r2p(w, x, y);
+        if (v->variant == 0)
+            gg_walk64_r2p(w, x, y);
+        else
+            gg_walk64_r2p<true>(w, x, y);  /* draw starts at global step l0 + 64 j: even */
     } else {
         const uint64_t s0 = (uint64_t)v->l0 + (uint64_t)v->l * (v->J0 + st->used);
         gg_walk_generic(rec, v->pitch, v->l, x, y, (uint32_t)v->m, v->pow2 != 0, v->variant, s0);

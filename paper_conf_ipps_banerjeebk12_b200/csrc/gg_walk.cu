@@ -32,11 +32,14 @@ __global__ void __launch_bounds__(128) gg_init_kernel(InitArgs a) {
         x = (uint32_t)(x % a.m);
         y = (uint32_t)(y % a.m);
     }
-    if (a.l0 == 64 && a.pow2 && a.variant == 0) {
+    if (a.l0 == 64 && a.pow2 && a.variant <= 1) {
         uint32_t w[6];
 #pragma unroll
         for (int r = 0; r < 6; r++) w[r] = rec[(uint64_t)(2 + r) * a.pitch];
-        gg_walk64_r2p(w, x, y);
+        if (a.variant == 0)
+            gg_walk64_r2p(w, x, y);
+        else
+            gg_walk64_r2p<true>(w, x, y);  // burn-in starts at global step 0 (even)
     } else {
         gg_walk_generic(rec + 2 * a.pitch, a.pitch, a.l0, x, y, (uint32_t)a.m, a.pow2 != 0,
                         a.variant, 0);
@@ -257,7 +260,7 @@ __global__ void __launch_bounds__(64, 32) gg_fill64_tma_kernel(const __grid_cons
 // lane); one TMA box of 64 x 6 words (1.5 KB) per draw; the two walks are
 // interleaved step by step.  STEP: 1 = R2P form of the walk step (default),
 // 0 = per-step LOP3.P predicates (A/B hook GG_FILL_STEP=0).
-template <int EMIT, int MINB = 1, int STEP = 1, int U2 = 1>
+template <int EMIT, int MINB = 1, int STEP = 1, int U2 = 1, bool BIP = false>
 __global__ void __launch_bounds__(64, MINB) gg_fill64x2_tma_kernel(const __grid_constant__ CUtensorMap tmap,
                                                          FillArgs a, uint32_t units64) {
     constexpr int kTile = 6 * 64;
@@ -319,7 +322,9 @@ __global__ void __launch_bounds__(64, MINB) gg_fill64x2_tma_kernel(const __grid_
                 wb[r] = buf[r * 64 + 32 + lane];
             }
             uint32_t nxa = xa, nya = ya, nxb = xb, nyb = yb;
-            if (STEP)
+            if (BIP)
+                gg_walk64x2_r2p<true>(wa, wb, nxa, nya, nxb, nyb);
+            else if (STEP)
                 gg_walk64x2_r2p(wa, wb, nxa, nya, nxb, nyb);
             else
                 gg_walk64x2(wa, wb, nxa, nya, nxb, nyb);
@@ -576,6 +581,26 @@ cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count) {
             } else {
                 plan_grid(gg_fill_l1_tma_kernel<1>, units, sm_count, blocks, threads);
                 gg_fill_l1_tma_kernel<1><<<blocks, threads, 0, s>>>(map, a, units);
+            }
+            return cudaGetLastError();
+        }
+    }
+    if (a.l == 64 && a.pow2 && a.variant == 1 && (a.l0 & 1u) == 0 && a.rows &&
+        getenv("GG_FILL_NO_BIP") == nullptr) {
+        // bipartite variant (f1): every draw starts at an even global step
+        // (l0 + 64 j), so the fixed (sigma, sigma^-1) pairing of the R2P walk holds
+        CUtensorMap map;
+        const uint32_t units64 = (a.W + 63u) / 64u;
+        if (make_window_map(&map, a.bits, a.pitch, a.rows, 64)) {
+            if (a.out_u32) {
+                plan_grid(gg_fill64x2_tma_kernel<2, 1, 1, 1, true>, units64, sm_count, blocks, threads);
+                gg_fill64x2_tma_kernel<2, 1, 1, 1, true><<<blocks, threads, 0, s>>>(map, a, units64);
+            } else if (a.log2m == 32) {
+                plan_grid(gg_fill64x2_tma_kernel<0, 1, 1, 1, true>, units64, sm_count, blocks, threads);
+                gg_fill64x2_tma_kernel<0, 1, 1, 1, true><<<blocks, threads, 0, s>>>(map, a, units64);
+            } else {
+                plan_grid(gg_fill64x2_tma_kernel<1, 1, 1, 1, true>, units64, sm_count, blocks, threads);
+                gg_fill64x2_tma_kernel<1, 1, 1, 1, true><<<blocks, threads, 0, s>>>(map, a, units64);
             }
             return cudaGetLastError();
         }

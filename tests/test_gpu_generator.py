@@ -334,3 +334,34 @@ def test_ggcpu_bit_source_parity(torch_cuda):
         for t in (0, 1, 150, W - 1):
             assert np.array_equal(got[t], O.walker_draws(M32, 64, 64, seed, t, 12, 3)), t
     g.close()
+
+
+@pytest.mark.parametrize("burnin", [64, 63])
+def test_bipartite_fast_kernel_parity(torch_cuda, burnin):
+    # variant 1 with l = 64 and m = 2^k takes the R2P (sigma, sigma^-1)-pair
+    # kernel when every draw starts at an even global step (l0 even); an odd
+    # l0 must fall back to the generic kernel.  Prefetched (K-mode) and
+    # streamed fills, ragged walker count, u64 and u32 formats.
+    torch = torch_cuda
+    W, D, seed = 1000, 9, 0x5EED0009
+    for m in (M32, 1 << 20):
+        g = G(walkers=W, seed=seed, m=m, variant=1, burnin_len=burnin)
+        g.prefetch(D)
+        o = torch.empty(W * D - 3, dtype=torch.int64, device="cuda")
+        g.fill(o)
+        want = O.bulk_v(m, 64, burnin, 1, seed, W, 0, W * D + 5)
+        assert np.array_equal(as_u64(o), want[: W * D - 3]), m
+        o2 = torch.empty(8, dtype=torch.int64, device="cuda")  # streamed past the window
+        g.fill(o2)
+        assert np.array_equal(as_u64(o2), want[W * D - 3: W * D + 5]), m
+        g.close()
+    # on demand through prng_next
+    g = G(walkers=W, seed=seed, variant=1, burnin_len=burnin)
+    g.epoch_begin(W, 3)
+    od = torch.empty(W * 3, dtype=torch.int64, device="cuda")
+    g.consume(W, uniform=3, out=od)
+    g.epoch_end()
+    got = as_u64(od).reshape(W, 3)
+    want = O.bulk_v(M32, 64, burnin, 1, seed, W, 0, W * 3).reshape(3, W).T
+    assert np.array_equal(got, want)
+    g.close()

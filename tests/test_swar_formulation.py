@@ -139,3 +139,62 @@ def test_r2p_recipe_every_field_value_at_every_position():
             w = [(bits >> (32 * r)) & M for r in range(6)]
             x0, y0 = (int(v) for v in rng.integers(0, 2 ** 32, 2, dtype=np.uint64))
             assert walk64_r2p(w, x0, y0) == O.walk(1 << 32, x0, y0, np.array(w, np.uint32), 64)
+
+
+# ---------------------------------------------------------------------------
+# Bipartite variant (gg_r2p_two_bip): in every R2P pair the
+# first step (even field index = even global step) applies sigma_k and the
+# second sigma_k^{-1}: r = 2x + c, @py y -= r | v = 2y + c, @px x -= v.
+
+def _word10_r2p_bip(Q, nk, x, y):
+    f1, f2 = Q >> 1, Q >> 2
+    MY = ((f1 | Q) & 0x09249249) & ~f2 & M
+    MX = (f2 & ~(f1 & Q)) & M
+    C = (Q - MY) & M
+    F = (MY | ((MX << 1) & 0x12492492)) & M
+    G = F >> G_SHIFT
+    for src, k, bit in (R2P_GROUPS_10 if nk == 10 else R2P_GROUPS_4):
+        S = F if src == "F" else G
+        P = _r2p_load(S, bit // 8)
+        py, px = P[bit % 8], P[bit % 8 + 1]
+        c = ((C << (30 - 3 * k)) & M) >> 30
+        if k % 2 == 0:
+            u = (x + y + c) & M
+            if py:
+                y = (u + x) & M
+            if px:
+                x = (u + y) & M
+        else:
+            r, v = (2 * x + c) & M, (2 * y + c) & M
+            if py:
+                y = (y - r) & M
+            if px:
+                x = (x - v) & M
+    return x, y
+
+
+def walk64_r2p_bip(w, x, y):
+    x, y = _word10_r2p_bip(w[0], 10, x, y)
+    for a, s in [(0, 30), (1, 28), (2, 26), (3, 24), (4, 22)]:
+        x, y = _word10_r2p_bip(_fsr(w[a], w[a + 1], s), 10, x, y)
+    return _word10_r2p_bip(w[5] >> 20, 4, x, y)
+
+
+def _oracle_bip(w, x0, y0, s0):
+    rec = np.array(w, np.uint32)
+    xs, ys = np.array([x0], np.uint64), np.array([y0], np.uint64)
+    O.lib().or_walk_bipartite(1 << 32, xs.ctypes.data, ys.ctypes.data, rec.ctypes.data, 64, s0)
+    return int(xs[0]), int(ys[0])
+
+
+def test_r2p_bipartite_recipe_every_field_value_at_every_position():
+    rng = np.random.default_rng(13)
+    for i in range(64):
+        for b in range(8):
+            bits = int.from_bytes(rng.bytes(24), "little")
+            bits &= ~(7 << (3 * i))
+            bits |= b << (3 * i)
+            w = [(bits >> (32 * r)) & M for r in range(6)]
+            x0, y0 = (int(v) for v in rng.integers(0, 2 ** 32, 2, dtype=np.uint64))
+            s0 = 64 * int(rng.integers(1, 1000))  # l0 + 64 j: even
+            assert walk64_r2p_bip(w, x0, y0) == _oracle_bip(w, x0, y0, s0)
