@@ -29,3 +29,15 @@ def test_c_consumer_matches_oracle(W, seed):
         assert val == int(O.walker_draws(M32, 64, 64, seed, t, draw, 1)[0]), line
         n += 1
     assert n == 5 * 4 + sum(t % 3 + 1 for t in (0, 1, 2, W // 2, W - 1))
+
+
+def test_python_quickstart_runs():
+    import sys
+    out = subprocess.run([sys.executable, os.path.join(ROOT, "examples", "quickstart.py")],
+                         capture_output=True, text=True, timeout=300)
+    assert out.returncode == 0, out.stderr[-2000:]
+    text = out.stdout
+    for key in ("bulk:", "fill_host:", "on demand:", "list ranking:", "Monte Carlo:",
+                "glibc rand_r bits:", "host generator bits:"):
+        assert key in text, text
+    assert "tail rank 1048575" in text and "overrun flag 0" in text, text
