@@ -356,7 +356,7 @@ def run_ours(args, rank, world, local_rank):
     # per number, HBM-bound; 2^20 walkers x 1024 draws, bits resident
     if not args.no_l1:
         g = Generator(walkers=W_PER_GPU, seed=SEED, walk_len=1, walker_base=rank * W_PER_GPU,
-                      device=local_rank)
+                      device=local_rank, host_threads=feed_threads)
         D1 = 1024
         g.prefetch(D1)
         g.mark()
@@ -390,7 +390,7 @@ def run_ours(args, rank, world, local_rank):
     if not args.no_ondemand:
         S = 100
         g = Generator(walkers=W_PER_GPU, seed=SEED + 1, walker_base=rank * W_PER_GPU,
-                      device=local_rank)
+                      device=local_rank, host_threads=feed_threads)
         xo = torch.empty(W_PER_GPU, dtype=torch.int64, device=dev)
         g.epoch_begin(W_PER_GPU, S * (args.warmup + 1))
         for _ in range(args.warmup):
@@ -600,6 +600,12 @@ def host_info():
     return {"nproc": os.cpu_count(), "cpu_model": model}
 
 
+def _feed_threads(world):
+    """Host FEED threads per rank: the ranks of a node share its cores."""
+    local_world = int(os.environ.get("LOCAL_WORLD_SIZE", str(world)))
+    return max(1, (os.cpu_count() or 1) // max(1, local_world))
+
+
 def _hash32(t, r):
     """Integer hash of (thread, round) on the device (activity pattern only)."""
     x = (t * 2654435761 + r * 0x27D4EB2F + 0x165667B1) & 0xFFFFFFFF
@@ -623,7 +629,10 @@ def ondemand_shaped(rank, world, local_rank, stream, max_over_ranks):
     out = {}
     # LR-shaped
     W, R = 1 << 24, 24
-    g = Generator(walkers=W, seed=SEED + 2, walker_base=rank * W, device=local_rank)
+    # 2^24 walkers fill the 24-bit walker-id space (R9), so the ranks run this
+    # replicated consumer (like list ranking's Phase I) on seeds of their own
+    g = Generator(walkers=W, seed=SEED + 2 + 1000 * rank, device=local_rank,
+                  host_threads=_feed_threads(world))
     t = torch.arange(W, dtype=torch.int64, device=dev)
     counts = []
     for r in range(R):
@@ -650,7 +659,10 @@ def ondemand_shaped(rank, world, local_rank, stream, max_over_ranks):
     g.close()
     del counts, t
     torch.cuda.empty_cache()
-    g = Generator(walkers=W, seed=SEED + 2, walker_base=rank * W, device=local_rank)
+    # 2^24 walkers fill the 24-bit walker-id space (R9), so the ranks run this
+    # replicated consumer (like list ranking's Phase I) on seeds of their own
+    g = Generator(walkers=W, seed=SEED + 2 + 1000 * rank, device=local_rank,
+                  host_threads=_feed_threads(world))
     g.epoch_begin(W, R)
     torch.cuda.synchronize()
     for r in range(R):
@@ -671,7 +683,8 @@ def ondemand_shaped(rank, world, local_rank, stream, max_over_ranks):
     c = torch.clamp(torch.ceil(torch.log1p(-u) / math.log1p(-1 / mean)), 1, cap).to(torch.int32)
     draws = int(c.sum().item())
     c = c.to(dev)
-    g = Generator(walkers=W, seed=SEED + 3, walker_base=rank * W, device=local_rank)
+    g = Generator(walkers=W, seed=SEED + 3, walker_base=rank * W, device=local_rank,
+                  host_threads=_feed_threads(world))
     g.epoch_begin(W, cap)
     a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     torch.cuda.synchronize()
