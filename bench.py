@@ -105,23 +105,31 @@ def cpu_baseline_block(target_seconds: float = 8.0):
 
 # ------------------------------------------------------------------ clocks
 class ClockSampler:
-    """SM clock and throttle reasons sampled every ~2 ms by NVML (power every 8th) in a
-    thread (nvidia-smi -lms 20 as the fallback).  start() before the warm-up,
-    mark(True/False) around the timed region: summary() keeps the samples
-    taken inside it (the recipe's clocks line), falling back to every sample
-    under load if the region is shorter than the sampling period."""
+    """SM clock and throttle reasons sampled during the run by two independent
+    samplers: NVML in a thread (~2 ms; power every 8th sample) and
+    `nvidia-smi -lms 20` in a subprocess (the recipe's clocks line).  Each
+    NVML query is tried on its own, so one unsupported call does not stop the
+    sampling.  start before the warm-up, mark(True/False) around the timed
+    region: summary() keeps the samples taken inside it (NVML's if it has
+    any, else nvidia-smi's), falling back to every sample under load if the
+    region is shorter than the sampling period."""
     REASONS = (("hw_slowdown", 0x8), ("hw_thermal_slowdown", 0x40), ("sw_thermal_slowdown", 0x20),
                ("sw_power_cap", 0x4), ("hw_power_brake_slowdown", 0x80))
 
     def __init__(self, gpu_id: str, index: int = 0):
         self.gpu_id, self.index = gpu_id, index
-        self.rows = []  # (t, sm_mhz, max_mhz, power_w, reasons bitmask)
+        self.rows = {"nvml": [], "nvidia-smi": []}  # (t, sm_mhz, max_mhz, power_w, reasons)
         self.t0 = self.t1 = None
         self.stop = threading.Event()
-        self.th = None
-        self.backend = None
+        self.threads = []
+        self.proc = None
 
     def __enter__(self):
+        self._nvml()
+        self._smi()
+        return self
+
+    def _nvml(self):
         try:
             import pynvml
             pynvml.nvmlInit()
@@ -129,28 +137,34 @@ class ClockSampler:
                 h = pynvml.nvmlDeviceGetHandleByUUID(self.gpu_id)
             except Exception:
                 h = pynvml.nvmlDeviceGetHandleByIndex(self.index)
-            self.backend = "nvml"
-
-            def run():
-                # clock + reasons every ~2 ms; power (a slower query) every 8th sample
-                mx = pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM)
-                pw, i = 0.0, 0
-                while not self.stop.is_set():
-                    try:
-                        if i % 8 == 0:
-                            pw = pynvml.nvmlDeviceGetPowerUsage(h) / 1000.0
-                        i += 1
-                        sm = pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM)
-                        rs = pynvml.nvmlDeviceGetCurrentClocksEventReasons(h)
-                        self.rows.append((time.perf_counter(), float(sm), float(mx), pw, int(rs)))
-                    except Exception:
-                        pass
-                    time.sleep(0.002)
-            self.th = threading.Thread(target=run, daemon=True)
-            self.th.start()
         except Exception:
-            self._smi()
-        return self
+            return
+        reasons_fn = getattr(pynvml, "nvmlDeviceGetCurrentClocksEventReasons", None) or \
+            getattr(pynvml, "nvmlDeviceGetCurrentClocksThrottleReasons", None)
+
+        def q(fn, *a):
+            try:
+                return fn(h, *a)
+            except Exception:
+                return None
+
+        def run():
+            mx = q(pynvml.nvmlDeviceGetMaxClockInfo, pynvml.NVML_CLOCK_SM)
+            pw, i = 0.0, 0
+            while not self.stop.is_set():
+                if i % 8 == 0:
+                    v = q(pynvml.nvmlDeviceGetPowerUsage)
+                    pw = v / 1000.0 if v is not None else pw
+                i += 1
+                sm = q(pynvml.nvmlDeviceGetClockInfo, pynvml.NVML_CLOCK_SM)
+                rs = q(reasons_fn) if reasons_fn else None
+                if sm is not None and rs is not None:
+                    self.rows["nvml"].append((time.perf_counter(), float(sm),
+                                              float(mx if mx is not None else sm), pw, int(rs)))
+                time.sleep(0.002)
+        th = threading.Thread(target=run, daemon=True)
+        th.start()
+        self.threads.append(th)
 
     def _smi(self):
         fields = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
@@ -162,8 +176,8 @@ class ClockSampler:
                  "--format=csv,noheader,nounits", "-lms", "20"],
                 stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
         except OSError:
+            self.proc = None
             return
-        self.backend = "nvidia-smi"
         bits = (0x8, 0x40, 0x20, 0x4)
 
         def run():
@@ -172,12 +186,13 @@ class ClockSampler:
                 if len(p) == 7:
                     try:
                         rs = sum(b for b, v in zip(bits, p[3:]) if v == "Active")
-                        self.rows.append((time.perf_counter(), float(p[0]), float(p[1]),
-                                          float(p[2]), rs))
+                        self.rows["nvidia-smi"].append((time.perf_counter(), float(p[0]),
+                                                        float(p[1]), float(p[2]), rs))
                     except ValueError:
                         pass
-        self.th = threading.Thread(target=run, daemon=True)
-        self.th.start()
+        th = threading.Thread(target=run, daemon=True)
+        th.start()
+        self.threads.append(th)
 
     def mark(self, start: bool):
         if start:
@@ -187,29 +202,42 @@ class ClockSampler:
 
     def __exit__(self, *exc):
         self.stop.set()
-        if self.backend == "nvidia-smi":
+        if self.proc is not None:
             self.proc.terminate()
             try:
                 self.proc.wait(timeout=5)
             except subprocess.TimeoutExpired:
                 self.proc.kill()
-        elif self.th:
-            self.th.join(timeout=1)
+        for th in self.threads:
+            th.join(timeout=1)
 
     def summary(self):
-        rows = list(self.rows)
-        inside = [r for r in rows if self.t0 is not None and self.t1 is not None
-                  and self.t0 <= r[0] <= self.t1]
-        use = inside if len(inside) >= 3 else rows
+        def inside(rows):
+            return [r for r in rows if self.t0 is not None and self.t1 is not None
+                    and self.t0 <= r[0] <= self.t1]
+        src, use, ins = None, [], []
+        for name in ("nvml", "nvidia-smi"):
+            rows = list(self.rows[name])
+            ins = inside(rows)
+            if len(ins) >= 3:
+                src, use = name, ins
+                break
+        if not use:
+            for name in ("nvml", "nvidia-smi"):
+                rows = list(self.rows[name])
+                if rows:
+                    src, use, ins = name, rows, inside(rows)
+                    break
         if not use:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"], "samples": 0}
         reasons = sorted({n for r in use for n, b in self.REASONS if r[4] & b})
         return {"sm_mhz": statistics.median(r[1] for r in use),
                 "sm_max_mhz": max(r[2] for r in use), "reasons": reasons,
                 "power_w_max": max(r[3] for r in use), "samples": len(use),
-                "samples_in_timed_region": len(inside),
-                "window": "timed region" if use is inside else "whole K-mode section (region < 3 samples)",
-                "source": self.backend}
+                "samples_in_timed_region": len(ins),
+                "window": "timed region" if use is ins else "whole K-mode section (region < 3 samples)",
+                "source": src,
+                "samples_by_source": {k: len(v) for k, v in self.rows.items()}}
 
 
 def committed_traffic():
