@@ -280,6 +280,14 @@ def pcie_bound(h2d_bytes: float, d2h_bytes: float, labels: float):
             "max_value": labels / t / 1e9, "source": "profiles/r01_measured_box.json"}
 
 
+def _measured_h2d_gbs():
+    try:
+        with open(os.path.join(ROOT, "profiles", "r01_measured_box.json")) as f:
+            return float(json.load(f)["h2d_pinned_gbs"])
+    except (OSError, KeyError, ValueError):
+        return None
+
+
 def measured_peaks():
     try:
         with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
@@ -774,6 +782,11 @@ def run_apps(args, rank, world, local_rank, max_over_ranks, feed_threads=0):
         "ranks_ok": ok,
         "note": "on-demand: the host feeds exactly the draws of each round after learning the "
                 "active count (FEED + H2D inside the measured time)"}
+    h2d = _measured_h2d_gbs()
+    if h2d:
+        floor = info["draws"] * BITS_BYTES_PER_LABEL / (h2d * 1e9)
+        out["list_ranking"]["pcie_floor_ms"] = floor * 1e3
+        out["list_ranking"]["frac_of_pcie_floor"] = floor / wall
     g.close()
     del s_t, p_t, rank_t
     torch.cuda.empty_cache()
@@ -801,6 +814,10 @@ def run_apps(args, rank, world, local_rank, max_over_ranks, feed_threads=0):
         "absorbed": [v / tal[0] for v in tal[5:]], "conserved": tal[0] == sum(tal[1:]),
         "host_bits_GB_used": draws * BITS_BYTES_PER_LABEL / 1e9,
         "host_bits_GB_fed": r["walker_epochs_fed"] * 192 * BITS_BYTES_PER_LABEL / 1e9 * world}
+    if h2d:  # per rank: its own fed bytes over its own link
+        floor = r["walker_epochs_fed"] * 192 * BITS_BYTES_PER_LABEL / (h2d * 1e9)
+        out["monte_carlo"]["pcie_floor_ms"] = floor * 1e3
+        out["monte_carlo"]["frac_of_pcie_floor"] = floor / wall
     g.close()
     return out
 
