@@ -298,6 +298,71 @@ __device__ __forceinline__ void gg_word10x2_r2p(uint32_t Qa, uint32_t Qb, uint32
     gg_steps10x2_r2p<NK, BIP>(Ca, Fa, Cb, Fb, xa, ya, xb, yb);
 }
 
+/* One step of the R2P form alone (the first of a pair, flags at bit B0). */
+template <int B0, int SH0>
+__device__ __forceinline__ void gg_r2p_single(uint32_t S, uint32_t C, uint32_t &x, uint32_t &y)
+{
+    asm volatile(
+        "{\n\t.reg .pred py0, px0;\n\t.reg .b32 t, ct, c, u, s;\n\t"
+        "and.b32 t, %2, %4;\n\tsetp.ne.b32 py0, t, 0;\n\t"
+        "and.b32 t, %2, %5;\n\tsetp.ne.b32 px0, t, 0;\n\t"
+        GG_R2P_U("%6") "@py0 add.u32 %1, u, %0;\n\t@px0 add.u32 %0, u, %1;\n\t}"
+        : "+r"(x), "+r"(y)
+        : "r"(S), "r"(C), "n"(1u << B0), "n"(2u << B0), "n"(SH0));
+}
+
+/* The first NK (1..10) steps of a 10-field word, forward maps, m = 2^k: the
+ * pairs of gg_word10_r2p, the last one cut to its first step for odd NK. */
+template <int NK>
+__device__ __forceinline__ void gg_word_r2p_n(uint32_t Q, uint32_t &x, uint32_t &y)
+{
+    uint32_t C, F;
+    gg_r2p_prep(Q, C, F);
+    const uint32_t G = F >> 4;
+    if (NK >= 2) gg_r2p_pair<false, 0, 3, 0>(F, C, x, y);
+    else gg_r2p_single<0, GG_SH(0)>(F, C, x, y);
+    if (NK >= 4) gg_r2p_pair<false, 2, 5, 2>(G, C, x, y);
+    else if (NK == 3) gg_r2p_single<2, GG_SH(2)>(G, C, x, y);
+    if (NK >= 6) gg_r2p_pair<false, 8, 11, 4>(G, C, x, y);
+    else if (NK == 5) gg_r2p_single<8, GG_SH(4)>(G, C, x, y);
+    if (NK >= 8) gg_r2p_pair<false, 18, 21, 6>(F, C, x, y);
+    else if (NK == 7) gg_r2p_single<18, GG_SH(6)>(F, C, x, y);
+    if (NK >= 10) gg_r2p_pair<false, 24, 27, 8>(F, C, x, y);
+    else if (NK == 9) gg_r2p_single<24, GG_SH(8)>(F, C, x, y);
+}
+
+/* l steps (any l >= 1), forward maps, m = 2^k, from a record of ceil(3l/32)
+ * words at rec[r * stride]: 10-field groups are funnel-shifted out of the
+ * record (each word is loaded once) and walked with the R2P step. */
+__device__ __forceinline__ void gg_walk_r2p_any(const uint32_t *rec, uint64_t stride, uint32_t l,
+                                                uint32_t R, uint32_t &x, uint32_t &y)
+{
+    uint32_t lo = __ldg(rec), hi = R > 1 ? __ldg(rec + stride) : 0u;
+    uint32_t wi = 0;  /* lo = word wi, hi = word wi + 1 (0 past the record) */
+    for (uint32_t g = 0; 10u * g < l; g++) {
+        const uint32_t bit = 30u * g, i = bit >> 5, sh = bit & 31u;
+        if (i != wi) {  /* advance one word (30-bit groups move at most one word) */
+            lo = hi;
+            wi = i;
+            hi = wi + 1 < R ? __ldg(rec + (uint64_t)(wi + 1) * stride) : 0u;
+        }
+        const uint32_t Q = __funnelshift_r(lo, hi, sh);
+        const uint32_t nk = min(10u, l - 10u * g);
+        switch (nk) {
+        case 10: gg_word_r2p_n<10>(Q, x, y); break;
+        case 9: gg_word_r2p_n<9>(Q, x, y); break;
+        case 8: gg_word_r2p_n<8>(Q, x, y); break;
+        case 7: gg_word_r2p_n<7>(Q, x, y); break;
+        case 6: gg_word_r2p_n<6>(Q, x, y); break;
+        case 5: gg_word_r2p_n<5>(Q, x, y); break;
+        case 4: gg_word_r2p_n<4>(Q, x, y); break;
+        case 3: gg_word_r2p_n<3>(Q, x, y); break;
+        case 2: gg_word_r2p_n<2>(Q, x, y); break;
+        default: gg_word_r2p_n<1>(Q, x, y); break;
+        }
+    }
+}
+
 /* 64 steps from a 6-word record (R2P form).  BIP: the bipartite variant with
  * an even first global step (steps 2i apply sigma, steps 2i+1 sigma^{-1}; every
  * R2P pair is (even, odd) because 10-field words and pairs start at even
@@ -456,6 +521,8 @@ __device__ __forceinline__ uint64_t prng_next(prng_state *st, const prng_view *v
             gg_walk64_r2p(w, x, y);
         else
             gg_walk64_r2p<true>(w, x, y);  /* draw starts at global step l0 + 64 j: even */
+    } else if (v->pow2 && v->variant == 0) {
+        gg_walk_r2p_any(rec, v->pitch, v->l, v->R, x, y);
     } else {
         const uint64_t s0 = (uint64_t)v->l0 + (uint64_t)v->l * (v->J0 + st->used);
         gg_walk_generic(rec, v->pitch, v->l, x, y, (uint32_t)v->m, v->pow2 != 0, v->variant, s0);

@@ -536,6 +536,39 @@ __global__ void __launch_bounds__(64) gg_fill_generic_kernel(FillArgs a, uint32_
     }
 }
 
+// Any walk length l (2..4096, l != 64), m = 2^k, forward maps: one walker per
+// lane, the draw's record read from the window word by word (coalesced across
+// the warp) and walked with the R2P step in 10-field groups
+// (gg_walk_r2p_any); the generic kernel stays the path for other m and the
+// bipartite variant at l != 64.
+__global__ void __launch_bounds__(64) gg_fill_any_kernel(FillArgs a, uint32_t units) {
+    const uint32_t lane = threadIdx.x & 31u;
+    const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+    for (uint32_t u = warp; u < units; u += nwarps) {
+        const uint32_t t = u * 32u + lane;
+        if (t >= a.W) break;
+        uint32_t j0, j1;
+        walker_draw_range(a.N, a.nl, a.W, t, j0, j1);
+        j0 = max(j0, a.ja);
+        j1 = min(j1, a.jb);
+        if (j0 >= j1) continue;
+        uint32_t x = a.x[t], y = a.y[t];
+        for (uint32_t j = j0; j < j1; j++) {
+            const uint32_t *rec = a.bits + t + (uint64_t)(j - a.Jw) * a.R * a.pitch;
+            gg_walk_r2p_any(rec, a.pitch, a.l, a.R, x, y);
+            const uint64_t lab = gg_label(x, y, a.m, a.log2m, true);
+            const uint64_t g = (uint64_t)j * a.W + t;
+            if (a.out_u32)
+                reinterpret_cast<uint32_t *>(a.out)[g - a.g_origin] = (uint32_t)lab;
+            else
+                reinterpret_cast<uint64_t *>(a.out)[g - a.g_origin] = lab;
+        }
+        a.x[t] = x;
+        a.y[t] = y;
+    }
+}
+
 // Grid of 64-thread blocks (2 warps each); `units` = work items a warp takes
 // round-robin (32 walkers; 64 for the x2 kernels).  One item per warp: the
 // block scheduler starts a new block wherever one finishes, so SMs stay busy to
@@ -661,6 +694,9 @@ cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count) {
             plan_grid(gg_fill64_kernel<0>, units, sm_count, blocks, threads);
             gg_fill64_kernel<0><<<blocks, threads, 0, s>>>(a, units);
         }
+    } else if (a.pow2 && a.variant == 0 && a.l >= 2 && getenv("GG_FILL_NO_ANY") == nullptr) {
+        plan_grid(gg_fill_any_kernel, units, sm_count, blocks, threads);
+        gg_fill_any_kernel<<<blocks, threads, 0, s>>>(a, units);
     } else {
         plan_grid(gg_fill_generic_kernel, units, sm_count, blocks, threads);
         gg_fill_generic_kernel<<<blocks, threads, 0, s>>>(a, units);
