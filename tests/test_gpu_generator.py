@@ -365,3 +365,23 @@ def test_bipartite_fast_kernel_parity(torch_cuda, burnin):
     want = O.bulk_v(M32, 64, burnin, 1, seed, W, 0, W * 3).reshape(3, W).T
     assert np.array_equal(got, want)
     g.close()
+
+
+def test_any_walk_length_parity(torch_cuda):
+    # gg_fill_any_kernel / gg_walk_r2p_any: every last-group size (l mod 10 =
+    # 0..9, single-step tails), records ending inside / exactly at a word, for
+    # bulk fills and prng_next
+    torch = torch_cuda
+    W, D, seed = 97, 3, 0x5EED000A
+    for l in list(range(2, 42)) + [63, 65, 100, 128, 333]:
+        g = G(walkers=W, seed=seed, walk_len=l, m=1 << 16)
+        o = torch.empty(W * D, dtype=torch.int64, device="cuda")
+        g.fill(o)
+        want = O.bulk_v(1 << 16, l, 64, 0, seed, W, 0, W * (D + 2))
+        assert np.array_equal(as_u64(o), want[: W * D]), l
+        g.epoch_begin(W, 2)
+        od = torch.empty(W * 2, dtype=torch.int64, device="cuda")
+        g.consume(W, uniform=2, out=od)
+        g.epoch_end()
+        assert np.array_equal(as_u64(od).reshape(W, 2), want[W * D:].reshape(2, W).T), l
+        g.close()
