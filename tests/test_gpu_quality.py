@@ -115,3 +115,25 @@ def test_crush_style_on_gpu_output():
         res = C.run(np.ascontiguousarray(arr).reshape(-1).view(np.uint32))
         bad = {k: v for k, v in res.items() if v < 1e-4}
         assert not bad, (name, bad)
+
+
+def test_c1_chi_square_on_gpu_output():
+    """BASELINE C1 ("tiny expander (m=2^8), 1024 walkers, 2^20 numbers - GPU vs
+    CPU oracle bit-exact, chi-square check"): the 2^20 labels computed on the
+    GPU are equidistributed over the m^2 = 65536 vertices (chi-square, 65535
+    dof), and so are the pairs (x mod 16, y mod 16) of consecutive draws of a
+    walker (serial test, 65535 dof over 16^4 cells)."""
+    import torch
+    from paper_conf_ipps_banerjeebk12_b200 import Generator
+    W, n = 1024, 1 << 20
+    g = Generator(walkers=W, seed=0x5EED0001, m=256)
+    o = torch.empty(n, dtype=torch.int64, device="cuda")
+    g.fill(o)
+    lab = o.cpu()
+    p1 = chi2_p(torch.bincount(lab, minlength=65536), n / 65536)
+    z = lab.view(n // W, W)
+    x, y = z % 256, z // 256
+    cell = ((x[:-1] % 16) * 16 + y[:-1] % 16) * 256 + (x[1:] % 16) * 16 + y[1:] % 16
+    p2 = chi2_p(torch.bincount(cell.reshape(-1), minlength=65536), cell.numel() / 65536)
+    assert p1 > ALPHA and p2 > ALPHA, (p1, p2)
+    g.close()
