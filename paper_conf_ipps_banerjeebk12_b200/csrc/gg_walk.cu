@@ -388,11 +388,17 @@ __device__ __forceinline__ void gg_step_l1(uint32_t b, uint32_t &x, uint32_t &y)
     x = (cx < 3u) ? tx : x;
 }
 
-template <int EMIT>
+// OST: interior tiles leave through the TMA store engine (the 16 x 32 labels
+// staged in shared memory, one cp.async.bulk.tensor store per tile; omap =
+// the output as a 2D tensor of 8-byte labels, dim0 = walkers, dim1 = draws)
+// instead of 16 STG.64 per lane.
+template <int EMIT, int OST = 0>
 __global__ void __launch_bounds__(64) gg_fill_l1_tma_kernel(const __grid_constant__ CUtensorMap tmap,
-                                                            FillArgs a, uint32_t units) {
+                                                            FillArgs a, uint32_t units,
+                                                            const __grid_constant__ CUtensorMap omap) {
     constexpr int kTile = kL1Draws * 32;
     __shared__ __align__(128) uint32_t tiles[kFillWarps][2][kTile];
+    __shared__ __align__(128) uint64_t otiles[OST ? kFillWarps : 1][2][OST ? kTile : 1];
     __shared__ __align__(8) uint64_t bars[kFillWarps][2];
     const uint32_t lane = threadIdx.x & 31u, wib = threadIdx.x >> 5;
     const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -444,11 +450,34 @@ __global__ void __launch_bounds__(64) gg_fill_l1_tma_kernel(const __grid_constan
                 uint32_t b[kL1Draws];
 #pragma unroll
                 for (int d = 0; d < kL1Draws; d++) b[d] = buf[d * 32 + lane];
-                const uint64_t i0 = (uint64_t)jt * a.W + t - a.g_origin;
+                if (OST) {
+                    uint64_t *ob = otiles[OST ? wib : 0][sidx];
+                    if (lane == 0)  // the store issued from this buffer two tiles ago has read it
+                        asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+                    __syncwarp();
 #pragma unroll
-                for (int d = 0; d < kL1Draws; d++) {
-                    gg_step_l1(b[d] & 7u, x, y);
-                    emit_label<EMIT>(a, i0 + (uint64_t)d * a.W, x, y);
+                    for (int d = 0; d < kL1Draws; d++) {
+                        gg_step_l1(b[d] & 7u, x, y);
+                        ob[d * 32 + lane] = EMIT == 0 ? ((uint64_t)y << 32 | x)
+                                                      : gg_label(x, y, a.m, a.log2m, true);
+                    }
+                    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                    __syncwarp();
+                    if (lane == 0) {
+                        asm volatile(
+                            "cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%1, %2}], [%3];"
+                            ::"l"(&omap), "r"((int32_t)(u * 32u)), "r"((int32_t)jt),
+                              "r"(smem_u32(ob))
+                            : "memory");
+                        asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+                    }
+                } else {
+                    const uint64_t i0 = (uint64_t)jt * a.W + t - a.g_origin;
+#pragma unroll
+                    for (int d = 0; d < kL1Draws; d++) {
+                        gg_step_l1(b[d] & 7u, x, y);
+                        emit_label<EMIT>(a, i0 + (uint64_t)d * a.W, x, y);
+                    }
                 }
             } else {
 #pragma unroll 4
@@ -473,6 +502,7 @@ __global__ void __launch_bounds__(64) gg_fill_l1_tma_kernel(const __grid_constan
             a.y[t] = y;
         }
     }
+    if (OST && lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
 }
 
 static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
@@ -491,6 +521,23 @@ static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
 }
 
 // 2D map over the SoA window: dim0 = walkers (pitch), dim1 = rows; box 32 x 6.
+// Output of a bulk fill as a 2D tensor of 8-byte labels: element (t, j) at
+// out + j * W + t - g_origin; box 32 walkers x kL1Draws draws.  TMA needs a
+// 16-byte aligned base and row stride: W even and (out - g_origin) aligned.
+static bool make_out_map(CUtensorMap *map, const FillArgs &a) {
+    auto enc = get_encode();
+    if (!enc || (a.W & 1u) || a.jb == 0) return false;
+    const uintptr_t base = (uintptr_t)a.out - (uintptr_t)(a.g_origin * 8ull);
+    if (base % 16) return false;
+    cuuint64_t dims[2] = {(cuuint64_t)a.W, (cuuint64_t)a.jb};
+    cuuint64_t strides[1] = {(cuuint64_t)a.W * 8};
+    cuuint32_t box[2] = {32, (cuuint32_t)kL1Draws};
+    cuuint32_t estr[2] = {1, 1};
+    return enc(map, CU_TENSOR_MAP_DATA_TYPE_UINT64, 2, (void *)base, dims, strides, box, estr,
+               CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+               CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
 static bool make_window_map(CUtensorMap *map, const uint32_t *bits, uint64_t pitch, uint64_t rows,
                             uint32_t box_walkers = 32, uint32_t box_rows = 6) {
     auto enc = get_encode();
@@ -605,15 +652,27 @@ cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count) {
     if (a.l == 1 && a.pow2 && a.variant == 0) {
         CUtensorMap map;
         if (a.rows && make_window_map(&map, a.bits, a.pitch, a.rows, 32, kL1Draws)) {
+            CUtensorMap omap;
+            static const bool ost_on = !(getenv("GG_L1_TMA_STORE") && atoi(getenv("GG_L1_TMA_STORE")) == 0);
+            const bool ost = ost_on && !a.out_u32 && make_out_map(&omap, a);
+            if (!ost) memset(&omap, 0, sizeof(omap));
             if (a.out_u32) {
                 plan_grid(gg_fill_l1_tma_kernel<2>, units, sm_count, blocks, threads);
-                gg_fill_l1_tma_kernel<2><<<blocks, threads, 0, s>>>(map, a, units);
+                gg_fill_l1_tma_kernel<2><<<blocks, threads, 0, s>>>(map, a, units, omap);
             } else if (a.log2m == 32) {
-                plan_grid(gg_fill_l1_tma_kernel<0>, units, sm_count, blocks, threads);
-                gg_fill_l1_tma_kernel<0><<<blocks, threads, 0, s>>>(map, a, units);
+                if (ost) {
+                    plan_grid(gg_fill_l1_tma_kernel<0, 1>, units, sm_count, blocks, threads);
+                    gg_fill_l1_tma_kernel<0, 1><<<blocks, threads, 0, s>>>(map, a, units, omap);
+                } else {
+                    plan_grid(gg_fill_l1_tma_kernel<0>, units, sm_count, blocks, threads);
+                    gg_fill_l1_tma_kernel<0><<<blocks, threads, 0, s>>>(map, a, units, omap);
+                }
+            } else if (ost) {
+                plan_grid(gg_fill_l1_tma_kernel<1, 1>, units, sm_count, blocks, threads);
+                gg_fill_l1_tma_kernel<1, 1><<<blocks, threads, 0, s>>>(map, a, units, omap);
             } else {
                 plan_grid(gg_fill_l1_tma_kernel<1>, units, sm_count, blocks, threads);
-                gg_fill_l1_tma_kernel<1><<<blocks, threads, 0, s>>>(map, a, units);
+                gg_fill_l1_tma_kernel<1><<<blocks, threads, 0, s>>>(map, a, units, omap);
             }
             return cudaGetLastError();
         }
