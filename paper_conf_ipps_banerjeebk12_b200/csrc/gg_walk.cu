@@ -169,11 +169,13 @@ constexpr int kFillWarps = 2;       // warps per block
 // m = 2^k < 2^32; 2 = low u32 word of the label (m <= 2^16).
 template <int EMIT>
 __device__ __forceinline__ void emit_label(const FillArgs &a, uint64_t idx, uint32_t x, uint32_t y) {
+    // EMIT: 0 = m = 2^32 (label = the pair), 1 / 2 = m = 2^k as u64 / u32,
+    // 3 / 4 = other m (x, y already reduced) as u64 / u32
     if (EMIT == 0) {
         reinterpret_cast<uint2 *>(a.out)[idx] = make_uint2(x, y);
     } else {
-        const uint64_t lab = gg_label(x, y, a.m, a.log2m, true);
-        if (EMIT == 2)
+        const uint64_t lab = gg_label(x, y, a.m, a.log2m, EMIT <= 2);
+        if (EMIT == 2 || EMIT == 4)
             reinterpret_cast<uint32_t *>(a.out)[idx] = (uint32_t)lab;
         else
             reinterpret_cast<uint64_t *>(a.out)[idx] = lab;
@@ -260,7 +262,7 @@ __global__ void __launch_bounds__(64, 32) gg_fill64_tma_kernel(const __grid_cons
 // lane); one TMA box of 64 x 6 words (1.5 KB) per draw; the two walks are
 // interleaved step by step.  STEP: 1 = R2P form of the walk step (default),
 // 0 = per-step LOP3.P predicates (A/B hook GG_FILL_STEP=0).
-template <int EMIT, int MINB = 1, int STEP = 1, int U2 = 1, bool BIP = false>
+template <int EMIT, int MINB = 1, int STEP = 1, int U2 = 1, bool BIP = false, bool MOD = false>
 __global__ void __launch_bounds__(64, MINB) gg_fill64x2_tma_kernel(const __grid_constant__ CUtensorMap tmap,
                                                          FillArgs a, uint32_t units64) {
     constexpr int kTile = 6 * 64;
@@ -322,7 +324,10 @@ __global__ void __launch_bounds__(64, MINB) gg_fill64x2_tma_kernel(const __grid_
                 wb[r] = buf[r * 64 + 32 + lane];
             }
             uint32_t nxa = xa, nya = ya, nxb = xb, nyb = yb;
-            if (BIP)
+            if (MOD) {  // m not a power of two, m <= 2^30
+                gg_walk64_r2p_mod(wa, (uint32_t)a.m, nxa, nya);
+                gg_walk64_r2p_mod(wb, (uint32_t)a.m, nxb, nyb);
+            } else if (BIP)
                 gg_walk64x2_r2p<true>(wa, wb, nxa, nya, nxb, nyb);
             else if (STEP)
                 gg_walk64x2_r2p(wa, wb, nxa, nya, nxb, nyb);
@@ -693,6 +698,22 @@ cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count) {
             } else {
                 plan_grid(gg_fill64x2_tma_kernel<1, 1, 1, 1, true>, units64, sm_count, blocks, threads);
                 gg_fill64x2_tma_kernel<1, 1, 1, 1, true><<<blocks, threads, 0, s>>>(map, a, units64);
+            }
+            return cudaGetLastError();
+        }
+    }
+    if (a.l == 64 && !a.pow2 && a.variant == 0 && a.m <= (1ull << 30) && a.rows &&
+        getenv("GG_FILL_NO_MOD") == nullptr) {
+        // other m <= 2^30: the R2P step with two conditional subtracts per step
+        CUtensorMap map;
+        const uint32_t units64 = (a.W + 63u) / 64u;
+        if (make_window_map(&map, a.bits, a.pitch, a.rows, 64)) {
+            if (a.out_u32) {
+                plan_grid(gg_fill64x2_tma_kernel<4, 1, 1, 1, false, true>, units64, sm_count, blocks, threads);
+                gg_fill64x2_tma_kernel<4, 1, 1, 1, false, true><<<blocks, threads, 0, s>>>(map, a, units64);
+            } else {
+                plan_grid(gg_fill64x2_tma_kernel<3, 1, 1, 1, false, true>, units64, sm_count, blocks, threads);
+                gg_fill64x2_tma_kernel<3, 1, 1, 1, false, true><<<blocks, threads, 0, s>>>(map, a, units64);
             }
             return cudaGetLastError();
         }

@@ -385,3 +385,31 @@ def test_any_walk_length_parity(torch_cuda):
         g.epoch_end()
         assert np.array_equal(as_u64(od).reshape(W, 2), want[W * D:].reshape(2, W).T), l
         g.close()
+
+
+@pytest.mark.parametrize("m", [3, 1000, 65521, (1 << 30) - 35, 1 << 30])
+def test_non_power_of_two_fast_kernel_parity(torch_cuda, m):
+    # m <= 2^30 not a power of two takes the R2P kernel with two conditional
+    # subtracts per step (bulk, u64 and u32 formats, and prng_next)
+    torch = torch_cuda
+    W, D, seed = 700, 5, 0x5EED000B
+    g = G(walkers=W, seed=seed, m=m)
+    g.prefetch(D)
+    o = torch.empty(W * D - 1, dtype=torch.int64, device="cuda")
+    g.fill(o)
+    want = O.bulk_v(m, 64, 64, 0, seed, W, 0, W * D + 2 * W)
+    assert np.array_equal(as_u64(o), want[: W * D - 1])
+    if m <= 65536:
+        g2 = G(walkers=W, seed=seed, m=m)
+        o32 = torch.empty(W * D, dtype=torch.int32, device="cuda")
+        g2.fill(o32)
+        assert np.array_equal(o32.cpu().numpy().view(np.uint32).astype(np.uint64), want[: W * D])
+        g2.close()
+    g.close()
+    g = G(walkers=W, seed=seed, m=m)  # on demand from draw 0 (a ragged fill would skip draws, R10)
+    g.epoch_begin(W, 2)
+    od = torch.empty(W * 2, dtype=torch.int64, device="cuda")
+    g.consume(W, uniform=2, out=od)
+    g.epoch_end()
+    assert np.array_equal(as_u64(od).reshape(W, 2), want[: 2 * W].reshape(2, W).T)
+    g.close()

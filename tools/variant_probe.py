@@ -14,6 +14,7 @@ W, D = 1 << 20, 64
 res = {}
 for name, kw in (("forward m=2^32 l=64", {}), ("bipartite m=2^32 l=64", {"variant": 1}),
                  ("forward m=2^32-5 l=64", {"m": (1 << 32) - 5}),
+                 ("forward m=2^30-35 l=64", {"m": (1 << 30) - 35}),
                  ("forward m=2^32 l=16", {"walk_len": 16})):
     g = Generator(walkers=W, seed=9, **kw)
     g.prefetch(D)
