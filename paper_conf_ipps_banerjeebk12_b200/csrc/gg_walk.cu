@@ -531,7 +531,8 @@ static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
 // 16-byte aligned base and row stride: W even and (out - g_origin) aligned.
 static bool make_out_map(CUtensorMap *map, const FillArgs &a) {
     auto enc = get_encode();
-    if (!enc || (a.W & 1u) || a.jb == 0) return false;
+    // coordinates are int32: absolute draw indices must stay below 2^31
+    if (!enc || (a.W & 1u) || a.jb == 0 || a.jb > 0x7FFFFFF0u) return false;
     const uintptr_t base = (uintptr_t)a.out - (uintptr_t)(a.g_origin * 8ull);
     if (base % 16) return false;
     cuuint64_t dims[2] = {(cuuint64_t)a.W, (cuuint64_t)a.jb};
