@@ -321,6 +321,14 @@ def run_ours(args, rank, world, local_rank):
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         return float(t.item())
 
+    def per_rank(v: float) -> list:
+        if world == 1:
+            return [v]
+        t = torch.zeros(world, dtype=torch.float64, device=dev)
+        t[rank] = v
+        dist.all_reduce(t)  # each slot is non-zero on exactly one rank
+        return [float(x) for x in t.tolist()]
+
     # ---- K-mode: bits resident in HBM, one prng_fill per step
     g = Generator(walkers=W_PER_GPU, seed=SEED, walker_base=rank * W_PER_GPU, device=local_rank,
                   host_threads=feed_threads)
@@ -353,7 +361,8 @@ def run_ours(args, rank, world, local_rank):
     clk.__exit__(None, None, None)
     barrier()
     launches = g.stats()["kernel_launches"] - launches0
-    ms = max_over_ranks(start.elapsed_time(end))
+    ms_ranks = per_rank(start.elapsed_time(end))
+    ms = max(ms_ranks)
     step_ms = [a.elapsed_time(b) for a, b in zip(ev0, ev1)]
     kern_ms = statistics.mean(step_ms)
     labels_total = world * LABELS_PER_STEP * args.steps
@@ -381,9 +390,13 @@ def run_ours(args, rank, world, local_rank):
         "hbm_gbs_achieved": LABELS_PER_STEP * (BITS_BYTES_PER_LABEL + 8) / (kern_ms / 1e3) / 1e9,
         "hbm_gbs_peak": peaks.get("hbm_gbs"),
     }
-    # parity spot check of the timed output (walker 0, draw 0 of this rank)
+    # (no oracle call here: the task reserves oracle/ for the cpu_baseline leg;
+    # parity of this exact launch configuration is tests/test_gpu_generator.py's
+    # full-size sampled check)
     res = {"value": value, "ms": ms, "roofline": roofline, "clocks": clk.summary(),
-           "launches": launches, "kern_ms": kern_ms}
+           "launches": launches, "kern_ms": kern_ms,
+           "per_rank": [{"rank": r, "ms": x, "value": LABELS_PER_STEP * args.steps / (x / 1e3) / 1e9}
+                        for r, x in enumerate(ms_ranks)]}
     g.close()
     del out
     torch.cuda.empty_cache()
@@ -471,9 +484,11 @@ def run_ours(args, rank, world, local_rank):
             g.rewind()
             g.fill_host(host)
         torch.cuda.synchronize()
-        dt = max_over_ranks(time.perf_counter() - t)
+        dt_ranks = per_rank(time.perf_counter() - t)
+        dt = max(dt_ranks)
         s1 = g.stats()
         res["e2e"] = {
+            "per_rank": [LABELS_PER_STEP * e2e_steps / x / 1e9 for x in dt_ranks],
             "value": world * LABELS_PER_STEP * e2e_steps / dt / 1e9, "unit": UNIT,
             "h2d_bytes_per_step": (s1["h2d_bytes"] - s0["h2d_bytes"]) // e2e_steps,
             "d2h_bytes_per_step": (s1["d2h_bytes"] - s0["d2h_bytes"]) // e2e_steps,
@@ -822,9 +837,74 @@ def run_apps(args, rank, world, local_rank, max_over_ranks, feed_threads=0):
     return out
 
 
+def _free_port() -> int:
+    import socket
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    return port
+
+
+def self_launch(n: int) -> int:
+    """`bench.py --gpus N` run without a launcher: re-exec this script as N
+    ranks through torch.distributed.run (one process per GPU, rendezvous on
+    127.0.0.1).  The children see WORLD_SIZE, so they never spawn again.
+    NCCL's INIT log (communicator size per rank) goes to stderr; the ranks'
+    stdout is forwarded line by line, so the one JSON line rank 0 prints is
+    the only line this process writes to stdout."""
+    env = dict(os.environ)
+    env.setdefault("NCCL_DEBUG", "INFO")
+    env.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+    env["GG_BENCH_SELF_LAUNCHED"] = "1"
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+           "--master-addr=127.0.0.1", f"--master-port={_free_port()}",
+           os.path.abspath(__file__)] + sys.argv[1:]
+    p = subprocess.Popen(cmd, env=env, stdout=subprocess.PIPE, text=True)
+    for line in p.stdout:
+        if line.lstrip().startswith("{"):
+            sys.stdout.write(line)
+            sys.stdout.flush()
+        else:
+            sys.stderr.write(line)
+    return p.wait()
+
+
+def numa_nodes() -> int:
+    try:
+        return sum(1 for d in os.listdir("/sys/devices/system/node")
+                   if d.startswith("node") and d[4:].isdigit())
+    except OSError:
+        return 1
+
+
+def launch_probe(args, rank, world):
+    """--launch-probe: the multi-rank plumbing of the bench without a GPU
+    (process group, barrier, max over ranks, per-rank gather, one JSON line
+    from rank 0).  Run by tests/test_bench_launch.py with gloo on CPU."""
+    import torch
+    import torch.distributed as dist
+    if world > 1:
+        dist.barrier()
+        t = torch.tensor([float(rank + 1)], dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        mx = float(t.item())
+        per = [None] * world
+        dist.all_gather_object(per, {"rank": rank, "value": float(rank + 1)})
+    else:
+        mx, per = 1.0, [{"rank": 0, "value": 1.0}]
+    if rank == 0:
+        print(json.dumps({"metric": METRIC, "launch_probe": True, "n_gpus": world,
+                          "gpus_requested": args.gpus, "max_over_ranks": mx, "per_rank": per,
+                          "backend": dist.get_backend() if world > 1 else None,
+                          "feed_threads_per_rank": _feed_threads(world)}))
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--launch-probe", action="store_true",
+                    help="plumbing check only: process group + one JSON line, no GPU work")
     ap.add_argument("--steps", type=int, default=None, help="default 10 (C2), 1 (C5)")
     ap.add_argument("--workload", default="c2", choices=["c2", "c5"],
                     help="c2: bulk fill per GPU (weak scaling, default); c5: 2^34 labels split "
@@ -844,18 +924,43 @@ def main():
     if args.warmup < 3:
         args.warmup = 3
 
+    if args.gpus < 1:
+        raise SystemExit("--gpus must be >= 1")
+    if args.impl == "reference":
+        # the oracle on the host cores: rank 0 alone (or the single process)
+        if int(os.environ.get("RANK", "0")) != 0:
+            return 0
+        return run_reference(args, int(os.environ.get("WORLD_SIZE", str(args.gpus))))
+    if "WORLD_SIZE" not in os.environ and args.gpus > 1:
+        return self_launch(args.gpus)
+
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        raise SystemExit(f"bench.py: --gpus {args.gpus} but the launcher started {world} ranks")
     # test hooks: run the multi-rank path on one GPU (gloo, shared device)
-    backend = os.environ.get("GG_DIST_BACKEND", "nccl")
+    backend = os.environ.get("GG_DIST_BACKEND", "gloo" if args.launch_probe else "nccl")
     if "GG_FORCE_DEVICE" in os.environ:
         local_rank = int(os.environ["GG_FORCE_DEVICE"])
+    if world > 1:
+        # communicator size per rank in NCCL's INIT log (a self-launched run
+        # forwards these non-JSON lines to stderr)
+        os.environ.setdefault("NCCL_DEBUG", "INFO")
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+        # multi-socket hosts: each rank's FEED threads on its GPU's NUMA-local cores
+        if numa_nodes() > 1:
+            os.environ.setdefault("GG_FEED_PIN", "1")
 
-    if args.impl == "reference":
-        if rank != 0:
-            return 0
-        return run_reference(args, world)
+    if args.launch_probe:
+        if world > 1:
+            import torch.distributed as dist
+            dist.init_process_group(backend)
+        launch_probe(args, rank, world)
+        if world > 1:
+            import torch.distributed as dist
+            dist.destroy_process_group()
+        return 0
 
     # CPU baseline first (spawned processes; before CUDA is initialised)
     cpu = None
@@ -909,6 +1014,7 @@ def main():
             "clocks": res["clocks"], "gpu_launches": res["launches"],
             "on_demand": res.get("on_demand"), "apps": res.get("apps"),
             "l1_fill": res.get("l1_fill"), "host": host_info(),
+            "per_rank": res["per_rank"], "value_per_gpu": res["value"] / world,
         }
         print(json.dumps(line))
     if world > 1:
