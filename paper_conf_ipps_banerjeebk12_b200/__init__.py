@@ -61,6 +61,18 @@ def _fmt_of(t) -> int:
     raise TypeError(f"output dtype must be a 32- or 64-bit integer, got {t.dtype}")
 
 
+def _checked_count(t, n):
+    """n (default: all) numbers fit the contiguous tensor t; the library
+    writes n * itemsize bytes from t.data_ptr()."""
+    if not t.is_contiguous():
+        raise ValueError("output tensor must be contiguous")
+    if n is None:
+        return t.numel()
+    if not 0 <= n <= t.numel():
+        raise ValueError(f"n = {n} outside [0, {t.numel()}] for this output tensor")
+    return n
+
+
 class Generator:
     """One prng_t handle: W walkers of the 7-regular Gabber-Galil walk."""
 
@@ -71,6 +83,7 @@ class Generator:
         self._h = ctypes.c_void_p()
         self.walkers, self.seed, self.m, self.walk_len = walkers, seed, m, walk_len
         self._walker_base = walker_base
+        self.device = device
         self._bits_fn = None
         if bits_fn is not None:
             # bits_fn(walker0, nwalkers, word0, nwords) -> numpy uint32 [nwords, nwalkers]
@@ -92,7 +105,9 @@ class Generator:
     def fill(self, out, n: int | None = None, stream=None) -> None:
         """prng_fill: next n numbers into a CUDA tensor (int64 = labels, int32 = words)."""
         fmt = _fmt_of(out)
-        n = out.numel() if n is None else n
+        if out.device.type != "cuda" or out.device.index != self.device:
+            raise ValueError(f"fill: output must live on cuda:{self.device}, got {out.device}")
+        n = _checked_count(out, n)
         check(_lib.prng_fill(self._h, out.data_ptr(), n, fmt, _stream_handle(stream)), "prng_fill")
 
     def fill_ptr(self, dev_ptr: int, n: int, fmt: int, stream: int) -> int:
@@ -101,12 +116,20 @@ class Generator:
     def fill_host(self, out, n: int | None = None) -> None:
         """prng_fill_host: next n numbers into a host tensor / numpy array."""
         if hasattr(out, "data_ptr"):
-            fmt, ptr, numel = _fmt_of(out), out.data_ptr(), out.numel()
+            if out.device.type != "cpu":
+                raise ValueError(f"fill_host: output must be host memory, got {out.device}")
+            fmt, ptr = _fmt_of(out), out.data_ptr()
+            n = _checked_count(out, n)
         else:
-            import numpy as np
+            if out.dtype.itemsize not in (4, 8) or out.dtype.kind not in "iu":
+                raise TypeError(f"output dtype must be a 32- or 64-bit integer, got {out.dtype}")
+            if not out.flags["C_CONTIGUOUS"]:
+                raise ValueError("fill_host: output array must be C-contiguous")
             fmt = PRNG_FMT_U64 if out.dtype.itemsize == 8 else PRNG_FMT_U32
-            ptr, numel = out.ctypes.data, out.size
-        n = numel if n is None else n
+            ptr = out.ctypes.data
+            n = out.size if n is None else n
+            if not 0 <= n <= out.size:
+                raise ValueError(f"fill_host: n = {n} outside [0, {out.size}]")
         check(_lib.prng_fill_host(self._h, ptr, n, fmt), "prng_fill_host")
 
     def prefetch(self, draws: int) -> None:

@@ -428,6 +428,12 @@ __global__ void __launch_bounds__(64) gg_fill_l1_tma_kernel(const __grid_constan
         const uint32_t jlo = __reduce_min_sync(0xFFFFFFFFu, j0);
         const uint32_t jhi = __reduce_max_sync(0xFFFFFFFFu, j1);
         if (jlo >= jhi) continue;
+        // A previous unit of this warp (GG_FILL_ONEWAVE / GG_FILL_KPW grids)
+        // may have a tile store still reading either output buffer; the
+        // in-unit "wait_group.read 1" below only covers stores of this unit
+        // (within a unit interior tiles are consecutive, so the newest group
+        // always came from the other buffer).
+        if (OST && lane == 0) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
         // draws every lane of the warp emits (empty if some lane is idle)
         const uint32_t jin0 = __reduce_max_sync(0xFFFFFFFFu, j0);
         const uint32_t jin1 = __reduce_min_sync(0xFFFFFFFFu, j1);

@@ -408,6 +408,15 @@ int check_fmt(const prng_s *h, uint64_t n, int fmt) {
     return PRNG_OK;
 }
 
+// Draw indices are 32-bit in the walk kernels (FillArgs::Jw/ja/jb, the
+// per-walker cursor j[]): a bulk call whose last draw ceil((N + nl) / W) - 1
+// would not fit is refused up front (PRNG_E_UNSUPPORTED, nothing enqueued).
+bool draws_fit(const prng_s *h, uint64_t N, uint64_t nl) {
+    const uint64_t W = h->W;
+    if (nl > UINT64_MAX - N - W) return false;
+    return (N + nl + W - 1) / W <= 0xFFFFFFFFull;
+}
+
 gg::FillArgs fill_args(prng_s *h, const uint32_t *bits, uint64_t pitch, uint64_t rows,
                        uint64_t Jw, uint64_t ja, uint64_t jb, uint64_t N, uint64_t nl,
                        uint64_t g_origin, void *out, int out_u32) {
@@ -674,6 +683,7 @@ int prng_fill(prng_t *h, void *dev_ptr, uint64_t n, int fmt, void *stream) {
     const uintptr_t align = (fmt == PRNG_FMT_U32 && h->g.m <= 65536ull) ? 4 : 8;
     if (!dev_ptr || ((uintptr_t)dev_ptr % align)) return PRNG_E_INVALID;
     if (h->od_open) return PRNG_E_STATE;
+    if (!draws_fit(h, h->N, labels_of(h, n, fmt))) return PRNG_E_UNSUPPORTED;
     return guard(h, [&] {
         cudaStream_t s = (cudaStream_t)stream;
         const uint64_t nl = labels_of(h, n, fmt);
@@ -701,6 +711,7 @@ int prng_fill_host(prng_t *h, void *host_ptr, uint64_t n, int fmt) {
     if (n == 0) return PRNG_OK;
     if (!host_ptr) return PRNG_E_INVALID;
     if (h->od_open) return PRNG_E_STATE;
+    if (!draws_fit(h, h->N, labels_of(h, n, fmt))) return PRNG_E_UNSUPPORTED;
     return guard(h, [&] {
         const uint64_t nl = labels_of(h, n, fmt);
         const int out_u32 = (fmt == PRNG_FMT_U32 && h->g.m <= 65536ull) ? 1 : 0;
@@ -757,6 +768,7 @@ int prng_prefetch(prng_t *h, uint64_t draws) {
     if (!h) return PRNG_E_INVALID;
     if (draws == 0) return PRNG_E_INVALID;
     if (h->od_open) return PRNG_E_STATE;
+    if (h->N / h->W + draws > 0xFFFFFFFFull) return PRNG_E_UNSUPPORTED;
     return guard(h, [&] {
         const uint64_t pitch = h->pitch();
         const size_t bytes = (size_t)draws * h->R * pitch * 4;
@@ -810,10 +822,14 @@ int prng_rewind(prng_t *h, void *stream) {
 }
 
 namespace {
+// Everything that selects the walkers' bit streams and walk is part of the
+// header, so a checkpoint loads only into a handle that would have produced
+// it (another shard's walker_base, variant, burn-in or bit source is refused).
 struct SavedHeader {
     uint64_t magic, W, N, od_J0, od_started, m, seed, walk_len;
+    uint64_t burnin_len, variant, walker_base, bit_source;
 };
-const uint64_t kMagic = 0x47475052'4e470001ull;
+const uint64_t kMagic = 0x47475052'4e470002ull;
 }  // namespace
 
 int prng_state_size(prng_t *h, size_t *bytes) {
@@ -826,8 +842,11 @@ int prng_save(prng_t *h, void *host_buf, size_t bytes) {
     if (!h || !host_buf || bytes < sizeof(SavedHeader) + 3 * h->W * 4) return PRNG_E_INVALID;
     if (h->od_open) return PRNG_E_STATE;
     return guard(h, [&] {
-        SavedHeader hd{kMagic, h->W, h->N, h->od_J0, h->od_started ? 1ull : 0ull, h->g.m, h->seed,
-                       h->g.walk_len};
+        SavedHeader hd{kMagic,           h->W,           h->N,
+                       h->od_J0,         h->od_started ? 1ull : 0ull,
+                       h->g.m,           h->seed,        h->g.walk_len,
+                       h->g.burnin_len,  h->g.variant,   h->o.walker_base,
+                       h->o.bit_source};
         CK(cudaDeviceSynchronize());
         memcpy(host_buf, &hd, sizeof(hd));
         char *p = (char *)host_buf + sizeof(hd);
@@ -843,8 +862,12 @@ int prng_load(prng_t *h, const void *host_buf, size_t bytes) {
     SavedHeader hd;
     memcpy(&hd, host_buf, sizeof(hd));
     if (hd.magic != kMagic || hd.W != h->W || hd.m != h->g.m || hd.seed != h->seed ||
-        hd.walk_len != h->g.walk_len)
+        hd.walk_len != h->g.walk_len || hd.burnin_len != h->g.burnin_len ||
+        hd.variant != h->g.variant || hd.walker_base != h->o.walker_base ||
+        hd.bit_source != h->o.bit_source)
         return PRNG_E_INVALID;
+    // a resumed position must itself be reachable by the 32-bit draw cursor
+    if (hd.N > (0xFFFFFFFFull * h->W) || hd.od_J0 > 0xFFFFFFFFull) return PRNG_E_INVALID;
     if (h->od_open) return PRNG_E_STATE;
     return guard(h, [&] {
         CK(cudaDeviceSynchronize());
@@ -1061,85 +1084,3 @@ int prng_destroy(prng_t *h) {
 }
 
 }  // extern "C"
-
-// Diagnostic (not part of the ABI): time H2D copies from the handle's pinned
-// chunk 0 and from fresh pinned buffers allocated different ways.
-extern "C" int gg_debug_h2d_probe(prng_t *h, uint64_t bytes) {
-    if (!h || bytes > h->chunk_bytes) return PRNG_E_INVALID;
-    cudaSetDevice(h->o.device);
-    void *d = nullptr;
-    if (cudaMalloc(&d, bytes) != cudaSuccess) return PRNG_E_NOMEM;
-    cudaPointerAttributes at{};
-    cudaPointerGetAttributes(&at, h->chunk[0]);
-    fprintf(stderr, "[probe] chunk0 %p type %d devicePointer %p\n", (void *)h->chunk[0], (int)at.type,
-            at.devicePointer);
-    void *p_def = nullptr, *p_mh = nullptr, *p_reg = nullptr;
-    cudaHostAlloc(&p_def, bytes, cudaHostAllocDefault);
-    cudaMallocHost(&p_mh, bytes);
-    p_reg = aligned_alloc(4096, (bytes + 4095) / 4096 * 4096);
-    cudaHostRegister(p_reg, (bytes + 4095) / 4096 * 4096, cudaHostRegisterDefault);
-    memset(p_def, 1, bytes);
-    memset(p_mh, 1, bytes);
-    memset(p_reg, 1, bytes);
-    cudaEvent_t a, b;
-    cudaEventCreate(&a);
-    cudaEventCreate(&b);
-    const char *names[4] = {"chunk0(portable)", "hostalloc-default", "mallochost", "registered"};
-    void *srcs[4] = {h->chunk[0], p_def, p_mh, p_reg};
-    for (int k = 0; k < 4; k++) {
-        for (int rep = 0; rep < 3; rep++) {
-            cudaEventRecord(a, h->copy_stream);
-            cudaMemcpyAsync(d, srcs[k], bytes, cudaMemcpyHostToDevice, h->copy_stream);
-            cudaEventRecord(b, h->copy_stream);
-            cudaEventSynchronize(b);
-            float ms = 0;
-            cudaEventElapsedTime(&ms, a, b);
-            fprintf(stderr, "[probe] %-18s %.1f MB: %.3f ms (%.1f GB/s)\n", names[k], bytes / 1e6, ms,
-                    bytes / 1e6 / ms);
-        }
-    }
-    // copy right after the feed wrote the chunk: pool threads vs one thread
-    const uint64_t words = bytes / 4;
-    for (int mode = 0; mode < 3; mode++) {
-        for (int rep = 0; rep < 3; rep++) {
-            auto t0 = std::chrono::steady_clock::now();
-            if (mode == 0)
-                feed_chunk(h, 0, words / 6, 8, 6, h->chunk[0], nullptr, words / 6, true);
-            else if (mode == 1)
-                gg::feed_splitmix_rows(h->seed, 0, words / 6, 8, 6, h->chunk[0], words / 6);
-            else
-                memset(h->chunk[0], rep, bytes);
-            auto t1 = std::chrono::steady_clock::now();
-            cudaEventRecord(a, h->copy_stream);
-            cudaMemcpyAsync(d, h->chunk[0], bytes, cudaMemcpyHostToDevice, h->copy_stream);
-            cudaEventRecord(b, h->copy_stream);
-            cudaEventSynchronize(b);
-            float ms = 0;
-            cudaEventElapsedTime(&ms, a, b);
-            fprintf(stderr, "[probe] after %s write (%.3f ms): copy %.3f ms\n",
-                    mode == 0 ? "pool-feed" : mode == 1 ? "1-thread-feed" : "memset",
-                    std::chrono::duration<double, std::milli>(t1 - t0).count(), ms);
-        }
-    }
-    // same copy on a fresh default-flag stream
-    cudaStream_t s2;
-    cudaStreamCreate(&s2);
-    for (int rep = 0; rep < 3; rep++) {
-        cudaEventRecord(a, s2);
-        cudaMemcpyAsync(d, h->chunk[0], bytes, cudaMemcpyHostToDevice, s2);
-        cudaEventRecord(b, s2);
-        cudaEventSynchronize(b);
-        float ms = 0;
-        cudaEventElapsedTime(&ms, a, b);
-        fprintf(stderr, "[probe] chunk0 on new stream: %.3f ms\n", ms);
-    }
-    cudaStreamDestroy(s2);
-    cudaEventDestroy(a);
-    cudaEventDestroy(b);
-    cudaFreeHost(p_def);
-    cudaFreeHost(p_mh);
-    cudaHostUnregister(p_reg);
-    free(p_reg);
-    cudaFree(d);
-    return PRNG_OK;
-}

@@ -413,3 +413,68 @@ def test_non_power_of_two_fast_kernel_parity(torch_cuda, m):
     g.epoch_end()
     assert np.array_equal(as_u64(od).reshape(W, 2), want[: 2 * W].reshape(2, W).T)
     g.close()
+
+
+# ------------------------------------------- 32-bit draw cursor, checkpoints
+def test_draw_index_limit_refused_without_side_effects(torch_cuda):
+    """Draw indices are 32-bit in the kernels: a fill or prefetch reaching
+    draw 2^32 - 1 is refused with PRNG_E_UNSUPPORTED before anything is
+    enqueued.  Up to the limit the numbers are still
+    the oracle's: a walk of draw J's record (stream words 2 + R0 + 6J ..,
+    R9) from the saved walker state (checkpoint resume at N = J*W)."""
+    import struct
+    torch = torch_cuda
+    from paper_conf_ipps_banerjeebk12_b200 import PrngError
+    W, seed = 64, 5
+    g = G(walkers=W, seed=seed)
+    blob = bytearray(g.save())
+    J = (1 << 32) - 4
+    struct.pack_into("<Q", blob, 16, J * W)          # SavedHeader.N
+    g.load(bytes(blob))
+    assert g.tell() == J * W
+    big = torch.full((4 * W,), 7, dtype=torch.int64, device="cuda")
+    for call in (lambda: g.fill(big), lambda: g.prefetch(4),
+                 lambda: g.fill_host(torch.empty(4 * W, dtype=torch.int64).pin_memory())):
+        with pytest.raises(PrngError) as e:
+            call()
+        assert e.value.status == -2  # PRNG_E_UNSUPPORTED
+    torch.cuda.synchronize()
+    assert g.tell() == J * W and bool((big == 7).all())
+    # draws J .. J+2 (the last index 2^32 - 2 still fits): OK, oracle-exact
+    g.fill(big, n=3 * W)
+    assert g.tell() == (J + 3) * W
+    z = as_u64(big[:3 * W]).reshape(3, W)
+    hdr = 12 * 8
+    xs = np.frombuffer(bytes(blob), dtype=np.uint32, count=W, offset=hdr)
+    ys = np.frombuffer(bytes(blob), dtype=np.uint32, count=W, offset=hdr + 4 * W)
+    for t in (0, 37, W - 1):
+        x, y = int(xs[t]), int(ys[t])
+        for d in range(3):
+            k0 = 2 + 6 + 6 * (J + d)
+            rec = [O.stream_word32(seed, t, k0 + r) for r in range(6)]
+            x, y = O.walk(M32, x, y, rec, 64)
+            assert int(z[d, t]) == O.label(M32, x, y), (t, d)
+    with pytest.raises(PrngError) as e:
+        g.fill(big, n=1)                               # would need draw 2^32 - 1
+    assert e.value.status == -2
+    assert g.tell() == (J + 3) * W
+    g.close()
+
+
+@pytest.mark.parametrize("other", [dict(walker_base=64), dict(variant=1), dict(burnin_len=32),
+                                   dict(bit_source=1)])
+def test_checkpoint_refused_by_a_different_stream(torch_cuda, other):
+    """prng_load only into a handle that selects the same bit streams and walk
+    (rank 1 must not load rank 0's checkpoint silently)."""
+    from paper_conf_ipps_banerjeebk12_b200 import PrngError
+    W, seed = 64, 9
+    a = G(walkers=W, seed=seed)
+    blob = a.save()
+    b = G(walkers=W, seed=seed, **other)
+    with pytest.raises(PrngError) as e:
+        b.load(blob)
+    assert e.value.status == -1
+    assert b.tell() == 0
+    c = G(walkers=W, seed=seed)
+    c.load(blob)  # the same configuration loads
+    a.close(), b.close(), c.close()

@@ -83,3 +83,35 @@ def test_variant_bit_exact(var, want):
     # consume(): slot k's draws at [2k, 2k+1] (offsets = k * uniform)
     assert np.array_equal(np.array(got["od"], dtype=np.uint64).reshape(-1, 2), od), var
     assert got["tallies"] == [int(t) for t in tallies], var
+
+
+L1_SNIPPET = r"""
+import sys
+import numpy as np, torch
+sys.path.insert(0, %(root)r)
+from paper_conf_ipps_banerjeebk12_b200 import Generator
+W, seed = 32 * 700 + 5, 0x5EED00F1
+g = Generator(walkers=W, seed=seed, walk_len=1)
+g.prefetch(70)
+o = torch.empty(W * 70 - 3, dtype=torch.int64, device="cuda")
+g.fill(o)
+np.save(sys.argv[1], o.cpu().numpy().view(np.uint64))
+"""
+
+
+@pytest.mark.parametrize("var", ["GG_FILL_KPW=2", "GG_FILL_KPW=3", "GG_FILL_ONEWAVE=1",
+                                 "GG_L1_TMA_STORE=0"])
+def test_l1_tma_store_several_units_per_warp(var, tmp_path):
+    """l = 1 TMA-store kernel when a warp handles several 32-walker units
+    (the first interior tile of a unit must not overwrite a staging
+    buffer the previous unit's bulk store is still reading)."""
+    env = dict(os.environ)
+    k, v = var.split("=")
+    env[k] = v
+    f = str(tmp_path / "l1.npy")
+    out = subprocess.run([sys.executable, "-c", L1_SNIPPET % {"root": ROOT}, f], env=env,
+                         capture_output=True, text=True, timeout=300)
+    assert out.returncode == 0, out.stderr[-2000:]
+    got = np.load(f)
+    W = 32 * 700 + 5
+    assert np.array_equal(got, O.bulk(M32, 1, 64, 0x5EED00F1, W, 0, W * 70 - 3)), var
