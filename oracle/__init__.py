@@ -97,6 +97,8 @@ def _bind_optional(L):
         "or_mc_hg": (f64, [f64, f64]),
         "or_mc_fresnel": (f64, [f64, f64, f64, P]),
         "or_mc_q": (u64, [f64]),
+        "or_mc_refract": (None, [f64, f64, f64, P, P, P]),
+        "or_mc_spin": (None, [f64, f64, f64, P, P, P]),
     }
     for name, (res, args) in opt.items():
         fn = getattr(L, name, None)
@@ -284,3 +286,17 @@ def mc_fresnel(n1: float, n2: float, ca1: float):
     ca2 = np.zeros(1)
     r = lib().or_mc_fresnel(n1, n2, ca1, _ptr(ca2))
     return float(r), float(ca2[0])
+
+
+def mc_refract(n1: float, n2: float, ca2: float, u):
+    """Transmitted direction (or_mc_refract) of direction u = (ux, uy, uz)."""
+    v = [np.array([float(c)]) for c in u]
+    lib().or_mc_refract(n1, n2, ca2, _ptr(v[0]), _ptr(v[1]), _ptr(v[2]))
+    return tuple(float(c[0]) for c in v)
+
+
+def mc_spin(g: float, xi_theta: float, xi_psi: float, u):
+    """Direction after one scattering event (or_mc_spin) of direction u."""
+    v = [np.array([float(c)]) for c in u]
+    lib().or_mc_spin(g, xi_theta, xi_psi, _ptr(v[0]), _ptr(v[1]), _ptr(v[2]))
+    return tuple(float(c[0]) for c in v)
