@@ -63,50 +63,74 @@ __device__ __forceinline__ uint64_t mc_frac(uint64_t w, uint64_t q) {
     return (__umul64hi(w, q) << 32) | ((w * q) >> 32);
 }
 
-__device__ __forceinline__ double mc_hg(double g, double xi) {
-    double cost;
-    if (g == 0.0) {
-        cost = 2.0 * xi - 1.0;
-    } else {
-        double temp = (1.0 - g * g) / (1.0 - g + 2.0 * g * xi);
-        cost = (1.0 + g * g - temp * temp) / (2.0 * g);
-        if (cost < -1.0)
-            cost = -1.0;
-        else if (cost > 1.0)
-            cost = 1.0;
-    }
-    return cost;
+// Deflection cosine, Henyey-Greenstein phase function (§VI "the angles of
+// deflection"; CUDAMCML [1]).  The HG CDF in mu = cos(theta) is
+//   F(mu) = (1 - g^2) / (2g) * [(1 + g^2 - 2g mu)^(-1/2) - (1 + g)^(-1)],
+// and F(mu) = xi solves to sqrt(1 + g^2 - 2g mu) = (1 - g^2) / (1 + g (2xi - 1)).
+__device__ __forceinline__ double hg_cos_theta(double g, double xi) {
+    const double t = 2.0 * xi - 1.0;  // isotropic: mu uniform on [-1, 1]
+    if (g == 0.0) return t;
+    const double k = (1.0 - g * g) / (1.0 + g * t);
+    const double mu = (1.0 + g * g - k * k) / (2.0 * g);
+    return mu < -1.0 ? -1.0 : (mu > 1.0 ? 1.0 : mu);
 }
 
-__device__ __forceinline__ double mc_fresnel(double n1, double n2, double ca1, double *ca2) {
-    double r;
+// Unpolarised Fresnel reflectance from index n1 into n2 at incidence cosine
+// c1, as the mean of the squared s- and p-amplitude coefficients
+//   r_s = (n1 c1 - n2 c2) / (n1 c1 + n2 c2),  r_p = (n2 c1 - n1 c2) / (n2 c1 + n1 c2),
+// c2 = cos of the transmitted angle (Snell, n1 sin t1 = n2 sin t2), written to *c2_out.
+// Conventions shared with the oracle's reading (DESIGN R22): within 1e-12 of
+// normal incidence c2 = c1; below c1 = 1e-6 (grazing) and beyond the critical
+// angle the photon is reflected (R = 1, c2 = 0).
+__device__ __forceinline__ double fresnel_unpolarised(double n1, double n2, double c1,
+                                                      double *c2_out) {
     if (n1 == n2) {
-        *ca2 = ca1;
-        r = 0.0;
-    } else if (ca1 > 1.0 - 1.0e-12) {
-        *ca2 = ca1;
-        r = (n2 - n1) / (n2 + n1);
-        r = r * r;
-    } else if (ca1 < 1.0e-6) {
-        *ca2 = 0.0;
-        r = 1.0;
-    } else {
-        double sa1 = sqrt(1.0 - ca1 * ca1);
-        double sa2 = n1 * sa1 / n2;
-        if (sa2 >= 1.0) {
-            *ca2 = 0.0;
-            r = 1.0;
-        } else {
-            double c2 = sqrt(1.0 - sa2 * sa2);
-            double cap = ca1 * c2 - sa1 * sa2;
-            double cam = ca1 * c2 + sa1 * sa2;
-            double sap = sa1 * c2 + ca1 * sa2;
-            double sam = sa1 * c2 - ca1 * sa2;
-            *ca2 = c2;
-            r = 0.5 * sam * sam * (cam * cam + cap * cap) / (sap * sap * cam * cam);
-        }
+        *c2_out = c1;
+        return 0.0;
     }
-    return r;
+    double c2;
+    if (c1 > 1.0 - 1.0e-12) {
+        c2 = c1;
+    } else if (c1 < 1.0e-6) {
+        *c2_out = 0.0;
+        return 1.0;
+    } else {
+        const double s2 = n1 * sqrt(1.0 - c1 * c1) / n2;
+        if (s2 >= 1.0) {
+            *c2_out = 0.0;
+            return 1.0;
+        }
+        c2 = sqrt(1.0 - s2 * s2);
+    }
+    *c2_out = c2;
+    const double rs = (n1 * c1 - n2 * c2) / (n1 * c1 + n2 * c2);
+    const double rp = (n2 * c1 - n1 * c2) / (n2 * c1 + n1 * c2);
+    return 0.5 * (rs * rs + rp * rp);
+}
+
+// Scattering: rotate the unit direction u by the polar angle theta (cos =
+// cost) and the azimuth psi about u, in the orthonormal frame
+//   e1 = (ux uz, uy uz, -(1 - uz^2)) / sqrt(1 - uz^2),  e2 = (-uy, ux, 0) / sqrt(1 - uz^2):
+//   u' = cost u + sint (cos psi e1 + sin psi e2).
+// Near the poles (|uz| > 0.99999) the frame is (x, y, sign(uz) z).
+__device__ __forceinline__ void scatter_direction(double cost, double psi, double &ux, double &uy,
+                                                  double &uz) {
+    const double sint = sqrt(1.0 - cost * cost);
+    const double cp = cos(psi), sp = sin(psi);
+    if (fabs(uz) > 0.99999) {
+        ux = sint * cp;
+        uy = sint * sp;
+        uz = uz >= 0.0 ? cost : -cost;
+        return;
+    }
+    const double rho = sqrt(1.0 - uz * uz);
+    const double a = sint * cp / rho, b = sint * sp / rho;  // weights of rho*e1, rho*e2
+    const double nx = ux * cost + (a * ux * uz - b * uy);
+    const double ny = uy * cost + (a * uy * uz + b * ux);
+    const double nz = uz * cost - sint * cp * rho;
+    ux = nx;
+    uy = ny;
+    uz = nz;
 }
 
 __global__ void mc_init_state(McState s, uint64_t n, uint32_t *iota) {
@@ -203,7 +227,7 @@ __global__ void __launch_bounds__(128, MINB) mc_epoch(prng_view v, McParams P, M
                 const int nb = uz < 0.0 ? layer - 1 : layer + 1;
                 const double n1 = P.nidx[layer], n2 = P.nidx[nb];
                 double ca2;
-                const double r = mc_fresnel(n1, n2, fabs(uz), &ca2);
+                const double r = fresnel_unpolarised(n1, n2, fabs(uz), &ca2);
                 bool reflect = false;
                 if (n1 != n2) reflect = mc_xi(lb) <= r;
                 if (reflect) {
@@ -214,10 +238,11 @@ __global__ void __launch_bounds__(128, MINB) mc_epoch(prng_view v, McParams P, M
                     alive = false;
                 } else {
                     layer = nb;
-                    if (n1 != n2) {
-                        ux = ux * (n1 / n2);
-                        uy = uy * (n1 / n2);
-                        uz = uz > 0.0 ? ca2 : -ca2;
+                    if (n1 != n2) {  // Snell: tangential part scales by n1/n2, |uz| = cos t2
+                        const double eta = n1 / n2;
+                        ux *= eta;
+                        uy *= eta;
+                        uz = copysign(ca2, uz);
                     }
                 }
             } else {
@@ -228,21 +253,7 @@ __global__ void __launch_bounds__(128, MINB) mc_epoch(prng_view v, McParams P, M
                 const uint64_t dw = mc_frac(w, P.qabs[layer]);
                 w -= dw;
                 tally(kFixed + layer - 1, dw);
-                const double cost = mc_hg(g, mc_xi(lb));
-                const double psi = 2.0 * kPi * mc_xi(lc);
-                const double cosp = cos(psi), sinp = sin(psi);
-                const double sint = sqrt(1.0 - cost * cost);
-                const double ox = ux, oy = uy, oz = uz;
-                if (fabs(oz) > 0.99999) {
-                    ux = sint * cosp;
-                    uy = sint * sinp;
-                    uz = oz >= 0.0 ? cost : -cost;
-                } else {
-                    const double temp = sqrt(1.0 - oz * oz);
-                    ux = sint * (ox * oz * cosp - oy * sinp) / temp + ox * cost;
-                    uy = sint * (oy * oz * cosp + ox * sinp) / temp + oy * cost;
-                    uz = -sint * cosp * temp + oz * cost;
-                }
+                scatter_direction(hg_cos_theta(g, mc_xi(lb)), 2.0 * kPi * mc_xi(lc), ux, uy, uz);
                 interactions++;
                 if (w < P.w_th) {
                     tally(4, w);
