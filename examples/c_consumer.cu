@@ -29,12 +29,13 @@
         }                                                                               \
     } while (0)
 
-__global__ void user_kernel(prng_view v, uint32_t walkers, unsigned long long *out) {
+__global__ void user_kernel(const __grid_constant__ prng_view v, uint32_t walkers,
+                            unsigned long long *out) {
     const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= walkers) return;
     prng_state st = prng_state_load(&v, t);
     const uint32_t calls = t % 3u + 1u;  // data-dependent demand
-    for (uint32_t i = 0; i < calls; i++) out[(size_t)t * 3 + i] = prng_next(&st, &v);
+    for (uint32_t i = 0; i < calls; i++) out[(size_t)t * 3 + i] = prng_next(&st);  // north_star's prng_next(&state)
     prng_state_store(&v, &st);
 }
 

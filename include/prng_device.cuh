@@ -1,15 +1,19 @@
 /*
  * include/prng_device.cuh — header-only device side of the expander-walk PRNG.
  *
- *   prng_next(&state, view)  = Alg.2 GetNextRand (§III-B) called by any
+ *   prng_next(&state)  = Alg.2 GetNextRand (§III-B) called by any
  *   GPU thread "at any point of time" (§III): l = 64 steps of the walk on
  *   the 7-regular Gabber–Galil expander (§III-A), 3 bits per step, and
  *   the walker's vertex label returned as a 64-bit number (§III-B).
  *
- * Usage inside a user kernel (after prng_epoch_begin + prng_device_view):
+ * Usage inside a user kernel (after prng_epoch_begin + prng_device_view;
+ * pass the view as a __grid_constant__ kernel parameter):
  *     prng_state st = prng_state_load(&view, slot);   // slot = walker by default
- *     uint64_t r = prng_next(&st, &view);      // as often as the epoch allows
+ *     uint64_t r = prng_next(&st);             // as often as the epoch allows
  *     prng_state_store(&view, &st);
+ * prng_next(&st, &view) is the same call with the view named explicitly, and
+ * prng_next<PRNG_WALK_L64>(...) compiles in only the paper's l = 64, m = 2^k
+ * walk (the host picks the mode with prng_walk_mode(&view); see below).
  * A walker must be used by one thread at a time (that is what makes the
  * generator thread-safe, §I-B).  A draw outside the epoch window sets a
  * sticky flag (read by prng_check) and returns 0 — never different bits.
@@ -50,6 +54,7 @@ struct prng_state {
     uint32_t walker;   /* walker id (handle-local): index of the state arrays */
     uint32_t slot;     /* column of the epoch window holding this walker's bits */
     uint32_t used;     /* draws consumed in this epoch */
+    const struct prng_view *view;  /* the view it was loaded from (one-argument prng_next) */
 };
 
 /* ------------------------------------------------------------------------
@@ -539,6 +544,7 @@ __device__ __forceinline__ prng_state prng_state_load(const prng_view *v, uint32
     st.y = v->y[walker];
     st.walker = walker;
     st.slot = slot;
+    st.view = v;
     const uint32_t j = v->j[walker];
     st.used = (j > v->J0) ? (j - v->J0) : 0u; /* walkers that skipped epochs jump to J0 */
     return st;
@@ -557,7 +563,60 @@ __device__ __forceinline__ uint32_t prng_available(const prng_view *v, const prn
     return (st->used < v->D) ? (v->D - st->used) : 0u;
 }
 
-/* Alg.2 GetNextRand: walk l steps with the bits of draw (J0 + used). */
+/* Walk implementations prng_next can use, picked from the view's (m, l,
+ * variant, l0).  A kernel that knows its generator's shape instantiates
+ * prng_next<MODE> so only that walk is compiled into it; prng_next without a
+ * mode (PRNG_WALK_AUTO) dispatches at run time over all of them.  Every mode
+ * returns the same numbers as the generic walk for the views it accepts. */
+enum {
+    PRNG_WALK_AUTO = 0,      /* run-time dispatch (any view) */
+    PRNG_WALK_L64 = 1,       /* l = 64, m = 2^k, forward maps (the paper's generator) */
+    PRNG_WALK_L64_BIP = 2,   /* l = 64, m = 2^k, bipartite, l0 even (draws start at even steps) */
+    PRNG_WALK_ANY_POW2 = 3,  /* any l, m = 2^k, forward maps */
+    PRNG_WALK_L64_MOD = 4,   /* l = 64, m <= 2^30 not a power of two, forward maps */
+    PRNG_WALK_GENERIC = 5    /* anything (per-step field loads, conditional-subtract mod m) */
+};
+
+/* The fastest mode that is exact for this view (host or device). */
+static inline __host__ __device__ int prng_walk_mode(const prng_view *v)
+{
+    if (v->l == 64u && v->pow2 && v->variant == 0) return PRNG_WALK_L64;
+    if (v->l == 64u && v->pow2 && v->variant == 1 && (v->l0 & 1u) == 0) return PRNG_WALK_L64_BIP;
+    if (v->pow2 && v->variant == 0) return PRNG_WALK_ANY_POW2;
+    if (v->l == 64u && v->variant == 0 && v->m <= (1ull << 30)) return PRNG_WALK_L64_MOD;
+    return PRNG_WALK_GENERIC;
+}
+
+/* One walk of l steps from (x, y) with the record at rec (column stride
+ * pitch), in walk mode MODE (not AUTO). */
+template <int MODE>
+__device__ __forceinline__ void prng_walk_mode_apply(const prng_view *v, const uint32_t *rec,
+                                                     uint32_t draw_in_window, uint32_t &x,
+                                                     uint32_t &y)
+{
+    if (MODE == PRNG_WALK_L64 || MODE == PRNG_WALK_L64_BIP || MODE == PRNG_WALK_L64_MOD) {
+        uint32_t w[6];
+#pragma unroll
+        for (int r = 0; r < 6; r++)
+            w[r] = __ldg(rec + (uint64_t)r * v->pitch);
+        if (MODE == PRNG_WALK_L64)
+            gg_walk64_r2p(w, x, y);
+        else if (MODE == PRNG_WALK_L64_BIP)
+            gg_walk64_r2p<true>(w, x, y);  /* draw starts at global step l0 + 64 j: even */
+        else
+            gg_walk64_r2p_mod(w, (uint32_t)v->m, x, y);
+    } else if (MODE == PRNG_WALK_ANY_POW2) {
+        gg_walk_r2p_any(rec, v->pitch, v->l, v->R, x, y);
+    } else {
+        const uint64_t s0 = (uint64_t)v->l0 + (uint64_t)v->l * (v->J0 + draw_in_window);
+        gg_walk_generic(rec, v->pitch, v->l, x, y, (uint32_t)v->m, v->pow2 != 0, v->variant, s0);
+    }
+}
+
+/* Alg.2 GetNextRand: walk l steps with the bits of draw (J0 + used).
+ * MODE = PRNG_WALK_AUTO picks the walk at run time; a fixed MODE must be
+ * prng_walk_mode(v) (or PRNG_WALK_GENERIC, which accepts any view). */
+template <int MODE = PRNG_WALK_AUTO>
 __device__ __forceinline__ uint64_t prng_next(prng_state *st, const prng_view *v)
 {
     if (st->used >= v->D || st->slot >= v->Wv) {
@@ -566,44 +625,55 @@ __device__ __forceinline__ uint64_t prng_next(prng_state *st, const prng_view *v
     }
     const uint32_t *rec = v->bits + (uint64_t)st->used * v->R * v->pitch + st->slot;
     uint32_t x = st->x, y = st->y;
-    if (v->l == 64u && v->pow2 && (v->variant == 0 || (v->variant == 1 && (v->l0 & 1u) == 0))) {
-        uint32_t w[6];
-#pragma unroll
-        for (int r = 0; r < 6; r++)
-            w[r] = __ldg(rec + (uint64_t)r * v->pitch);
-        if (v->variant == 0)
-            gg_walk64_r2p(w, x, y);
-        else
-            gg_walk64_r2p<true>(w, x, y);  /* draw starts at global step l0 + 64 j: even */
-    } else if (v->pow2 && v->variant == 0) {
-        gg_walk_r2p_any(rec, v->pitch, v->l, v->R, x, y);
-    } else if (v->l == 64u && v->variant == 0 && v->m <= (1ull << 30)) {
-        uint32_t w[6];
-#pragma unroll
-        for (int r = 0; r < 6; r++)
-            w[r] = __ldg(rec + (uint64_t)r * v->pitch);
-        gg_walk64_r2p_mod(w, (uint32_t)v->m, x, y);
+    if (MODE == PRNG_WALK_AUTO) {
+        switch (prng_walk_mode(v)) {
+        case PRNG_WALK_L64: prng_walk_mode_apply<PRNG_WALK_L64>(v, rec, st->used, x, y); break;
+        case PRNG_WALK_L64_BIP:
+            prng_walk_mode_apply<PRNG_WALK_L64_BIP>(v, rec, st->used, x, y);
+            break;
+        case PRNG_WALK_ANY_POW2:
+            prng_walk_mode_apply<PRNG_WALK_ANY_POW2>(v, rec, st->used, x, y);
+            break;
+        case PRNG_WALK_L64_MOD:
+            prng_walk_mode_apply<PRNG_WALK_L64_MOD>(v, rec, st->used, x, y);
+            break;
+        default: prng_walk_mode_apply<PRNG_WALK_GENERIC>(v, rec, st->used, x, y); break;
+        }
     } else {
-        const uint64_t s0 = (uint64_t)v->l0 + (uint64_t)v->l * (v->J0 + st->used);
-        gg_walk_generic(rec, v->pitch, v->l, x, y, (uint32_t)v->m, v->pow2 != 0, v->variant, s0);
+        prng_walk_mode_apply<MODE>(v, rec, st->used, x, y);
     }
     st->x = x;
     st->y = y;
     st->used++;
-    return gg_label(x, y, v->m, v->log2m, v->pow2 != 0);
+    const bool pow2 = (MODE == PRNG_WALK_L64 || MODE == PRNG_WALK_L64_BIP ||
+                       MODE == PRNG_WALK_ANY_POW2) ? true
+                      : (MODE == PRNG_WALK_L64_MOD) ? false : (v->pow2 != 0);
+    return gg_label(x, y, v->m, v->log2m, pow2);
+}
+
+/* north_star's one-argument form prng_next(&state): the state remembers the
+ * view it was loaded from (prng_state_load).  Same numbers as
+ * prng_next(&state, view). */
+template <int MODE = PRNG_WALK_AUTO>
+__device__ __forceinline__ uint64_t prng_next(prng_state *st)
+{
+    return prng_next<MODE>(st, st->view);
 }
 
 /* K draws at once: the K records' loads are issued together before the
  * first walk, so a consumer that needs several numbers per iteration (the
  * Monte Carlo consumer takes three) waits for memory once, not K times.
- * Same numbers, same order, same overrun rule as K calls of prng_next. */
-template <int K, bool ROLL = false>
+ * Same numbers, same order, same overrun rule as K calls of prng_next.
+ * The batched form needs l = 64, m = 2^k, forward maps (MODE L64, or AUTO
+ * on such a view); every other view takes K single calls. */
+template <int K, bool ROLL = false, int MODE = PRNG_WALK_AUTO>
 __device__ __forceinline__ void prng_next_n(prng_state *st, const prng_view *v, uint64_t (&out)[K])
 {
-    if (!(v->l == 64u && v->pow2 && v->variant == 0) || st->used + K > v->D ||
-        st->slot >= v->Wv) {
+    const bool l64 = MODE == PRNG_WALK_L64 ||
+                     (MODE == PRNG_WALK_AUTO && prng_walk_mode(v) == PRNG_WALK_L64);
+    if (!l64 || st->used + K > v->D || st->slot >= v->Wv) {
 #pragma unroll
-        for (int k = 0; k < K; k++) out[k] = prng_next(st, v);
+        for (int k = 0; k < K; k++) out[k] = prng_next<MODE>(st, v);
         return;
     }
     uint32_t w[K][6];

@@ -12,7 +12,12 @@
 
 namespace {
 
-__global__ void __launch_bounds__(128) consume_kernel(prng_view v, uint64_t threads,
+// MODE: the walk compiled into this instantiation (prng_walk_mode of the
+// view, picked on the host), so the hot loop holds one walk, not the
+// run-time dispatch over all of them.
+template <int MODE>
+__global__ void __launch_bounds__(128) consume_kernel(const __grid_constant__ prng_view v,
+                                                      uint64_t threads,
                                                       const uint32_t *counts, uint32_t uniform,
                                                       uint64_t *out, const uint64_t *offsets,
                                                       uint64_t *xor_out) {
@@ -29,7 +34,7 @@ __global__ void __launch_bounds__(128) consume_kernel(prng_view v, uint64_t thre
     uint32_t r = 0;
     for (; r + 4 <= c; r += 4) {  // four records' loads in flight together
         uint64_t z4[4];
-        prng_next_n<4>(&st, &v, z4);
+        prng_next_n<4, false, MODE>(&st, &v, z4);
 #pragma unroll
         for (int k = 0; k < 4; k++) {
             acc ^= z4[k];
@@ -37,7 +42,7 @@ __global__ void __launch_bounds__(128) consume_kernel(prng_view v, uint64_t thre
         }
     }
     for (; r < c; r++) {
-        const uint64_t z = prng_next(&st, &v);
+        const uint64_t z = prng_next<MODE>(&st, &v);
         acc ^= z;
         if (out) out[base + r] = z;
     }
@@ -60,7 +65,17 @@ extern "C" int gg_consume(prng_t *h, uint64_t threads, const uint32_t *counts, u
     if (mis(counts, 4) || mis(out, 8) || mis(offsets, 8) || mis(xor_out, 8)) return PRNG_E_INVALID;
     const uint32_t tpb = 128;
     const uint64_t blocks = (threads + tpb - 1) / tpb;
-    consume_kernel<<<(unsigned)blocks, tpb, 0, (cudaStream_t)stream>>>(v, threads, counts, uniform,
-                                                                       out, offsets, xor_out);
+    cudaStream_t st = (cudaStream_t)stream;
+#define GG_CONSUME(M)                                                                        \
+    consume_kernel<M><<<(unsigned)blocks, tpb, 0, st>>>(v, threads, counts, uniform, out, offsets, \
+                                                        xor_out)
+    switch (prng_walk_mode(&v)) {
+    case PRNG_WALK_L64: GG_CONSUME(PRNG_WALK_L64); break;
+    case PRNG_WALK_L64_BIP: GG_CONSUME(PRNG_WALK_L64_BIP); break;
+    case PRNG_WALK_ANY_POW2: GG_CONSUME(PRNG_WALK_ANY_POW2); break;
+    case PRNG_WALK_L64_MOD: GG_CONSUME(PRNG_WALK_L64_MOD); break;
+    default: GG_CONSUME(PRNG_WALK_GENERIC); break;
+    }
+#undef GG_CONSUME
     return cudaGetLastError() == cudaSuccess ? PRNG_OK : PRNG_E_CUDA;
 }

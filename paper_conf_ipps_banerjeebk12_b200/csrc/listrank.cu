@@ -63,12 +63,15 @@ __global__ void lr_find_tail(int64_t n, const int32_t *succ, int32_t *tail) {
 }
 
 // Alg.3 l.6-7: temp = getnextrand(); b(u) = bit 63 of temp.
-__global__ void __launch_bounds__(128) lr_draw(prng_view v, const int32_t *act, int64_t A,
-                                               uint8_t *bit) {
+// MODE: PRNG_WALK_L64 for the paper's generator (only that walk compiled in),
+// PRNG_WALK_AUTO (run-time dispatch) for other graph parameters.
+template <int MODE>
+__global__ void __launch_bounds__(128) lr_draw(const __grid_constant__ prng_view v,
+                                               const int32_t *act, int64_t A, uint8_t *bit) {
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= A) return;
     prng_state st = prng_state_load(&v, (uint32_t)i);
-    const uint64_t z = prng_next(&st, &v);
+    const uint64_t z = prng_next<MODE>(&st, &v);
     prng_state_store(&v, &st);
     bit[act[i]] = (uint8_t)(z >> 63);
 }
@@ -101,13 +104,15 @@ __global__ void lr_splice(const int32_t *act, int64_t A, const uint8_t *keep, in
 }
 
 // Phase II splitter choice (R18).
-__global__ void __launch_bounds__(128) lr_splitter_draw(prng_view v, const int32_t *act, int64_t A,
+template <int MODE>
+__global__ void __launch_bounds__(128) lr_splitter_draw(const __grid_constant__ prng_view v,
+                                                        const int32_t *act, int64_t A,
                                                         int32_t head, uint8_t *spl_node,
                                                         uint8_t *spl_slot, int32_t *spl_out) {
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= A) return;
     prng_state st = prng_state_load(&v, (uint32_t)i);
-    const uint64_t z = prng_next(&st, &v);
+    const uint64_t z = prng_next<MODE>(&st, &v);
     prng_state_store(&v, &st);
     const int32_t u = act[i];
     const uint8_t s = (u == head || (z >> 58) == 0) ? 1 : 0;
@@ -320,7 +325,10 @@ extern "C" int gg_list_rank(prng_t *h, int64_t n, const int32_t *succ, const int
             auto tq = std::chrono::steady_clock::now();
             sync_t("copy-wait", tq);
             LRC(prng_device_view(h, &view, sizeof(view)));
-            lr_draw<<<nblk(A, 128), 128, 0, s>>>(view, act, A, bit);
+            if (prng_walk_mode(&view) == PRNG_WALK_L64)
+                lr_draw<PRNG_WALK_L64><<<nblk(A, 128), 128, 0, s>>>(view, act, A, bit);
+            else
+                lr_draw<PRNG_WALK_AUTO><<<nblk(A, 128), 128, 0, s>>>(view, act, A, bit);
             LRC(prng_epoch_end(h, s));
             sync_t("draw", tq);
             draws += A;
@@ -368,8 +376,12 @@ extern "C" int gg_list_rank(prng_t *h, int64_t n, const int32_t *succ, const int
         LRC(prng_epoch_begin(h, (uint64_t)A, 1, s));
         LRC(prng_device_view(h, &view, sizeof(view)));
         LCK(cudaMemsetAsync(spl_node, 0, n, s));
-        lr_splitter_draw<<<nblk(A, 128), 128, 0, s>>>(view, act, A, (int32_t)head, spl_node, keep,
-                                                      is_splitter);
+        if (prng_walk_mode(&view) == PRNG_WALK_L64)
+            lr_splitter_draw<PRNG_WALK_L64><<<nblk(A, 128), 128, 0, s>>>(
+                view, act, A, (int32_t)head, spl_node, keep, is_splitter);
+        else
+            lr_splitter_draw<PRNG_WALK_AUTO><<<nblk(A, 128), 128, 0, s>>>(
+                view, act, A, (int32_t)head, spl_node, keep, is_splitter);
         LRC(prng_epoch_end(h, s));
         draws += A;
         LCK(cub::DeviceSelect::Flagged(tmp, tmp_bytes, act, keep, act2, d_num, (int)A, s));

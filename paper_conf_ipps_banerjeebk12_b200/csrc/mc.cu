@@ -150,8 +150,11 @@ __global__ void mc_init_state(McState s, uint64_t n, uint32_t *iota) {
     iota[i] = (uint32_t)i;
 }
 
-template <int MINB>
-__global__ void __launch_bounds__(128, MINB) mc_epoch(prng_view v, McParams P, McState S,
+// MODE: PRNG_WALK_L64 for the paper's generator (only that walk compiled into
+// the epoch loop), PRNG_WALK_AUTO (run-time dispatch) for other parameters.
+template <int MINB, int MODE>
+__global__ void __launch_bounds__(128, MINB) mc_epoch(const __grid_constant__ prng_view v,
+                                                      McParams P, McState S,
                                                 unsigned long long *tallies,
                                                 long long *per_thread,
                                                 unsigned long long *counters) {
@@ -185,7 +188,7 @@ __global__ void __launch_bounds__(128, MINB) mc_epoch(prng_view v, McParams P, M
             if (!alive && launched == budget) break;
             // three draws at a convergent point (R22), their loads in flight together
             uint64_t d3[3];
-            prng_next_n<3, true>(&st, &v, d3);
+            prng_next_n<3, true, MODE>(&st, &v, d3);
             const uint64_t la = d3[0], lb = d3[1], lc = d3[2];
             draws += 3;
             if (!alive) {
@@ -287,6 +290,21 @@ __global__ void __launch_bounds__(128, MINB) mc_epoch(prng_view v, McParams P, M
         for (int o = 16; o > 0; o >>= 1) vsum += __shfl_down_sync(full, vsum, o);
         if ((threadIdx.x & 31) == 0 && vsum) atomicAdd(&counters[k], vsum);
     }
+}
+
+// GG_MC_MINB hook: blocks per SM in the register budget (default 8).
+template <int MODE>
+void launch_epoch(int minb, unsigned grid, cudaStream_t s, const prng_view &v, const McParams &P,
+                  const McState &S, unsigned long long *tal, long long *per_thread,
+                  unsigned long long *cnt) {
+    if (minb >= 12)
+        mc_epoch<12, MODE><<<grid, 128, 0, s>>>(v, P, S, tal, per_thread, cnt);
+    else if (minb >= 8)
+        mc_epoch<8, MODE><<<grid, 128, 0, s>>>(v, P, S, tal, per_thread, cnt);
+    else if (minb >= 6)
+        mc_epoch<6, MODE><<<grid, 128, 0, s>>>(v, P, S, tal, per_thread, cnt);
+    else
+        mc_epoch<4, MODE><<<grid, 128, 0, s>>>(v, P, S, tal, per_thread, cnt);
 }
 
 struct Fail {
@@ -409,27 +427,13 @@ extern "C" int gg_mc_run(prng_t *h, const gg_mc_config *cfg, int64_t *tallies, i
                 MRC(prng_device_view(h, &v, sizeof(v)));
                 MCK(cudaEventRecord(k0, s));
                 static const int minb = getenv("GG_MC_MINB") ? atoi(getenv("GG_MC_MINB")) : 8;
-                if (minb >= 12)
-                    mc_epoch<12><<<(unsigned)((wslots + 127) / 128), 128, 0, s>>>(
-                        v, P, S, d_tal, (long long *)per_thread, d_cnt);
-                else if (minb >= 10)
-                    mc_epoch<10><<<(unsigned)((wslots + 127) / 128), 128, 0, s>>>(
-                        v, P, S, d_tal, (long long *)per_thread, d_cnt);
-                else if (minb >= 8)
-                    mc_epoch<8><<<(unsigned)((wslots + 127) / 128), 128, 0, s>>>(
-                        v, P, S, d_tal, (long long *)per_thread, d_cnt);
-                else if (minb == 7)
-                    mc_epoch<7><<<(unsigned)((wslots + 127) / 128), 128, 0, s>>>(
-                        v, P, S, d_tal, (long long *)per_thread, d_cnt);
-                else if (minb >= 6)
-                    mc_epoch<6><<<(unsigned)((wslots + 127) / 128), 128, 0, s>>>(
-                        v, P, S, d_tal, (long long *)per_thread, d_cnt);
-                else if (minb == 5)
-                    mc_epoch<5><<<(unsigned)((wslots + 127) / 128), 128, 0, s>>>(
-                        v, P, S, d_tal, (long long *)per_thread, d_cnt);
+                const unsigned grid = (unsigned)((wslots + 127) / 128);
+                if (prng_walk_mode(&v) == PRNG_WALK_L64)
+                    launch_epoch<PRNG_WALK_L64>(minb, grid, s, v, P, S, d_tal,
+                                                (long long *)per_thread, d_cnt);
                 else
-                    mc_epoch<4><<<(unsigned)((wslots + 127) / 128), 128, 0, s>>>(
-                        v, P, S, d_tal, (long long *)per_thread, d_cnt);
+                    launch_epoch<PRNG_WALK_AUTO>(minb, grid, s, v, P, S, d_tal,
+                                                 (long long *)per_thread, d_cnt);
                 MCK(cudaGetLastError());
                 MCK(cudaEventRecord(k1, s));
                 MRC(prng_epoch_end(h, s));
