@@ -81,6 +81,18 @@ void feed_ggcpu_rows(uint64_t seed, uint64_t base, uint64_t l0, const uint32_t *
 // pitch `pitch`) ahead of prng_epoch_begin (prng_capi.cu); list ranking.
 int epoch_prefeed(prng_s *h, uint64_t hi, uint64_t pitch);
 
+// Stable single-pass compaction (compact.cu): items i < n with flags[i] != 0
+// go, in order, to kept_out (the item is in[i], or i when in is null); the
+// others, in order, to removed_out (if not null).  The kept count is written
+// to *d_count and, if h_count (mapped pinned host memory) is given, as
+// (tag << 32 | count) to *h_count once the count is final, for the host to
+// poll without a device synchronisation.  scratch: compact_scratch_bytes(n)
+// bytes of device memory, reset on the stream by every call.
+size_t compact_scratch_bytes(int64_t n);
+cudaError_t compact_flagged(const int32_t *in, const uint8_t *flags, int64_t n, int32_t *kept_out,
+                            int32_t *removed_out, int32_t *d_count, volatile uint64_t *h_count,
+                            uint32_t tag, void *scratch, cudaStream_t s);
+
 // Library-owned stream-ordered scratch pool of the current device (listrank.cu):
 // keeps its memory between calls; nullptr on CUDA failure.
 cudaMemPool_t scratch_pool();

@@ -5,8 +5,10 @@
 //   lr_draw   : active slot i (walker i) calls prng_next; b(u) = bit 63 (R13)
 //   lr_decide : u leaves iff b(u)=1, b(pred)=0, b(succ)=0, u not head/tail (R14)
 //   lr_splice : splice u out; remember (pred, distance) for Phase III
-//   cub::DevicePartition::Flagged : stable compaction of the survivors; the
-//               removed nodes of the round go to the re-insertion log
+//   gg::compact_flagged : stable single-pass compaction of the survivors
+//               (compact.cu); the removed nodes of the round go straight to
+//               the re-insertion log, the survivor count to mapped host
+//               memory that the host polls while it stages the next round
 //   repeat until active <= ceil(n / floor(log2 n)) (R15).  The host learns the
 //   new active count each round and the feed supplies exactly that many draws
 //   (on demand, instead of [3]'s upper-bound pre-generation).
@@ -24,7 +26,9 @@
 #include <mutex>
 #include <vector>
 
-#include <cub/cub.cuh>
+#include <atomic>
+#include <thread>
+
 #include <cuda_runtime.h>
 
 #include "gg_apps.h"
@@ -218,6 +222,59 @@ __global__ void lr_reinsert(const int32_t *list, int64_t cnt, const int32_t *rem
 
 inline unsigned nblk(int64_t n, int t = 256) { return (unsigned)((n + t - 1) / t); }
 
+// Mapped pinned 8-byte slots the compaction kernel writes its count into
+// (one per concurrent gg_list_rank call; allocated in blocks, never freed).
+struct CountSlot {
+    volatile uint64_t *p = nullptr;
+    CountSlot() {
+        std::lock_guard<std::mutex> lk(mu());
+        if (free_list().empty()) {
+            void *blk = nullptr;
+            if (cudaHostAlloc(&blk, 64 * 64, cudaHostAllocMapped | cudaHostAllocPortable) !=
+                cudaSuccess)
+                throw Fail{PRNG_E_NOMEM};
+            for (int i = 0; i < 64; i++)
+                free_list().push_back((volatile uint64_t *)((char *)blk + 64 * i));
+        }
+        p = free_list().back();
+        free_list().pop_back();
+    }
+    ~CountSlot() {
+        std::lock_guard<std::mutex> lk(mu());
+        free_list().push_back(p);
+    }
+    static std::mutex &mu() {
+        static std::mutex m;
+        return m;
+    }
+    static std::vector<volatile uint64_t *> &free_list() {
+        static std::vector<volatile uint64_t *> v;
+        return v;
+    }
+};
+
+std::atomic<uint32_t> g_tag{1};
+
+// Wait until the compaction kernel tagged `tag` has published its count
+// (polling mapped host memory, no stream synchronisation); CUDA errors on the
+// stream end the wait.
+int32_t wait_count(volatile uint64_t *slot, uint32_t tag, cudaStream_t s) {
+    for (uint32_t spin = 0;; spin++) {
+        const uint64_t v = *slot;
+        if ((uint32_t)(v >> 32) == tag) return (int32_t)(uint32_t)v;
+        if ((spin & 255u) == 255u) {
+            const cudaError_t e = cudaStreamQuery(s);
+            if (e != cudaSuccess && e != cudaErrorNotReady) throw Fail{PRNG_E_CUDA};
+            if (e == cudaSuccess) {
+                const uint64_t w = *slot;  // the stream is done: the value must be there
+                if ((uint32_t)(w >> 32) == tag) return (int32_t)(uint32_t)w;
+                throw Fail{PRNG_E_CUDA};
+            }
+            std::this_thread::yield();
+        }
+    }
+}
+
 }  // namespace
 
 // Stream-ordered scratch pool of this library, one per device, that keeps its
@@ -288,12 +345,8 @@ extern "C" int gg_list_rank(prng_t *h, int64_t n, const int32_t *succ, const int
         lr_find_tail<<<nblk(n), 256, 0, s>>>(n, d_succ, d_num + 1);
         int32_t tail = -1;
         LCK(cudaMemcpyAsync(&tail, d_num + 1, 4, cudaMemcpyDeviceToHost, s));
-        size_t tmp_bytes = 0;
-        LCK(cub::DevicePartition::Flagged(nullptr, tmp_bytes, act, keep, act2, d_num, (int)n, s));
-        size_t tmp2 = 0;
-        LCK(cub::DeviceSelect::Flagged(nullptr, tmp2, act, keep, act2, d_num, (int)n, s));
-        if (tmp2 > tmp_bytes) tmp_bytes = tmp2;
-        void *tmp = alloc(tmp_bytes);
+        void *tmp = alloc(gg::compact_scratch_bytes(n));
+        CountSlot slot;
         LCK(cudaStreamSynchronize(s));
         if (tail < 0) throw Fail{PRNG_E_INVALID};
 
@@ -336,7 +389,9 @@ extern "C" int gg_list_rank(prng_t *h, int64_t n, const int32_t *succ, const int
             lr_splice<<<nblk(A), 256, 0, s>>>(act, A, keep, d_pred, d_succ, w, rem_pred, rem_dist,
                                               removed_round, (int32_t)rounds);
             sync_t("decide+splice", tq);
-            LCK(cub::DevicePartition::Flagged(tmp, tmp_bytes, act, keep, act2, d_num, (int)A, s));
+            const uint32_t tag = g_tag.fetch_add(1);
+            LCK(gg::compact_flagged(act, keep, A, act2, rem_log + log_off, d_num, slot.p, tag, tmp,
+                                    s));
             sync_t("partition", tq);
             // While this round's kernels run, stage the next round's bits for the
             // slots that certainly stay active: an interior node is removed with
@@ -350,9 +405,7 @@ extern "C" int gg_list_rank(prng_t *h, int64_t n, const int32_t *succ, const int
                 const int64_t lo = (int64_t)(0.875 * (double)A - 8.0 * sd);
                 if (lo > 0) LRC(gg::epoch_prefeed(h, (uint64_t)lo, ((uint64_t)A + 31) / 32 * 32));
             }
-            int32_t kept = 0;
-            LCK(cudaMemcpyAsync(&kept, d_num, 4, cudaMemcpyDeviceToHost, s));
-            LCK(cudaStreamSynchronize(s));
+            const int32_t kept = wait_count(slot.p, tag, s);
             if (trace) {
                 auto tr2 = std::chrono::steady_clock::now();
                 fprintf(stderr, "[lr] round %ld A=%ld feed+enqueue %.3f ms, kernels+sync %.3f ms\n",
@@ -361,8 +414,6 @@ extern "C" int gg_list_rank(prng_t *h, int64_t n, const int32_t *succ, const int
                         std::chrono::duration<double, std::milli>(tr2 - tr1).count());
             }
             const int64_t gone = A - kept;
-            LCK(cudaMemcpyAsync(rem_log + log_off, act2 + kept, (size_t)gone * 4,
-                                cudaMemcpyDeviceToDevice, s));
             round_off.push_back(log_off);
             round_cnt.push_back(gone);
             log_off += gone;
@@ -384,10 +435,9 @@ extern "C" int gg_list_rank(prng_t *h, int64_t n, const int32_t *succ, const int
                 view, act, A, (int32_t)head, spl_node, keep, is_splitter);
         LRC(prng_epoch_end(h, s));
         draws += A;
-        LCK(cub::DeviceSelect::Flagged(tmp, tmp_bytes, act, keep, act2, d_num, (int)A, s));
-        int32_t ns = 0;
-        LCK(cudaMemcpyAsync(&ns, d_num, 4, cudaMemcpyDeviceToHost, s));
-        LCK(cudaStreamSynchronize(s));
+        const uint32_t tag2 = g_tag.fetch_add(1);
+        LCK(gg::compact_flagged(act, keep, A, act2, nullptr, d_num, slot.p, tag2, tmp, s));
+        const int32_t ns = wait_count(slot.p, tag2, s);
         int32_t *spl = act2;
         int32_t *spl_idx = (int32_t *)alloc(n4);
         int32_t *local = (int32_t *)alloc(n4), *sub = (int32_t *)alloc(n4);

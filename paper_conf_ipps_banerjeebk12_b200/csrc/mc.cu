@@ -20,7 +20,6 @@
 #include <cstdlib>
 #include <vector>
 
-#include <cub/cub.cuh>
 #include <cuda_runtime.h>
 
 #include "gg_apps.h"
@@ -133,7 +132,7 @@ __device__ __forceinline__ void scatter_direction(double cost, double psi, doubl
     uz = nz;
 }
 
-__global__ void mc_init_state(McState s, uint64_t n, uint32_t *iota) {
+__global__ void mc_init_state(McState s, uint64_t n) {
     const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= n) return;
     s.alive[i] = 0;
@@ -147,7 +146,6 @@ __global__ void mc_init_state(McState s, uint64_t n, uint32_t *iota) {
     s.sleft[i] = 0.0;
     s.layer[i] = 0;
     s.busy[i] = 1;
-    iota[i] = (uint32_t)i;
 }
 
 // MODE: PRNG_WALK_L64 for the paper's generator (only that walk compiled into
@@ -387,18 +385,15 @@ extern "C" int gg_mc_run(prng_t *h, const gg_mc_config *cfg, int64_t *tallies, i
         S.alive = (uint32_t *)alloc(n * 4);
         S.launched = (uint32_t *)alloc(n * 4);
         S.busy = (uint8_t *)alloc(n);
-        uint32_t *iota = (uint32_t *)alloc(n * 4);
         uint32_t *d_list = (uint32_t *)alloc(n * 4);
         int32_t *d_count = (int32_t *)alloc(8);
-        size_t sel_bytes = 0;
-        MCK(cub::DeviceSelect::Flagged(nullptr, sel_bytes, iota, S.busy, d_list, d_count, (int)n, s));
-        void *sel_tmp = alloc(sel_bytes);
+        void *sel_tmp = alloc(gg::compact_scratch_bytes((int64_t)n));
         unsigned long long *d_tal = (unsigned long long *)alloc(nt * 8);
         unsigned long long *d_cnt = (unsigned long long *)alloc(4 * 8);
         MCK(cudaMemsetAsync(d_tal, 0, nt * 8, s));
         MCK(cudaMemsetAsync(d_cnt, 0, 4 * 8, s));
         if (per_thread) MCK(cudaMemsetAsync(per_thread, 0, n * nt * 8, s));
-        mc_init_state<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(S, n, iota);
+        mc_init_state<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(S, n);
         cudaEvent_t e0, e1;
         MCK(cudaEventCreate(&e0));
         MCK(cudaEventCreate(&e1));
@@ -440,8 +435,8 @@ extern "C" int gg_mc_run(prng_t *h, const gg_mc_config *cfg, int64_t *tallies, i
                 epochs++;
                 window_slots += wslots;
                 // threads that still have work after this epoch
-                MCK(cub::DeviceSelect::Flagged(sel_tmp, sel_bytes, iota, S.busy, d_list, d_count,
-                                               (int)n, s));
+                MCK(gg::compact_flagged(nullptr, S.busy, (int64_t)n, (int32_t *)d_list, nullptr, d_count,
+                                        nullptr, 0, sel_tmp, s));
                 MCK(cudaMemcpyAsync(h_count, d_count, 4, cudaMemcpyDeviceToHost, s));
                 MCK(cudaMemcpyAsync(h_list, d_list, n * 4, cudaMemcpyDeviceToHost, s));
                 MCK(cudaMemcpyAsync(counters, d_cnt, 4 * sizeof(unsigned long long),
