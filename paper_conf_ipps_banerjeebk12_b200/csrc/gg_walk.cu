@@ -378,6 +378,257 @@ __global__ void __launch_bounds__(64, MINB) gg_fill64x2_tma_kernel(const __grid_
     }
 }
 
+// Pair variant of the x2 kernel (m = 2^32, forward maps): lane owns the
+// ADJACENT walkers u*64 + 2*lane and u*64 + 2*lane + 1, so both records of a
+// row come from one LDS.64 (6 per draw instead of 12) and both labels leave
+// in one 16-byte store (V4: the output index of walker u*64 + 2*lane is even
+// for every draw, i.e. W and g_origin even and out 16-byte aligned; else two
+// 8-byte stores).  Draws where every walker of the unit is active (the whole
+// fill for full units) take a copy of the draw body without per-walker range
+// checks or state commits.
+template <bool V4>
+__global__ void __launch_bounds__(64, 1) gg_fill64p_tma_kernel(const __grid_constant__ CUtensorMap tmap,
+                                                               FillArgs a, uint32_t units64) {
+    constexpr int kTile = 6 * 64;
+    __shared__ __align__(128) uint32_t tiles[kFillWarps][2][kTile];
+    __shared__ __align__(8) uint64_t bars[kFillWarps][2];
+    const uint32_t lane = threadIdx.x & 31u, wib = threadIdx.x >> 5;
+    const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+    uint32_t *buf0 = tiles[wib][0], *buf1 = tiles[wib][1];
+    uint64_t *bar0 = &bars[wib][0], *bar1 = &bars[wib][1];
+    if (lane == 0) {
+        mbar_init(bar0, 1);
+        mbar_init(bar1, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncwarp();
+    uint32_t ph0 = 0, ph1 = 0;
+    const uint32_t kBytes = kTile * 4;
+    for (uint32_t u = warp; u < units64; u += nwarps) {
+        const uint32_t ta = u * 64u + 2u * lane, tb = ta + 1u;
+        uint32_t ja0 = 0xFFFFFFFFu, ja1 = 0, jb0 = 0xFFFFFFFFu, jb1 = 0;
+        if (ta < a.W) {
+            walker_draw_range(a.N, a.nl, a.W, ta, ja0, ja1);
+            ja0 = max(ja0, a.ja);
+            ja1 = min(ja1, a.jb);
+        }
+        if (tb < a.W) {
+            walker_draw_range(a.N, a.nl, a.W, tb, jb0, jb1);
+            jb0 = max(jb0, a.ja);
+            jb1 = min(jb1, a.jb);
+        }
+        const uint32_t jlo = __reduce_min_sync(0xFFFFFFFFu, min(ja0, jb0));
+        const uint32_t jhi = __reduce_max_sync(0xFFFFFFFFu, max(ja1, jb1));
+        if (jlo >= jhi) continue;
+        // draws in which all 64 walkers of the unit are active (empty if one is idle)
+        const uint32_t jin0 = __reduce_max_sync(0xFFFFFFFFu, max(ja0, jb0));
+        const uint32_t jin1 = __reduce_min_sync(0xFFFFFFFFu, min(ja1, jb1));
+        uint32_t xa = 0, ya = 0, xb = 0, yb = 0;
+        if (tb < a.W) {
+            const uint2 px = *reinterpret_cast<const uint2 *>(a.x + ta);
+            const uint2 py = *reinterpret_cast<const uint2 *>(a.y + ta);
+            xa = px.x, xb = px.y, ya = py.x, yb = py.y;
+        } else if (ta < a.W) {
+            xa = a.x[ta];
+            ya = a.y[ta];
+        }
+        if (lane == 0) {
+            mbar_expect_tx(bar0, kBytes);
+            tma_load_tile(buf0, &tmap, bar0, (int32_t)(u * 64u), (int32_t)((jlo - a.Jw) * 6u));
+            if (jlo + 1 < jhi) {
+                mbar_expect_tx(bar1, kBytes);
+                tma_load_tile(buf1, &tmap, bar1, (int32_t)(u * 64u), (int32_t)((jlo + 1 - a.Jw) * 6u));
+            }
+        }
+        auto refill = [&](uint32_t *buf, uint64_t *bar, uint32_t j) {
+            __syncwarp();
+            if (lane == 0 && j + 2 < jhi) {
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                mbar_expect_tx(bar, kBytes);
+                tma_load_tile(buf, &tmap, bar, (int32_t)(u * 64u), (int32_t)((j + 2 - a.Jw) * 6u));
+            }
+        };
+        auto load = [&](const uint32_t *buf, uint32_t (&wa)[6], uint32_t (&wb)[6]) {
+#pragma unroll
+            for (int r = 0; r < 6; r++) {
+                const uint2 v = *reinterpret_cast<const uint2 *>(buf + r * 64 + 2 * lane);
+                wa[r] = v.x;
+                wb[r] = v.y;
+            }
+        };
+        // all 64 walkers active: walk in place, one store
+        auto draw_in = [&](uint32_t *buf, uint64_t *bar, uint32_t ph, uint32_t j) {
+            mbar_wait(bar, ph);
+            uint32_t wa[6], wb[6];
+            load(buf, wa, wb);
+            gg_walk64x2_r2p(wa, wb, xa, ya, xb, yb);
+            const uint64_t idx = (uint64_t)j * a.W + ta - a.g_origin;
+            if (V4) {
+                *reinterpret_cast<uint4 *>(reinterpret_cast<uint2 *>(a.out) + idx) =
+                    make_uint4(xa, ya, xb, yb);
+            } else {
+                reinterpret_cast<uint2 *>(a.out)[idx] = make_uint2(xa, ya);
+                reinterpret_cast<uint2 *>(a.out)[idx + 1] = make_uint2(xb, yb);
+            }
+            refill(buf, bar, j);
+        };
+        // edge draws: per-walker range checks
+        auto draw_edge = [&](uint32_t *buf, uint64_t *bar, uint32_t ph, uint32_t j) {
+            mbar_wait(bar, ph);
+            uint32_t wa[6], wb[6];
+            load(buf, wa, wb);
+            uint32_t nxa = xa, nya = ya, nxb = xb, nyb = yb;
+            gg_walk64x2_r2p(wa, wb, nxa, nya, nxb, nyb);
+            if (j >= ja0 && j < ja1) {
+                xa = nxa;
+                ya = nya;
+                emit_label<0>(a, (uint64_t)j * a.W + ta - a.g_origin, xa, ya);
+            }
+            if (j >= jb0 && j < jb1) {
+                xb = nxb;
+                yb = nyb;
+                emit_label<0>(a, (uint64_t)j * a.W + tb - a.g_origin, xb, yb);
+            }
+            refill(buf, bar, j);
+        };
+        for (uint32_t j = jlo; j < jhi; j += 2) {
+            if (j >= jin0 && j + 2 <= jin1) {  // warp-uniform
+                draw_in(buf0, bar0, ph0, j);
+                ph0 ^= 1u;
+                draw_in(buf1, bar1, ph1, j + 1);
+                ph1 ^= 1u;
+            } else {
+                draw_edge(buf0, bar0, ph0, j);
+                ph0 ^= 1u;
+                if (j + 1 < jhi) {
+                    draw_edge(buf1, bar1, ph1, j + 1);
+                    ph1 ^= 1u;
+                }
+            }
+        }
+        if (tb < a.W) {
+            *reinterpret_cast<uint2 *>(a.x + ta) = make_uint2(xa, xb);
+            *reinterpret_cast<uint2 *>(a.y + ta) = make_uint2(ya, yb);
+        } else if (ta < a.W) {
+            a.x[ta] = xa;
+            a.y[ta] = ya;
+        }
+    }
+}
+
+// Pair variant with per-lane cp.async staging instead of TMA: each lane
+// copies its own 8-byte slice of the 6 record rows (its two adjacent
+// walkers) into a lane-private column of a 3-stage shared-memory ring
+// (layout [stage][row][lane], conflict-free), so there is no cross-lane
+// hazard: no mbarrier, no __syncwarp, no elected issuer.  Per draw: 6
+// LDGSTS.64 + commit + wait + 6 LDS.64 (the TMA path spends ~23 issue slots
+// per draw on the elected copy alone).
+constexpr int kPcStages = 3;
+
+__device__ __forceinline__ void cp_async8(void *smem, const void *gmem, uint32_t src_bytes) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;" ::"r"(smem_u32(smem)), "l"(gmem),
+                 "r"(src_bytes)
+                 : "memory");
+}
+
+template <bool V4>
+__global__ void __launch_bounds__(64, 1) gg_fill64pc_kernel(FillArgs a, uint32_t units64) {
+    __shared__ __align__(16) uint2 ring[kFillWarps][kPcStages][6][32];
+    const uint32_t lane = threadIdx.x & 31u, wib = threadIdx.x >> 5;
+    const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+    const uint64_t rstride = a.pitch;  // words between rows
+    for (uint32_t u = warp; u < units64; u += nwarps) {
+        const uint32_t ta = u * 64u + 2u * lane, tb = ta + 1u;
+        uint32_t ja0 = 0xFFFFFFFFu, ja1 = 0, jb0 = 0xFFFFFFFFu, jb1 = 0;
+        if (ta < a.W) {
+            walker_draw_range(a.N, a.nl, a.W, ta, ja0, ja1);
+            ja0 = max(ja0, a.ja);
+            ja1 = min(ja1, a.jb);
+        }
+        if (tb < a.W) {
+            walker_draw_range(a.N, a.nl, a.W, tb, jb0, jb1);
+            jb0 = max(jb0, a.ja);
+            jb1 = min(jb1, a.jb);
+        }
+        const uint32_t jlo = __reduce_min_sync(0xFFFFFFFFu, min(ja0, jb0));
+        const uint32_t jhi = __reduce_max_sync(0xFFFFFFFFu, max(ja1, jb1));
+        if (jlo >= jhi) continue;
+        const uint32_t jin0 = __reduce_max_sync(0xFFFFFFFFu, max(ja0, jb0));
+        const uint32_t jin1 = __reduce_min_sync(0xFFFFFFFFu, min(ja1, jb1));
+        uint32_t xa = 0, ya = 0, xb = 0, yb = 0;
+        if (tb < a.W) {
+            const uint2 px = *reinterpret_cast<const uint2 *>(a.x + ta);
+            const uint2 py = *reinterpret_cast<const uint2 *>(a.y + ta);
+            xa = px.x, xb = px.y, ya = py.x, yb = py.y;
+        } else if (ta < a.W) {
+            xa = a.x[ta];
+            ya = a.y[ta];
+        }
+        // bytes of this lane's 8-byte slice that exist (the window's pitch is
+        // a multiple of 32 walkers, so the slice never straddles its end)
+        const uint32_t src_bytes = ta < a.W ? 8u : 0u;
+        const uint32_t *col = a.bits + ta;
+        auto issue = [&](uint32_t j, int stage) {
+            if (j < jhi) {
+                const uint32_t *rec = col + (uint64_t)(j - a.Jw) * 6u * rstride;
+#pragma unroll
+                for (int r = 0; r < 6; r++)
+                    cp_async8(&ring[wib][stage][r][lane], rec + r * rstride, src_bytes);
+            }
+            asm volatile("cp.async.commit_group;" ::: "memory");
+        };
+        issue(jlo, 0);
+        issue(jlo + 1, 1);
+        uint32_t stage = 0;
+        for (uint32_t j = jlo; j < jhi; j++) {
+            issue(j + 2, stage == 0 ? 2 : stage - 1);  // the stage read two draws ago
+            asm volatile("cp.async.wait_group 2;" ::: "memory");
+            uint32_t wa[6], wb[6];
+#pragma unroll
+            for (int r = 0; r < 6; r++) {
+                const uint2 v = ring[wib][stage][r][lane];
+                wa[r] = v.x;
+                wb[r] = v.y;
+            }
+            stage = stage == 2 ? 0 : stage + 1;
+            if (j >= jin0 && j < jin1) {  // warp-uniform: all 64 walkers active
+                gg_walk64x2_r2p(wa, wb, xa, ya, xb, yb);
+                const uint64_t idx = (uint64_t)j * a.W + ta - a.g_origin;
+                if (V4) {
+                    *reinterpret_cast<uint4 *>(reinterpret_cast<uint2 *>(a.out) + idx) =
+                        make_uint4(xa, ya, xb, yb);
+                } else {
+                    reinterpret_cast<uint2 *>(a.out)[idx] = make_uint2(xa, ya);
+                    reinterpret_cast<uint2 *>(a.out)[idx + 1] = make_uint2(xb, yb);
+                }
+            } else {
+                uint32_t nxa = xa, nya = ya, nxb = xb, nyb = yb;
+                gg_walk64x2_r2p(wa, wb, nxa, nya, nxb, nyb);
+                if (j >= ja0 && j < ja1) {
+                    xa = nxa;
+                    ya = nya;
+                    emit_label<0>(a, (uint64_t)j * a.W + ta - a.g_origin, xa, ya);
+                }
+                if (j >= jb0 && j < jb1) {
+                    xb = nxb;
+                    yb = nyb;
+                    emit_label<0>(a, (uint64_t)j * a.W + tb - a.g_origin, xb, yb);
+                }
+            }
+        }
+        asm volatile("cp.async.wait_group 0;" ::: "memory");
+        if (tb < a.W) {
+            *reinterpret_cast<uint2 *>(a.x + ta) = make_uint2(xa, xb);
+            *reinterpret_cast<uint2 *>(a.y + ta) = make_uint2(ya, yb);
+        } else if (ta < a.W) {
+            a.x[ta] = xa;
+            a.y[ta] = ya;
+        }
+    }
+}
+
 // l = 1 ("emit every vertex"): one 32-bit record word per
 // number (R = 1: 3 bits used), so a number costs 4 B read + 8 B written and
 // ~10 instructions: the bound is HBM, not the integer pipes.  Each warp owns
@@ -743,6 +994,33 @@ cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count) {
                 static const int minb = getenv("GG_FILL_MINB") ? atoi(getenv("GG_FILL_MINB")) : 1;
                 static const bool r2p = !(getenv("GG_FILL_STEP") && atoi(getenv("GG_FILL_STEP")) == 0);
                 static const bool u2 = !(getenv("GG_FILL_U2") && atoi(getenv("GG_FILL_U2")) == 0);
+                static const bool pair = getenv("GG_FILL_PAIR") && atoi(getenv("GG_FILL_PAIR")) == 1;
+                static const bool pair_cp = getenv("GG_FILL_PAIR") && atoi(getenv("GG_FILL_PAIR")) == 2;
+                if (pair_cp && r2p && minb == 1 && u2) {
+                    const bool v4 = (a.W % 2 == 0) && (a.g_origin % 2 == 0) &&
+                                    ((uintptr_t)a.out % 16 == 0);
+                    if (v4) {
+                        plan_grid(gg_fill64pc_kernel<true>, units64, sm_count, blocks, threads);
+                        gg_fill64pc_kernel<true><<<blocks, threads, 0, s>>>(a, units64);
+                    } else {
+                        plan_grid(gg_fill64pc_kernel<false>, units64, sm_count, blocks, threads);
+                        gg_fill64pc_kernel<false><<<blocks, threads, 0, s>>>(a, units64);
+                    }
+                    return cudaGetLastError();
+                }
+                if (pair && r2p && minb == 1 && u2) {
+                    // adjacent-walker lanes (LDS.64, 16-B stores when the output index parity allows)
+                    const bool v4 = (a.W % 2 == 0) && (a.g_origin % 2 == 0) &&
+                                    ((uintptr_t)a.out % 16 == 0);
+                    if (v4) {
+                        plan_grid(gg_fill64p_tma_kernel<true>, units64, sm_count, blocks, threads);
+                        gg_fill64p_tma_kernel<true><<<blocks, threads, 0, s>>>(map, a, units64);
+                    } else {
+                        plan_grid(gg_fill64p_tma_kernel<false>, units64, sm_count, blocks, threads);
+                        gg_fill64p_tma_kernel<false><<<blocks, threads, 0, s>>>(map, a, units64);
+                    }
+                    return cudaGetLastError();
+                }
 #define GG_LAUNCH_X2(...)                                                                   \
     do {                                                                                    \
         plan_grid(gg_fill64x2_tma_kernel<__VA_ARGS__>, units64, sm_count, blocks, threads); \

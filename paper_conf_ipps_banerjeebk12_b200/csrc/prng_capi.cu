@@ -15,10 +15,12 @@
 #include <functional>
 #include <mutex>
 #include <new>
+#include <string>
 #include <thread>
 #include <vector>
 
 #include <cuda_runtime.h>
+#include <nvtx3/nvToolsExt.h>
 
 #include "gg_internal.h"
 #include "prng.h"
@@ -147,7 +149,71 @@ struct CudaFail {
 
 }  // namespace
 
+// Fig.4 timeline (diagnostic, GG_TIMELINE=<path>): every FEED chunk (host
+// interval of the feed threads), H2D copy, walk kernel and D2H copy of the
+// handle as [kind, start_us, end_us] on one clock, written to <path> as JSON
+// by prng_destroy.  Device intervals are event pairs on the stream the work
+// ran on, placed on the host clock through a base event synchronised at
+// creation (alignment error ~10 us).  Host work also carries NVTX ranges
+// ("gg.feed", "gg.stage", "gg.fill") for an attached Nsight Systems.
+struct Timeline {
+    std::string path;
+    std::chrono::steady_clock::time_point t0;
+    cudaEvent_t base = nullptr;
+    struct Host { const char *kind; double a, b; };
+    struct Dev { const char *kind; cudaEvent_t a, b; };
+    std::vector<Host> host;
+    std::vector<Dev> dev;
+    std::mutex mu;
+    double now_us() const {
+        return std::chrono::duration<double, std::micro>(std::chrono::steady_clock::now() - t0)
+            .count();
+    }
+    void host_span(const char *kind, double a, double b) {
+        std::lock_guard<std::mutex> lk(mu);
+        host.push_back({kind, a, b});
+    }
+    // event pair around work enqueued on s between begin() and end()
+    cudaEvent_t begin(cudaStream_t s) {
+        cudaEvent_t e = nullptr;
+        cudaEventCreate(&e);
+        cudaEventRecord(e, s);
+        return e;
+    }
+    void end(const char *kind, cudaEvent_t a, cudaStream_t s) {
+        cudaEvent_t e = nullptr;
+        cudaEventCreate(&e);
+        cudaEventRecord(e, s);
+        std::lock_guard<std::mutex> lk(mu);
+        dev.push_back({kind, a, e});
+    }
+    void dump() {
+        cudaDeviceSynchronize();
+        FILE *f = fopen(path.c_str(), "w");
+        if (!f) return;
+        fprintf(f, "[");
+        bool first = true;
+        for (auto &r : host) {
+            fprintf(f, "%s[\"%s\", %.3f, %.3f]", first ? "" : ",\n", r.kind, r.a, r.b);
+            first = false;
+        }
+        for (auto &r : dev) {
+            float a = 0, b = 0;
+            cudaEventElapsedTime(&a, base, r.a);
+            cudaEventElapsedTime(&b, base, r.b);
+            fprintf(f, "%s[\"%s\", %.3f, %.3f]", first ? "" : ",\n", r.kind, a * 1e3, b * 1e3);
+            first = false;
+            cudaEventDestroy(r.a);
+            cudaEventDestroy(r.b);
+        }
+        fprintf(f, "]\n");
+        fclose(f);
+        cudaEventDestroy(base);
+    }
+};
+
 struct prng_s {
+    Timeline *tl = nullptr;
     prng_graph_params g{};
     prng_options o{};
     uint64_t W = 0, seed = 0;
@@ -253,6 +319,8 @@ void feed_chunk(prng_s *h, uint64_t wa, uint64_t wb, uint64_t k0, uint32_t nrows
     const bool nt_st = streaming_stores;
     const unsigned nt = h->pool->size();
     auto t0 = std::chrono::steady_clock::now();
+    const double tl0 = h->tl ? h->tl->now_us() : 0.0;
+    nvtxRangePushA("gg.feed");
     h->pool->run([&](unsigned ti) {
         // contiguous, 16-walker aligned slices
         uint64_t per = round_up((cw + nt - 1) / nt, 16);
@@ -287,9 +355,18 @@ void feed_chunk(prng_s *h, uint64_t wa, uint64_t wb, uint64_t k0, uint32_t nrows
         else
             gg::feed_splitmix_rows(h->seed, tg0, hi - lo, k0, nrows, buf + lo, bpitch, nt_st);
     });
+    nvtxRangePop();
+    if (h->tl) h->tl->host_span("feed", tl0, h->tl->now_us());
     auto t1 = std::chrono::steady_clock::now();
     h->stats.feed_seconds += std::chrono::duration<double>(t1 - t0).count();
     h->stats.bits_bytes_fed += (uint64_t)nrows * cw * 4;
+}
+
+// H2D copy of a fed chunk on the copy stream (timeline: one "h2d" span).
+void h2d_copy(prng_s *h, void *dst, const void *src, size_t bytes) {
+    cudaEvent_t a = h->tl ? h->tl->begin(h->copy_stream) : nullptr;
+    CK(cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, h->copy_stream));
+    if (a) h->tl->end("h2d", a, h->copy_stream);
 }
 
 // FEED + TRANSFER: stream words [k0, k0+nrows) of local walkers [0, Wv) into
@@ -349,8 +426,7 @@ void stage_rows(prng_s *h, uint64_t k0, uint64_t nrows, uint64_t Wv, uint32_t *d
             h->chunk_next = (b + 1) % h->kChunks;
             CK(cudaEventSynchronize(h->chunk_done[b]));  // pinned chunk free again
             feed_chunk(h, 0, Wv, k0 + r, (uint32_t)nr, h->chunk[b], ids, dpitch, bursty);
-            CK(cudaMemcpyAsync(dst + r * dpitch, h->chunk[b], nr * dpitch * 4,
-                               cudaMemcpyHostToDevice, h->copy_stream));
+            h2d_copy(h, dst + r * dpitch, h->chunk[b], nr * dpitch * 4);
             CK(cudaEventRecord(h->chunk_done[b], h->copy_stream));
             h->stats.h2d_bytes += nr * dpitch * 4;
             r += nr;
@@ -373,8 +449,7 @@ void stage_rows(prng_s *h, uint64_t k0, uint64_t nrows, uint64_t Wv, uint32_t *d
             const uint64_t cp = round_up(cw, 8);
             feed_chunk(h, wa, wb, k0 + r, (uint32_t)nr, h->chunk[b], ids, cp, bursty);
             for (uint64_t i = 0; i < nr; i++)  // one contiguous DMA per row segment
-                CK(cudaMemcpyAsync(dst + (r + i) * dpitch + wa, h->chunk[b] + i * cp, cw * 4,
-                                   cudaMemcpyHostToDevice, h->copy_stream));
+                h2d_copy(h, dst + (r + i) * dpitch + wa, h->chunk[b] + i * cp, cw * 4);
             CK(cudaEventRecord(h->chunk_done[b], h->copy_stream));
             h->stats.h2d_bytes += (uint64_t)nr * cw * 4;
         }
@@ -603,6 +678,14 @@ int prng_create(prng_t **out, const prng_graph_params *g, uint64_t walkers, uint
             }
         }
         h->pool = new ThreadPool(nt, cpus);
+        if (const char *tp = getenv("GG_TIMELINE")) {
+            h->tl = new Timeline();
+            h->tl->path = tp;
+            CK(cudaEventCreate(&h->tl->base));
+            CK(cudaEventRecord(h->tl->base, nullptr));
+            CK(cudaEventSynchronize(h->tl->base));
+            h->tl->t0 = std::chrono::steady_clock::now();
+        }
         CK(cudaStreamCreateWithFlags(&h->copy_stream, cudaStreamNonBlocking));
         CK(cudaStreamCreateWithFlags(&h->d2h_stream, cudaStreamNonBlocking));
         CK(cudaStreamCreateWithFlags(&h->work_stream, cudaStreamNonBlocking));
@@ -694,7 +777,9 @@ int prng_fill(prng_t *h, void *dev_ptr, uint64_t n, int fmt, void *stream) {
                        uint64_t rows, uint64_t Jw, cudaStream_t st) {
                        gg::FillArgs a = fill_args(h, bits, pitch, rows, Jw, ja, jb, N, nl, N,
                                                   dev_ptr, out_u32);
+                       cudaEvent_t ta = h->tl ? h->tl->begin(st) : nullptr;
                        CK(gg::launch_fill(a, st, h->sm_count));
+                       if (ta) h->tl->end("walk", ta, st);
                        h->stats.kernel_launches++;
                    });
         h->N = N + nl;
@@ -743,13 +828,17 @@ int prng_fill_host(prng_t *h, void *host_ptr, uint64_t n, int fmt) {
                            CK(cudaStreamWaitEvent(st, h->hout_free[oslot], 0));
                            gg::FillArgs a = fill_args(h, bits, pitch, rows, Jw, a0, a1, N, nl,
                                                       gA, h->hout[oslot], out_u32);
+                           cudaEvent_t ta = h->tl ? h->tl->begin(st) : nullptr;
                            CK(gg::launch_fill(a, st, h->sm_count));
+                           if (ta) h->tl->end("walk", ta, st);
                            h->stats.kernel_launches++;
                            CK(cudaEventRecord(h->ev_tmp, st));
                            CK(cudaStreamWaitEvent(h->d2h_stream, h->ev_tmp, 0));
+                           cudaEvent_t tc = h->tl ? h->tl->begin(h->d2h_stream) : nullptr;
                            CK(cudaMemcpyAsync(dst + (gA - N) * esz, h->hout[oslot],
                                               (gB - gA) * esz, cudaMemcpyDeviceToHost,
                                               h->d2h_stream));
+                           if (tc) h->tl->end("d2h", tc, h->d2h_stream);
                            CK(cudaEventRecord(h->hout_free[oslot], h->d2h_stream));
                            h->stats.d2h_bytes += (gB - gA) * esz;
                            oslot ^= 1;
@@ -1078,6 +1167,12 @@ int prng_get_stats(prng_t *h, prng_stats *s) {
 
 int prng_destroy(prng_t *h) {
     if (!h) return PRNG_OK;
+    if (h->tl) {
+        cudaSetDevice(h->o.device);
+        h->tl->dump();
+        delete h->tl;
+        h->tl = nullptr;
+    }
     free_all(h);
     delete h;
     return PRNG_OK;
