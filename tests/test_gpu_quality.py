@@ -137,3 +137,25 @@ def test_c1_chi_square_on_gpu_output():
     p2 = chi2_p(torch.bincount(cell.reshape(-1), minlength=65536), cell.numel() / 65536)
     assert p1 > ALPHA and p2 > ALPHA, (p1, p2)
     g.close()
+
+
+def test_crush_scale_battery_small():
+    """The 15 streaming statistics of tests/battery_gpu.py (the ones
+    tools/battery_big.py runs at 2^33 words, profiles/r02_battery.json) at
+    2^26 words: l = 64 passes all 15 in bulk and walker-major order, the
+    l = 1 walk fails several (§IV-B Table III)."""
+    import os
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    sys.path.insert(0, os.path.join(root, "tools"))
+    import battery_big as BB
+    import battery_gpu as G
+
+    def tests():
+        return G.crush_scale_tests(rank300_matrices=1 << 11, samples_n=1 << 22)
+    for r in (BB.run_stream(BB.gen_chunks(1 << 25, 1 << 20), tests()),
+              BB.run_stream(BB.gen_chunks(1 << 25, 4096, walker_major=True), tests())):
+        assert r["failed"] == [], r
+        assert r["passed"] == "15/15"
+    bad = BB.run_stream(BB.gen_chunks(1 << 24, 1 << 20, walk_len=1), tests())
+    assert len(bad["failed"]) >= 3, bad
