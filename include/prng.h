@@ -142,6 +142,10 @@ int prng_create(prng_t **out, const prng_graph_params *g, uint64_t walkers,
  * other draws are fed by host threads into pinned ring slots and copied on
  * a side stream, overlapped with the walk (E-mode, Fig.4 FEED/TRANSFER/
  * GENERATE).  Not allowed while an on-demand epoch is open (PRNG_E_STATE).
+ * Draw indices are 32-bit: a call that would need draw 2^32 - 256 or later of
+ * any walker (ceil((N + labels) / W) > 2^32 - 256) returns
+ * PRNG_E_UNSUPPORTED before anything is enqueued (same for prng_prefetch,
+ * prng_epoch_begin and a prng_load of such a position).
  */
 int prng_fill(prng_t *h, void *dev_ptr, uint64_t n, int fmt, void *stream);
 
@@ -175,7 +179,8 @@ int prng_rewind(prng_t *h, void *stream);
  * Host checkpoint: prng_state_size gives the bytes of a serialised state;
  * prng_save / prng_load copy walker state + N (+ epoch cursor) to/from a
  * caller buffer of that size.  prng_load requires a handle created with the
- * same params, walkers and seed.
+ * same params, walkers, seed, walker_base and bit_source (the checkpoint
+ * header records them; a mismatch returns PRNG_E_INVALID and changes nothing).
  */
 int prng_state_size(prng_t *h, size_t *bytes);
 int prng_save(prng_t *h, void *host_buf, size_t bytes);

@@ -484,12 +484,15 @@ int check_fmt(const prng_s *h, uint64_t n, int fmt) {
 }
 
 // Draw indices are 32-bit in the walk kernels (FillArgs::Jw/ja/jb, the
-// per-walker cursor j[]): a bulk call whose last draw ceil((N + nl) / W) - 1
-// would not fit is refused up front (PRNG_E_UNSUPPORTED, nothing enqueued).
+// per-walker cursor j[]), and the kernels' loops step them by up to 2 draws
+// and look up to 16 draws ahead: a bulk call whose end ceil((N + nl) / W)
+// exceeds kDrawLimit = 2^32 - 256 is refused up front (PRNG_E_UNSUPPORTED,
+// nothing enqueued), so no loop index can wrap.
+constexpr uint64_t kDrawLimit = 0xFFFFFF00ull;
 bool draws_fit(const prng_s *h, uint64_t N, uint64_t nl) {
     const uint64_t W = h->W;
     if (nl > UINT64_MAX - N - W) return false;
-    return (N + nl + W - 1) / W <= 0xFFFFFFFFull;
+    return (N + nl + W - 1) / W <= kDrawLimit;
 }
 
 gg::FillArgs fill_args(prng_s *h, const uint32_t *bits, uint64_t pitch, uint64_t rows,
@@ -857,7 +860,7 @@ int prng_prefetch(prng_t *h, uint64_t draws) {
     if (!h) return PRNG_E_INVALID;
     if (draws == 0) return PRNG_E_INVALID;
     if (h->od_open) return PRNG_E_STATE;
-    if (h->N / h->W + draws > 0xFFFFFFFFull) return PRNG_E_UNSUPPORTED;
+    if (h->N / h->W + draws > kDrawLimit) return PRNG_E_UNSUPPORTED;
     return guard(h, [&] {
         const uint64_t pitch = h->pitch();
         const size_t bytes = (size_t)draws * h->R * pitch * 4;
@@ -956,7 +959,7 @@ int prng_load(prng_t *h, const void *host_buf, size_t bytes) {
         hd.bit_source != h->o.bit_source)
         return PRNG_E_INVALID;
     // a resumed position must itself be reachable by the 32-bit draw cursor
-    if (hd.N > (0xFFFFFFFFull * h->W) || hd.od_J0 > 0xFFFFFFFFull) return PRNG_E_INVALID;
+    if (hd.N > kDrawLimit * h->W || hd.od_J0 > kDrawLimit) return PRNG_E_INVALID;
     if (h->od_open) return PRNG_E_STATE;
     return guard(h, [&] {
         CK(cudaDeviceSynchronize());
@@ -976,7 +979,7 @@ static int epoch_begin_impl(prng_t *h, uint64_t active_walkers, const uint32_t *
     return guard(h, [&] {
         cudaStream_t s = (cudaStream_t)stream;
         const uint64_t J0 = h->od_started ? h->od_J0 : (h->N + h->W - 1) / h->W;
-        if (J0 + draws > 0xFFFFFFFFull) return PRNG_E_UNSUPPORTED;
+        if (J0 + draws > kDrawLimit) return PRNG_E_UNSUPPORTED;
         const int slot = h->od_slot ^ 1;
         // walkers [0, pf_hi) of this window were staged ahead (gg_epoch_prefeed)
         const bool pf = h->pf_valid && !ids && draws == 1 && h->pf_J0 == J0 &&

@@ -417,18 +417,19 @@ def test_non_power_of_two_fast_kernel_parity(torch_cuda, m):
 
 # ------------------------------------------- 32-bit draw cursor, checkpoints
 def test_draw_index_limit_refused_without_side_effects(torch_cuda):
-    """Draw indices are 32-bit in the kernels: a fill or prefetch reaching
-    draw 2^32 - 1 is refused with PRNG_E_UNSUPPORTED before anything is
-    enqueued.  Up to the limit the numbers are still
-    the oracle's: a walk of draw J's record (stream words 2 + R0 + 6J ..,
-    R9) from the saved walker state (checkpoint resume at N = J*W)."""
+    """Draw indices are 32-bit in the kernels: a fill or prefetch whose end
+    passes 2^32 - 256 draws (the kernels' loop margin) is refused with
+    PRNG_E_UNSUPPORTED before anything is enqueued.  Up
+    to the limit the numbers are still the oracle's: a walk of draw J's
+    record (stream words 2 + R0 + 6J .., R9) from the saved walker state
+    (checkpoint resume at N = J*W)."""
     import struct
     torch = torch_cuda
     from paper_conf_ipps_banerjeebk12_b200 import PrngError
     W, seed = 64, 5
     g = G(walkers=W, seed=seed)
     blob = bytearray(g.save())
-    J = (1 << 32) - 4
+    J = (1 << 32) - 256 - 3
     struct.pack_into("<Q", blob, 16, J * W)          # SavedHeader.N
     g.load(bytes(blob))
     assert g.tell() == J * W
@@ -440,7 +441,7 @@ def test_draw_index_limit_refused_without_side_effects(torch_cuda):
         assert e.value.status == -2  # PRNG_E_UNSUPPORTED
     torch.cuda.synchronize()
     assert g.tell() == J * W and bool((big == 7).all())
-    # draws J .. J+2 (the last index 2^32 - 2 still fits): OK, oracle-exact
+    # draws J .. J+2 (end = 2^32 - 256, the limit): OK, oracle-exact
     g.fill(big, n=3 * W)
     assert g.tell() == (J + 3) * W
     z = as_u64(big[:3 * W]).reshape(3, W)
@@ -455,7 +456,7 @@ def test_draw_index_limit_refused_without_side_effects(torch_cuda):
             x, y = O.walk(M32, x, y, rec, 64)
             assert int(z[d, t]) == O.label(M32, x, y), (t, d)
     with pytest.raises(PrngError) as e:
-        g.fill(big, n=1)                               # would need draw 2^32 - 1
+        g.fill(big, n=1)                               # one draw past the limit
     assert e.value.status == -2
     assert g.tell() == (J + 3) * W
     g.close()
