@@ -133,3 +133,24 @@ def test_on_demand_single_walker_single_draw():
     g.epoch_end()
     assert int(u64(o)[0]) == int(O.walker_draws(M32, 64, 64, 12, 0, 0, 1)[0])
     assert g.check() == 0
+
+
+def test_binding_rejects_unsafe_outputs():
+    """The Python binding checks what the C ABI cannot: the output tensor is
+    contiguous, holds n numbers and lives on the handle's device (host memory
+    for fill_host); nothing is generated on a refusal."""
+    import torch
+    g = G(walkers=64, seed=1)
+    d = torch.empty(256, dtype=torch.int64, device="cuda")
+    for bad in (lambda: g.fill(d[::2]),                         # strided view
+                lambda: g.fill(d, n=257),                       # n > numel
+                lambda: g.fill(torch.empty(8, dtype=torch.int64)),  # host tensor
+                lambda: g.fill_host(d),                         # device tensor
+                lambda: g.fill_host(torch.empty(8, dtype=torch.int64), n=9),
+                lambda: g.fill_host(np.empty((4, 4), dtype=np.uint64)[:, ::2])):
+        with pytest.raises(ValueError):
+            bad()
+    assert g.tell() == 0
+    g.fill(d, n=100)
+    assert g.tell() == 100
+    g.close()
