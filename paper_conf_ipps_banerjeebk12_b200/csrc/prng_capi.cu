@@ -221,8 +221,6 @@ struct prng_s {
     int sm_count = 148;
     bool poisoned = false;
     cudaStream_t copy_stream = nullptr;  // H2D of seed bits
-    cudaStream_t copy_stream2 = nullptr; // second H2D stream (GG_FEED_STREAMS=2): chunks alternate
-    int chunk_seq = 0;                   // chunks staged so far (picks the copy stream)
     cudaStream_t d2h_stream = nullptr;   // D2H of results (prng_fill_host)
     cudaStream_t work_stream = nullptr;  // kernels of prng_fill_host
     ThreadPool *pool = nullptr;
@@ -306,7 +304,7 @@ void free_all(prng_s *h) {
         if (h->od_free[i]) cudaEventDestroy(h->od_free[i]);
     }
     if (h->ev_tmp) cudaEventDestroy(h->ev_tmp);
-    for (auto s : {h->copy_stream, h->copy_stream2, h->d2h_stream, h->work_stream})
+    for (auto s : {h->copy_stream, h->d2h_stream, h->work_stream})
         if (s) cudaStreamDestroy(s);
     delete h->pool;
     h->pool = nullptr;
@@ -364,24 +362,11 @@ void feed_chunk(prng_s *h, uint64_t wa, uint64_t wb, uint64_t k0, uint32_t nrows
     h->stats.bits_bytes_fed += (uint64_t)nrows * cw * 4;
 }
 
-// H2D copy of a fed chunk on copy stream cs (timeline: one "h2d" span).
-void h2d_copy(prng_s *h, void *dst, const void *src, size_t bytes, cudaStream_t cs) {
-    cudaEvent_t a = h->tl ? h->tl->begin(cs) : nullptr;
-    CK(cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, cs));
-    if (a) h->tl->end("h2d", a, cs);
-}
-
-// Copy stream of the next chunk: chunks alternate between the two copy
-// streams when the second exists (two DMA queues in flight).
-cudaStream_t next_copy_stream(prng_s *h) {
-    const int k = h->chunk_seq++;
-    return (h->copy_stream2 && (k & 1)) ? h->copy_stream2 : h->copy_stream;
-}
-
-// Every copy stream waits for ev (a window slot is free again).
-void copies_wait(prng_s *h, cudaEvent_t ev) {
-    CK(cudaStreamWaitEvent(h->copy_stream, ev, 0));
-    if (h->copy_stream2) CK(cudaStreamWaitEvent(h->copy_stream2, ev, 0));
+// H2D copy of a fed chunk on the copy stream (timeline: one "h2d" span).
+void h2d_copy(prng_s *h, void *dst, const void *src, size_t bytes) {
+    cudaEvent_t a = h->tl ? h->tl->begin(h->copy_stream) : nullptr;
+    CK(cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, h->copy_stream));
+    if (a) h->tl->end("h2d", a, h->copy_stream);
 }
 
 // FEED + TRANSFER: stream words [k0, k0+nrows) of local walkers [0, Wv) into
@@ -441,9 +426,8 @@ void stage_rows(prng_s *h, uint64_t k0, uint64_t nrows, uint64_t Wv, uint32_t *d
             h->chunk_next = (b + 1) % h->kChunks;
             CK(cudaEventSynchronize(h->chunk_done[b]));  // pinned chunk free again
             feed_chunk(h, 0, Wv, k0 + r, (uint32_t)nr, h->chunk[b], ids, dpitch, bursty);
-            cudaStream_t cs = next_copy_stream(h);
-            h2d_copy(h, dst + r * dpitch, h->chunk[b], nr * dpitch * 4, cs);
-            CK(cudaEventRecord(h->chunk_done[b], cs));
+            h2d_copy(h, dst + r * dpitch, h->chunk[b], nr * dpitch * 4);
+            CK(cudaEventRecord(h->chunk_done[b], h->copy_stream));
             h->stats.h2d_bytes += nr * dpitch * 4;
             r += nr;
         }
@@ -464,10 +448,9 @@ void stage_rows(prng_s *h, uint64_t k0, uint64_t nrows, uint64_t Wv, uint32_t *d
             // stores there halved the DMA rate of whole rounds (LR trace)
             const uint64_t cp = round_up(cw, 8);
             feed_chunk(h, wa, wb, k0 + r, (uint32_t)nr, h->chunk[b], ids, cp, bursty);
-            cudaStream_t cs = next_copy_stream(h);
             for (uint64_t i = 0; i < nr; i++)  // one contiguous DMA per row segment
-                h2d_copy(h, dst + (r + i) * dpitch + wa, h->chunk[b] + i * cp, cw * 4, cs);
-            CK(cudaEventRecord(h->chunk_done[b], cs));
+                h2d_copy(h, dst + (r + i) * dpitch + wa, h->chunk[b] + i * cp, cw * 4);
+            CK(cudaEventRecord(h->chunk_done[b], h->copy_stream));
             h->stats.h2d_bytes += (uint64_t)nr * cw * 4;
         }
         r += nr;
@@ -478,10 +461,6 @@ void stage_rows(prng_s *h, uint64_t k0, uint64_t nrows, uint64_t Wv, uint32_t *d
 void join_copies(prng_s *h, cudaStream_t s) {
     CK(cudaEventRecord(h->ev_tmp, h->copy_stream));
     CK(cudaStreamWaitEvent(s, h->ev_tmp, 0));
-    if (h->copy_stream2) {
-        CK(cudaEventRecord(h->ev_tmp, h->copy_stream2));
-        CK(cudaStreamWaitEvent(s, h->ev_tmp, 0));
-    }
 }
 
 void ensure_dev(uint32_t *&p, size_t &cap, size_t bytes) {
@@ -575,7 +554,7 @@ void run_pieces(prng_s *h, uint64_t N, uint64_t nl, cudaStream_t s, Emit emit) {
             for (auto &p : h->ring) CK(cudaMalloc(&p, rbytes));
             h->ring_cap = rbytes;
         }
-        copies_wait(h, h->ring_free[slot]);  // slot no longer read
+        CK(cudaStreamWaitEvent(h->copy_stream, h->ring_free[slot], 0));  // slot no longer read
         stage_rows(h, 2 + h->R0 + h->R * j, (jb - j) * h->R, W, h->ring[slot], pitch);
         join_copies(h, s);
         emit(j, jb, h->ring[slot], pitch, (jb - j) * h->R, j, s);
@@ -711,8 +690,6 @@ int prng_create(prng_t **out, const prng_graph_params *g, uint64_t walkers, uint
             h->tl->t0 = std::chrono::steady_clock::now();
         }
         CK(cudaStreamCreateWithFlags(&h->copy_stream, cudaStreamNonBlocking));
-        static const int nstreams = getenv("GG_FEED_STREAMS") ? atoi(getenv("GG_FEED_STREAMS")) : 1;
-        if (nstreams >= 2) CK(cudaStreamCreateWithFlags(&h->copy_stream2, cudaStreamNonBlocking));
         CK(cudaStreamCreateWithFlags(&h->d2h_stream, cudaStreamNonBlocking));
         CK(cudaStreamCreateWithFlags(&h->work_stream, cudaStreamNonBlocking));
         CK(cudaEventCreateWithFlags(&h->ev_tmp, cudaEventDisableTiming));
@@ -721,11 +698,7 @@ int prng_create(prng_t **out, const prng_graph_params *g, uint64_t walkers, uint
         h->chunk_bytes = (size_t)(chunk_mb > 0 ? chunk_mb : 32) << 20;
         h->kChunks = std::min(prng_s::kMaxChunks, std::max(2, nchunks));
         for (int i = 0; i < h->kChunks; i++) {
-            // A/B hook GG_FEED_WC=1: write-combined pinned chunks (the feed only
-            // writes them; the DMA then reads without snooping the CPU caches)
-            static const bool wc = getenv("GG_FEED_WC") && atoi(getenv("GG_FEED_WC")) == 1;
-            CK(cudaHostAlloc((void **)&h->chunk[i], h->chunk_bytes,
-                             cudaHostAllocPortable | (wc ? cudaHostAllocWriteCombined : 0)));
+            CK(cudaHostAlloc((void **)&h->chunk[i], h->chunk_bytes, cudaHostAllocPortable));
             CK(cudaEventCreateWithFlags(&h->chunk_done[i], cudaEventDisableTiming));
         }
         for (int i = 0; i < 2; i++) {
@@ -896,7 +869,6 @@ int prng_prefetch(prng_t *h, uint64_t draws) {
         const uint64_t J = h->N / h->W;
         stage_rows(h, 2 + h->R0 + h->R * J, draws * h->R, h->W, h->res_bits, pitch);
         CK(cudaStreamSynchronize(h->copy_stream));
-        if (h->copy_stream2) CK(cudaStreamSynchronize(h->copy_stream2));
         h->res_J = J;
         h->res_D = draws;
         return PRNG_OK;
@@ -1033,7 +1005,7 @@ static int epoch_begin_impl(prng_t *h, uint64_t active_walkers, const uint32_t *
             }
         } else {
             // kernels of the epoch that last used this slot must be done with it
-            copies_wait(h, h->od_free[slot]);
+            CK(cudaStreamWaitEvent(h->copy_stream, h->od_free[slot], 0));
         }
         h->od_slot = slot;
         h->od_bits = h->od_buf[slot];
@@ -1089,7 +1061,7 @@ int epoch_prefeed(prng_t *h, uint64_t hi, uint64_t pitch) {
         const uint64_t J0 = h->od_J0;
         const size_t bytes = (size_t)h->R * pitch * 4;
         if (bytes > h->od_cap[slot]) return PRNG_OK;  // not reserved: skip the prefeed
-        copies_wait(h, h->od_free[slot]);
+        CK(cudaStreamWaitEvent(h->copy_stream, h->od_free[slot], 0));
         stage_rows(h, 2 + h->R0 + h->R * J0, h->R, hi, h->od_buf[slot], pitch, nullptr, true);
         h->pf_valid = true;
         h->pf_slot = slot;
