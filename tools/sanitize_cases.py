@@ -2,7 +2,9 @@
 
     compute-sanitizer --tool memcheck|racecheck|synccheck python tools/sanitize_cases.py
 Covers: init, bulk fill (x2 TMA u64/u32, x1 TMA, LDG, generic m, bipartite,
-l = 1 TMA), on-demand consume, list ranking (Phase I-III), Monte Carlo epoch.
+l = 1 TMA; the GG_FILL_PAIR variants when run under that hook), on-demand
+consume in every walk mode, list ranking (Phase I-III, the compaction
+kernel over several tiles), Monte Carlo epoch.
 Sizes are tiny (the sanitizer slows kernels by orders of magnitude) but
 ragged: partial units, partial warps, several draws per TMA stage.
 """
@@ -32,16 +34,19 @@ for kw in ({}, {"m": 256}, {"m": 1000}, {"walk_len": 1}, {"walk_len": 17, "m": 1
     g.close()
 print("fill ok")
 
-g = Generator(walkers=W, seed=12)
-g.epoch_begin(W, 4)
-o = torch.empty(W * 4, dtype=torch.int64, device=dev)
-g.consume(W, uniform=4, out=o)
-g.epoch_end()
-torch.cuda.synchronize()
-g.close()
+# on demand, one generator per walk mode (prng_walk_mode: l = 64 pow2, its
+# bipartite form, any l pow2, l = 64 with m <= 2^30, generic)
+for kw in ({}, {"variant": 1}, {"walk_len": 17}, {"m": 1000}, {"m": (1 << 32) - 5}):
+    g = Generator(walkers=W, seed=12, **kw)
+    g.epoch_begin(W, 5)
+    o = torch.empty(W * 5, dtype=torch.int64, device=dev)
+    g.consume(W, uniform=5, out=o)
+    g.epoch_end()
+    torch.cuda.synchronize()
+    g.close()
 print("consume ok")
 
-n = 3000
+n = 10000  # several compaction tiles (2048 items each) per round
 succ, pred, head = inputs.random_list(n, 5)
 g = Generator(walkers=n, seed=13)
 r, info = g.list_rank(torch.from_numpy(succ).to(dev), torch.from_numpy(pred).to(dev), head)
