@@ -26,11 +26,6 @@ struct InitArgs {
 };
 cudaError_t launch_init(const InitArgs &a, cudaStream_t s);
 
-// H2D of `bytes` from pinned host memory by an SM copy kernel (A/B hook
-// GG_FEED_PULL=1 of the FEED's TRANSFER; src must be 16-byte aligned).
-cudaError_t launch_h2d_pull(void *dst, const void *src, size_t bytes, cudaStream_t s,
-                            int sm_count);
-
 // Bulk Alg.2 over draws [ja, jb) of every walker, restricted to bulk
 // positions g in [N, N + nl) (R11: g = j*W + t).  The bits of draw j are rows
 // (j - Jw)*R .. (j - Jw)*R + R-1 of the window `bits` (pitch words per row).

@@ -10,7 +10,6 @@
 // warp at a time; the grid is sized so every resident warp owns the same
 // number of units (static balance, ~1-2% tail) instead of relying on a
 // partially filled last wave.
-#include <algorithm>
 #include <cstdint>
 #include <cstdlib>
 #include <cstring>
@@ -50,43 +49,6 @@ __global__ void __launch_bounds__(128) gg_init_kernel(InitArgs a) {
     a.x[t] = x;
     a.y[t] = y;
     a.j[t] = 0;
-}
-
-// TRANSFER by the SMs instead of a copy engine (A/B hook GG_FEED_PULL=1):
-// threads read the pinned chunk through the PCIe mapping 16 bytes at a time,
-// with four loads in flight per thread, and write device memory.  Many
-// thousand outstanding reads instead of one DMA queue.
-__global__ void __launch_bounds__(256) gg_h2d_pull_kernel(uint4 *__restrict__ dst,
-                                                          const uint4 *__restrict__ src,
-                                                          uint64_t n16) {
-    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-    uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    for (; i + 3 * stride < n16; i += 4 * stride) {
-        uint4 v[4];
-#pragma unroll
-        for (int k = 0; k < 4; k++) v[k] = __ldcs(src + i + k * stride);
-#pragma unroll
-        for (int k = 0; k < 4; k++) dst[i + k * stride] = v[k];
-    }
-    for (; i < n16; i += stride) dst[i] = __ldcs(src + i);
-}
-
-cudaError_t launch_h2d_pull(void *dst, const void *src, size_t bytes, cudaStream_t s,
-                            int sm_count) {
-    if (bytes == 0) return cudaSuccess;
-    // 16-byte body, byte tail
-    const uint64_t n16 = bytes / 16;
-    if (n16) {
-        const uint32_t blocks = (uint32_t)std::min<uint64_t>((uint64_t)sm_count * 4,
-                                                             (n16 + 255) / 256);
-        gg_h2d_pull_kernel<<<blocks, 256, 0, s>>>((uint4 *)dst, (const uint4 *)src, n16);
-    }
-    if (bytes % 16) {
-        cudaError_t e = cudaMemcpyAsync((char *)dst + n16 * 16, (const char *)src + n16 * 16,
-                                        bytes % 16, cudaMemcpyHostToDevice, s);
-        if (e != cudaSuccess) return e;
-    }
-    return cudaGetLastError();
 }
 
 cudaError_t launch_init(const InitArgs &a, cudaStream_t s) {

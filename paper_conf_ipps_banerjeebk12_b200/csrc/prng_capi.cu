@@ -365,11 +365,7 @@ void feed_chunk(prng_s *h, uint64_t wa, uint64_t wb, uint64_t k0, uint32_t nrows
 // H2D copy of a fed chunk on the copy stream (timeline: one "h2d" span).
 void h2d_copy(prng_s *h, void *dst, const void *src, size_t bytes) {
     cudaEvent_t a = h->tl ? h->tl->begin(h->copy_stream) : nullptr;
-    static const bool pull = getenv("GG_FEED_PULL") && atoi(getenv("GG_FEED_PULL")) == 1;
-    if (pull && ((uintptr_t)src % 16) == 0 && ((uintptr_t)dst % 16) == 0)
-        CK(gg::launch_h2d_pull(dst, src, bytes, h->copy_stream, h->sm_count));
-    else
-        CK(cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, h->copy_stream));
+    CK(cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, h->copy_stream));
     if (a) h->tl->end("h2d", a, h->copy_stream);
 }
 

@@ -45,7 +45,7 @@ VARIANTS = ["GG_FILL_NO_TMA=1", "GG_FILL_X1=1", "GG_FILL_MINB=24", "GG_FILL_STEP
             "GG_FILL_MINB=24 GG_FILL_U2=0",
             "GG_FILL_ONEWAVE=1", "GG_FILL_KPW=2", "GG_FEED_NT_ALL=1", "GG_FEED_NO_NT=1",
             "GG_FEED_CHUNK_MB=1", "GG_FEED_CHUNKS=2", "GG_MC_MINB=4", "GG_FILL_PAIR=1",
-            "GG_FILL_PAIR=2", "GG_FILL_PAIR=3", "GG_FILL_PAIR=4", "GG_FEED_PULL=1"]
+            "GG_FILL_PAIR=2", "GG_FILL_PAIR=3", "GG_FILL_PAIR=4"]
 
 
 @pytest.fixture(scope="module")
