@@ -23,6 +23,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <map>
+#include <memory>
 #include <mutex>
 #include <vector>
 
@@ -326,6 +327,9 @@ extern "C" int gg_list_rank(prng_t *h, int64_t n, const int32_t *succ, const int
         return p;
     };
     int rc = PRNG_OK;
+    // held until the stream is known idle: a compaction kernel still in
+    // flight after a failure must not write into a slot another call owns
+    std::unique_ptr<CountSlot> slot_owner;
     try {
         cudaEvent_t ev[4];
         for (auto &e : ev) LCK(cudaEventCreate(&e));
@@ -346,7 +350,8 @@ extern "C" int gg_list_rank(prng_t *h, int64_t n, const int32_t *succ, const int
         int32_t tail = -1;
         LCK(cudaMemcpyAsync(&tail, d_num + 1, 4, cudaMemcpyDeviceToHost, s));
         void *tmp = alloc(gg::compact_scratch_bytes(n));
-        CountSlot slot;
+        slot_owner.reset(new CountSlot());
+        CountSlot &slot = *slot_owner;
         LCK(cudaStreamSynchronize(s));
         if (tail < 0) throw Fail{PRNG_E_INVALID};
 
@@ -508,6 +513,8 @@ extern "C" int gg_list_rank(prng_t *h, int64_t n, const int32_t *succ, const int
         rc = f.rc;
     }
     for (void *p : bufs) cudaFreeAsync(p, s);
-    if (rc == PRNG_OK && cudaStreamSynchronize(s) != cudaSuccess) rc = PRNG_E_CUDA;
+    const bool idle = cudaStreamSynchronize(s) == cudaSuccess;
+    if (rc == PRNG_OK && !idle) rc = PRNG_E_CUDA;
+    if (!idle) slot_owner.release();  // never reuse a slot a kernel may still write
     return rc;
 }
