@@ -36,7 +36,7 @@ __global__ void user_kernel(const __grid_constant__ prng_view v, uint32_t walker
     prng_state st = prng_state_load(&v, t);
     const uint32_t calls = t % 3u + 1u;  // data-dependent demand
     for (uint32_t i = 0; i < calls; i++) out[(size_t)t * 3 + i] = prng_next(&st);  // north_star's prng_next(&state)
-    prng_state_store(&v, &st);
+    prng_state_store(&st);
 }
 
 int main(int argc, char **argv) {

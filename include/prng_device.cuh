@@ -563,6 +563,17 @@ __device__ __forceinline__ uint32_t prng_available(const prng_view *v, const prn
     return (st->used < v->D) ? (v->D - st->used) : 0u;
 }
 
+/* One-argument forms: the state carries its view. */
+__device__ __forceinline__ uint32_t prng_available(const prng_state *st)
+{
+    return prng_available(st->view, st);
+}
+
+__device__ __forceinline__ void prng_state_store(const prng_state *st)
+{
+    prng_state_store(st->view, st);
+}
+
 /* Walk implementations prng_next can use, picked from the view's (m, l,
  * variant, l0).  A kernel that knows its generator's shape instantiates
  * prng_next<MODE> so only that walk is compiled into it; prng_next without a
