@@ -800,6 +800,226 @@ __global__ void __launch_bounds__(64, 1) gg_fill64ps_tma_kernel(const __grid_con
     }
 }
 
+// ---------------------------------------------------------------------------
+// Composed-step ("table") walk, l = 64, m = 2^k, forward maps.  The 64 steps
+// of a draw are 16 groups of 4 steps; a group reads 12 consecutive record
+// bits (fields f0..f3, R3) and the composition of its 4 Gabber-Galil steps
+// (§III-A, k = f mod 7, R4) is ONE affine map over Z/2^32:
+//     x' = a x + b y + e,   y' = c x + d y + f.
+// Every step is affine (sigma_1..3: y += 2x + c; sigma_4..6: x += 2y + c), so
+// the composition is exact in wrapped 32-bit arithmetic; over all 4096 bit
+// patterns the coefficients are a, d <= 29, b, c <= 22, e, f <= 40 (checked by
+// enumeration in tests/test_table_formulation.py), so one 32-bit word holds
+// them (5-5-5-5-6-6 bits) and the 4096-entry table is 16 KB of shared memory,
+// built by each block at start.  Per group and walker: the 12 bits as a
+// scaled table offset (2 ALU), one LDS, the six coefficients (balanced
+// between left shifts on the FMA pipe and right shifts on the ALU pipe), four
+// IMAD -- ~17 SASS per 4 steps instead of ~25 for four R2P steps.
+// ---------------------------------------------------------------------------
+constexpr int kTabEntries = 4096;
+
+__device__ __forceinline__ uint32_t gg_compose4(uint32_t p) {
+    uint32_t a = 1, b = 0, e = 0, c = 0, d = 1, f = 0;
+#pragma unroll
+    for (int i = 0; i < 4; i++) {
+        const uint32_t k = ((p >> (3 * i)) & 7u) % 7u;
+        if (k >= 1 && k <= 3) {  // y <- y + 2x + (k - 1)
+            c += 2 * a;
+            d += 2 * b;
+            f += 2 * e + (k - 1);
+        } else if (k >= 4) {     // x <- x + 2y + (k - 4)
+            a += 2 * c;
+            b += 2 * d;
+            e += 2 * f + (k - 4);
+        }
+    }
+    return a | b << 5 | c << 10 | d << 15 | e << 20 | f << 26;
+}
+
+__device__ __forceinline__ void gg_build_table(uint32_t *tab) {
+    for (uint32_t p = threadIdx.x; p < kTabEntries; p += blockDim.x) tab[p] = gg_compose4(p);
+    __syncthreads();
+}
+
+// shared-memory byte offset of group G's entry: its 12 record bits times 4
+template <int G>
+__device__ __forceinline__ uint32_t gg_group_off(const uint32_t (&w)[6]) {
+    constexpr int bit = 12 * G, wi = bit >> 5, sh = bit & 31;
+    if (sh == 0) return (w[wi] << 2) & 0x3FFCu;
+    if (sh <= 20) return (w[wi] >> (sh - 2)) & 0x3FFCu;
+    return __funnelshift_r(w[wi], w[wi + 1], sh - 2) & 0x3FFCu;
+}
+
+// Left shifts by multiplications with opaque powers of two (IMAD on the
+// FMA-heavy pipe), right shifts and masks on the ALU pipe: ptxas would
+// otherwise fuse each (t << s) >> r into SHF + LOP3 and put the whole unpack
+// on the ALU pipe.
+struct TabShifts {
+    uint32_t k22, k17, k12, k6;
+};
+__device__ __forceinline__ TabShifts gg_tab_shifts() {
+    TabShifts k{1u << 22, 1u << 17, 1u << 12, 1u << 6};
+    asm volatile("" : "+r"(k.k22), "+r"(k.k17), "+r"(k.k12), "+r"(k.k6));
+    return k;
+}
+
+__device__ __forceinline__ void gg_group_apply(const uint32_t *tab, uint32_t off, uint32_t &x,
+                                               uint32_t &y, const TabShifts &k) {
+    const uint32_t t = *reinterpret_cast<const uint32_t *>(reinterpret_cast<const char *>(tab) + off);
+    const uint32_t a = t & 31u, b = (t * k.k22) >> 27, c = (t * k.k17) >> 27, d = (t * k.k12) >> 27;
+    const uint32_t e = (t * k.k6) >> 26, f = t >> 26;
+    const uint32_t nx = b * y + (a * x + e);
+    const uint32_t ny = d * y + (c * x + f);
+    x = nx;
+    y = ny;
+}
+
+__device__ __forceinline__ void gg_walk64x2_table(const uint32_t *tab, const uint32_t (&wa)[6],
+                                                  const uint32_t (&wb)[6], uint32_t &xa,
+                                                  uint32_t &ya, uint32_t &xb, uint32_t &yb,
+                                                  const TabShifts &k) {
+#define GG_TG(G)                                           \
+    gg_group_apply(tab, gg_group_off<G>(wa), xa, ya, k);   \
+    gg_group_apply(tab, gg_group_off<G>(wb), xb, yb, k);
+    GG_TG(0) GG_TG(1) GG_TG(2) GG_TG(3) GG_TG(4) GG_TG(5) GG_TG(6) GG_TG(7)
+    GG_TG(8) GG_TG(9) GG_TG(10) GG_TG(11) GG_TG(12) GG_TG(13) GG_TG(14) GG_TG(15)
+#undef GG_TG
+}
+
+// The pair kernel (adjacent walkers per lane, per-warp TMA, two stages) with
+// the composed-step walk; NW warps per block share one table.  EMIT: 0 = u64
+// label for m = 2^32 ((y << 32) | x), 1 = u64 label for m = 2^k < 2^32,
+// 2 = low u32 word (m <= 2^16); V4: 16-byte stores of two m = 2^32 labels.
+template <int NW, int EMIT, bool V4>
+__global__ void __launch_bounds__(NW * 32) gg_fill64t_tma_kernel(const __grid_constant__ CUtensorMap tmap,
+                                                                 FillArgs a, uint32_t units64) {
+    constexpr int kTile = 6 * 64;
+    __shared__ __align__(128) uint32_t tiles[NW][2][kTile];
+    __shared__ __align__(8) uint64_t bars[NW][2];
+    __shared__ __align__(16) uint32_t tab[kTabEntries];
+    const uint32_t lane = threadIdx.x & 31u, wib = threadIdx.x >> 5;
+    const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+    uint32_t *buf0 = tiles[wib][0], *buf1 = tiles[wib][1];
+    uint64_t *bar0 = &bars[wib][0], *bar1 = &bars[wib][1];
+    if (lane == 0) {
+        mbar_init(bar0, 1);
+        mbar_init(bar1, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    gg_build_table(tab);  // includes __syncthreads
+    const TabShifts ksh = gg_tab_shifts();
+    uint32_t ph0 = 0, ph1 = 0;
+    const uint32_t kBytes = kTile * 4;
+    for (uint32_t u = warp; u < units64; u += nwarps) {
+        const uint32_t ta = u * 64u + 2u * lane, tb = ta + 1u;
+        uint32_t ja0 = 0xFFFFFFFFu, ja1 = 0, jb0 = 0xFFFFFFFFu, jb1 = 0;
+        if (ta < a.W) {
+            walker_draw_range(a.N, a.nl, a.W, ta, ja0, ja1);
+            ja0 = max(ja0, a.ja);
+            ja1 = min(ja1, a.jb);
+        }
+        if (tb < a.W) {
+            walker_draw_range(a.N, a.nl, a.W, tb, jb0, jb1);
+            jb0 = max(jb0, a.ja);
+            jb1 = min(jb1, a.jb);
+        }
+        const uint32_t jlo = __reduce_min_sync(0xFFFFFFFFu, min(ja0, jb0));
+        const uint32_t jhi = __reduce_max_sync(0xFFFFFFFFu, max(ja1, jb1));
+        if (jlo >= jhi) continue;
+        const uint32_t jin0 = __reduce_max_sync(0xFFFFFFFFu, max(ja0, jb0));
+        const uint32_t jin1 = __reduce_min_sync(0xFFFFFFFFu, min(ja1, jb1));
+        uint32_t xa = 0, ya = 0, xb = 0, yb = 0;
+        if (tb < a.W) {
+            const uint2 px = *reinterpret_cast<const uint2 *>(a.x + ta);
+            const uint2 py = *reinterpret_cast<const uint2 *>(a.y + ta);
+            xa = px.x, xb = px.y, ya = py.x, yb = py.y;
+        } else if (ta < a.W) {
+            xa = a.x[ta];
+            ya = a.y[ta];
+        }
+        if (lane == 0) {
+            mbar_expect_tx(bar0, kBytes);
+            tma_load_tile(buf0, &tmap, bar0, (int32_t)(u * 64u), (int32_t)((jlo - a.Jw) * 6u));
+            if (jlo + 1 < jhi) {
+                mbar_expect_tx(bar1, kBytes);
+                tma_load_tile(buf1, &tmap, bar1, (int32_t)(u * 64u), (int32_t)((jlo + 1 - a.Jw) * 6u));
+            }
+        }
+        auto refill = [&](uint32_t *buf, uint64_t *bar, uint32_t j) {
+            __syncwarp();
+            if (lane == 0 && j + 2 < jhi) {
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                mbar_expect_tx(bar, kBytes);
+                tma_load_tile(buf, &tmap, bar, (int32_t)(u * 64u), (int32_t)((j + 2 - a.Jw) * 6u));
+            }
+        };
+        auto load = [&](const uint32_t *buf, uint32_t (&wa)[6], uint32_t (&wb)[6]) {
+#pragma unroll
+            for (int r = 0; r < 6; r++) {
+                const uint2 v = *reinterpret_cast<const uint2 *>(buf + r * 64 + 2 * lane);
+                wa[r] = v.x;
+                wb[r] = v.y;
+            }
+        };
+        auto draw_in = [&](uint32_t *buf, uint64_t *bar, uint32_t ph, uint32_t j) {
+            mbar_wait(bar, ph);
+            uint32_t wa[6], wb[6];
+            load(buf, wa, wb);
+            gg_walk64x2_table(tab, wa, wb, xa, ya, xb, yb, ksh);
+            const uint64_t idx = (uint64_t)j * a.W + ta - a.g_origin;
+            if (EMIT == 0 && V4) {
+                *reinterpret_cast<uint4 *>(reinterpret_cast<uint2 *>(a.out) + idx) =
+                    make_uint4(xa, ya, xb, yb);
+            } else {
+                emit_label<EMIT>(a, idx, xa, ya);
+                emit_label<EMIT>(a, idx + 1, xb, yb);
+            }
+            refill(buf, bar, j);
+        };
+        auto draw_edge = [&](uint32_t *buf, uint64_t *bar, uint32_t ph, uint32_t j) {
+            mbar_wait(bar, ph);
+            uint32_t wa[6], wb[6];
+            load(buf, wa, wb);
+            uint32_t nxa = xa, nya = ya, nxb = xb, nyb = yb;
+            gg_walk64x2_table(tab, wa, wb, nxa, nya, nxb, nyb, ksh);
+            if (j >= ja0 && j < ja1) {
+                xa = nxa;
+                ya = nya;
+                emit_label<EMIT>(a, (uint64_t)j * a.W + ta - a.g_origin, xa, ya);
+            }
+            if (j >= jb0 && j < jb1) {
+                xb = nxb;
+                yb = nyb;
+                emit_label<EMIT>(a, (uint64_t)j * a.W + tb - a.g_origin, xb, yb);
+            }
+            refill(buf, bar, j);
+        };
+        for (uint32_t j = jlo; j < jhi; j += 2) {
+            if (j >= jin0 && j + 2 <= jin1) {  // warp-uniform
+                draw_in(buf0, bar0, ph0, j);
+                ph0 ^= 1u;
+                draw_in(buf1, bar1, ph1, j + 1);
+                ph1 ^= 1u;
+            } else {
+                draw_edge(buf0, bar0, ph0, j);
+                ph0 ^= 1u;
+                if (j + 1 < jhi) {
+                    draw_edge(buf1, bar1, ph1, j + 1);
+                    ph1 ^= 1u;
+                }
+            }
+        }
+        if (tb < a.W) {
+            *reinterpret_cast<uint2 *>(a.x + ta) = make_uint2(xa, xb);
+            *reinterpret_cast<uint2 *>(a.y + ta) = make_uint2(ya, yb);
+        } else if (ta < a.W) {
+            a.x[ta] = xa;
+            a.y[ta] = ya;
+        }
+    }
+}
+
 // Pair variant with per-lane cp.async staging instead of TMA: each lane
 // copies its own 8-byte slice of the 6 record rows (its two adjacent
 // walkers) into a lane-private column of a 3-stage shared-memory ring
@@ -1256,6 +1476,30 @@ cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count) {
                 plan_grid(gg_fill64x2_tma_kernel<3, 1, 1, 1, false, true>, units64, sm_count, blocks, threads);
                 gg_fill64x2_tma_kernel<3, 1, 1, 1, false, true><<<blocks, threads, 0, s>>>(map, a, units64);
             }
+            return cudaGetLastError();
+        }
+    }
+    static const int table_nw = getenv("GG_FILL_TABLE") ? atoi(getenv("GG_FILL_TABLE")) : 0;
+    if (a.l == 64 && a.pow2 && a.variant == 0 && table_nw > 0 && a.rows) {
+        // composed-step table walk; GG_FILL_TABLE = warps per block (2, 4 or 8)
+        CUtensorMap map;
+        const uint32_t units64 = (a.W + 63u) / 64u;
+        if (make_window_map(&map, a.bits, a.pitch, a.rows, 64)) {
+            const bool v4 = (a.W % 2 == 0) && (a.g_origin % 2 == 0) && ((uintptr_t)a.out % 16 == 0);
+#define GG_LAUNCH_T(NW, E, V)                                                                    \
+    gg_fill64t_tma_kernel<NW, E, V><<<(units64 + NW - 1) / NW, NW * 32, 0, s>>>(map, a, units64)
+#define GG_LAUNCH_TNW(NW)                                                                        \
+    do {                                                                                         \
+        if (a.out_u32) GG_LAUNCH_T(NW, 2, false);                                                \
+        else if (a.log2m != 32) GG_LAUNCH_T(NW, 1, false);                                       \
+        else if (v4) GG_LAUNCH_T(NW, 0, true);                                                   \
+        else GG_LAUNCH_T(NW, 0, false);                                                          \
+    } while (0)
+            if (table_nw >= 8) GG_LAUNCH_TNW(8);
+            else if (table_nw >= 4) GG_LAUNCH_TNW(4);
+            else GG_LAUNCH_TNW(2);
+#undef GG_LAUNCH_TNW
+#undef GG_LAUNCH_T
             return cudaGetLastError();
         }
     }
