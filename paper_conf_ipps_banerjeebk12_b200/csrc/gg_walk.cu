@@ -10,6 +10,7 @@
 // warp at a time; the grid is sized so every resident warp owns the same
 // number of units (static balance, ~1-2% tail) instead of relying on a
 // partially filled last wave.
+#include <algorithm>
 #include <cstdint>
 #include <cstdlib>
 #include <cstring>
@@ -891,7 +892,7 @@ __device__ __forceinline__ void gg_walk64x2_table(const uint32_t *tab, const uin
 // label for m = 2^32 ((y << 32) | x), 1 = u64 label for m = 2^k < 2^32,
 // 2 = low u32 word (m <= 2^16); V4: 16-byte stores of two m = 2^32 labels.
 template <int NW, int EMIT, bool V4>
-__global__ void __launch_bounds__(NW * 32) gg_fill64t_tma_kernel(const __grid_constant__ CUtensorMap tmap,
+__global__ void __launch_bounds__(NW * 32, NW == 8 ? 5 : 1) gg_fill64t_tma_kernel(const __grid_constant__ CUtensorMap tmap,
                                                                  FillArgs a, uint32_t units64) {
     constexpr int kTile = 6 * 64;
     __shared__ __align__(128) uint32_t tiles[NW][2][kTile];
@@ -1479,15 +1480,19 @@ cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count) {
             return cudaGetLastError();
         }
     }
-    static const int table_nw = getenv("GG_FILL_TABLE") ? atoi(getenv("GG_FILL_TABLE")) : 0;
+    // composed-step table walk (the default for l = 64, m = 2^k, forward maps);
+    // GG_FILL_TABLE = warps per block (2, 4, 8; default 8), 0 = the R2P kernels
+    static const int table_nw = getenv("GG_FILL_TABLE") ? atoi(getenv("GG_FILL_TABLE")) : 8;
     if (a.l == 64 && a.pow2 && a.variant == 0 && table_nw > 0 && a.rows) {
-        // composed-step table walk; GG_FILL_TABLE = warps per block (2, 4 or 8)
         CUtensorMap map;
         const uint32_t units64 = (a.W + 63u) / 64u;
         if (make_window_map(&map, a.bits, a.pitch, a.rows, 64)) {
             const bool v4 = (a.W % 2 == 0) && (a.g_origin % 2 == 0) && ((uintptr_t)a.out % 16 == 0);
+            // one 64-walker unit per warp; A/B hook GG_FILL_KPW = units per warp
+            static const int kpw_t = getenv("GG_FILL_KPW") ? std::max(1, atoi(getenv("GG_FILL_KPW"))) : 1;
 #define GG_LAUNCH_T(NW, E, V)                                                                    \
-    gg_fill64t_tma_kernel<NW, E, V><<<(units64 + NW - 1) / NW, NW * 32, 0, s>>>(map, a, units64)
+    gg_fill64t_tma_kernel<NW, E, V><<<(units64 + NW * kpw_t - 1) / (NW * kpw_t), NW * 32, 0, s>>>( \
+        map, a, units64)
 #define GG_LAUNCH_TNW(NW)                                                                        \
     do {                                                                                         \
         if (a.out_u32) GG_LAUNCH_T(NW, 2, false);                                                \
