@@ -892,7 +892,7 @@ __device__ __forceinline__ void gg_walk64x2_table(const uint32_t *tab, const uin
 // label for m = 2^32 ((y << 32) | x), 1 = u64 label for m = 2^k < 2^32,
 // 2 = low u32 word (m <= 2^16); V4: 16-byte stores of two m = 2^32 labels.
 template <int NW, int EMIT, bool V4>
-__global__ void __launch_bounds__(NW * 32, NW == 8 ? 5 : 1) gg_fill64t_tma_kernel(const __grid_constant__ CUtensorMap tmap,
+__global__ void __launch_bounds__(NW * 32) gg_fill64t_tma_kernel(const __grid_constant__ CUtensorMap tmap,
                                                                  FillArgs a, uint32_t units64) {
     constexpr int kTile = 6 * 64;
     __shared__ __align__(128) uint32_t tiles[NW][2][kTile];
@@ -1481,8 +1481,10 @@ cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count) {
         }
     }
     // composed-step table walk (the default for l = 64, m = 2^k, forward maps);
-    // GG_FILL_TABLE = warps per block (2, 4, 8; default 8), 0 = the R2P kernels
-    static const int table_nw = getenv("GG_FILL_TABLE") ? atoi(getenv("GG_FILL_TABLE")) : 8;
+    // GG_FILL_TABLE = warps per block (2, 4, 8; default 4: 63 registers, 7 blocks
+    // = 28 warps per SM, shared memory bound; C2 A/B 4.78 / 5.01 / 5.22 ms for
+    // 4 / 8 / 2, 5.08 ms for 8 warps at 48 registers), 0 = the R2P kernels
+    static const int table_nw = getenv("GG_FILL_TABLE") ? atoi(getenv("GG_FILL_TABLE")) : 4;
     if (a.l == 64 && a.pow2 && a.variant == 0 && table_nw > 0 && a.rows) {
         CUtensorMap map;
         const uint32_t units64 = (a.W + 63u) / 64u;
