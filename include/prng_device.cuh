@@ -47,6 +47,7 @@ struct prng_view {
     uint32_t variant;      /* 0 = forward maps; 1 = bipartite (sigma / sigma^-1 alternating) */
     uint32_t l0;           /* burn-in steps (global step parity for variant 1) */
     uint32_t _pad;
+    const uint32_t *tab;   /* composed-step table in global memory (PRNG_TABLE_WORDS words) */
 };
 
 struct prng_state {
@@ -451,6 +452,77 @@ __device__ __forceinline__ void gg_walk64x2_r2p(const uint32_t a[6], const uint3
     gg_word10x2_r2p<4, BIP>(a[5] >> 20, b[5] >> 20, xa, ya, xb, yb);
 }
 
+/* ------------------------------------------------------------------------
+ * Composed-step ("table") walk for l = 64, m = 2^k, forward maps.  The 64
+ * steps of a draw are 16 groups of 4 steps (12 record bits each, R3); the
+ * composition of a group's 4 steps is one affine map over Z/2^32,
+ *     x' = a x + b y + e,  y' = c x + d y + f,
+ * with a, d <= 29, b, c <= 22, e, f <= 40 for all 4096 bit patterns, packed
+ * a | b<<5 | c<<10 | d<<15 | e<<20 | f<<26 into one 32-bit word.  The
+ * library builds the 4096-word table once per device (prng_view::tab); a
+ * kernel stages it in shared memory (prng_table_stage) and walks with one
+ * lookup and four IMAD per 4 steps (the bulk fill: 311 SASS per number
+ * instead of 454 for the R2P step).  Exact: the same wrapped arithmetic as
+ * the step-by-step walk, checked in tests/test_table_formulation.py.
+ * ------------------------------------------------------------------------ */
+#define PRNG_TABLE_WORDS 4096
+
+/* Shared-memory byte offset of group G's entry: its 12 record bits times 4. */
+template <int G>
+__device__ __forceinline__ uint32_t prng_group_off(const uint32_t (&w)[6]) {
+    constexpr int bit = 12 * G, wi = bit >> 5, sh = bit & 31;
+    if (sh == 0) return (w[wi] << 2) & 0x3FFCu;
+    if (sh <= 20) return (w[wi] >> (sh - 2)) & 0x3FFCu;
+    return __funnelshift_r(w[wi], w[wi + 1], sh - 2) & 0x3FFCu;
+}
+
+// Left shifts by multiplications with opaque powers of two (IMAD on the
+// FMA-heavy pipe), right shifts and masks on the ALU pipe: ptxas would
+// otherwise fuse each (t << s) >> r into SHF + LOP3 and put the whole unpack
+// on the ALU pipe.
+struct prng_tab_shifts {
+    uint32_t k22, k17, k12, k6;
+};
+__device__ __forceinline__ prng_tab_shifts prng_tab_shifts_load() {
+    prng_tab_shifts k{1u << 22, 1u << 17, 1u << 12, 1u << 6};
+    asm volatile("" : "+r"(k.k22), "+r"(k.k17), "+r"(k.k12), "+r"(k.k6));
+    return k;
+}
+
+__device__ __forceinline__ void prng_group_apply(const uint32_t *tab, uint32_t off, uint32_t &x,
+                                               uint32_t &y, const prng_tab_shifts &k) {
+    const uint32_t t = *reinterpret_cast<const uint32_t *>(reinterpret_cast<const char *>(tab) + off);
+    const uint32_t a = t & 31u, b = (t * k.k22) >> 27, c = (t * k.k17) >> 27, d = (t * k.k12) >> 27;
+    const uint32_t e = (t * k.k6) >> 26, f = t >> 26;
+    const uint32_t nx = b * y + (a * x + e);
+    const uint32_t ny = d * y + (c * x + f);
+    x = nx;
+    y = ny;
+}
+
+__device__ __forceinline__ void prng_walk64x2_table(const uint32_t *tab, const uint32_t (&wa)[6],
+                                                  const uint32_t (&wb)[6], uint32_t &xa,
+                                                  uint32_t &ya, uint32_t &xb, uint32_t &yb,
+                                                  const prng_tab_shifts &k) {
+#define PRNG_TG(G)                                           \
+    prng_group_apply(tab, prng_group_off<G>(wa), xa, ya, k);   \
+    prng_group_apply(tab, prng_group_off<G>(wb), xb, yb, k);
+    PRNG_TG(0) PRNG_TG(1) PRNG_TG(2) PRNG_TG(3) PRNG_TG(4) PRNG_TG(5) PRNG_TG(6) PRNG_TG(7)
+    PRNG_TG(8) PRNG_TG(9) PRNG_TG(10) PRNG_TG(11) PRNG_TG(12) PRNG_TG(13) PRNG_TG(14) PRNG_TG(15)
+#undef PRNG_TG
+}
+
+
+__device__ __forceinline__ void prng_walk64_table(const uint32_t *tab, const uint32_t (&w)[6],
+                                                  uint32_t &x, uint32_t &y,
+                                                  const prng_tab_shifts &k)
+{
+#define PRNG_TG1(G) prng_group_apply(tab, prng_group_off<G>(w), x, y, k);
+    PRNG_TG1(0) PRNG_TG1(1) PRNG_TG1(2) PRNG_TG1(3) PRNG_TG1(4) PRNG_TG1(5) PRNG_TG1(6) PRNG_TG1(7)
+    PRNG_TG1(8) PRNG_TG1(9) PRNG_TG1(10) PRNG_TG1(11) PRNG_TG1(12) PRNG_TG1(13) PRNG_TG1(14) PRNG_TG1(15)
+#undef PRNG_TG1
+}
+
 /* One step, any m (generic path), x, y < m.  m = 2^k: wrapped 32-bit
  * arithmetic.  Other m <= 2^30: every pre-reduction value is < 4m < 2^32, so
  * two conditional subtracts reduce it.  Other m < 2^32 ("wide"): the same in
@@ -722,6 +794,86 @@ __device__ __forceinline__ void prng_next_n(prng_state *st, const prng_view *v, 
         for (int q = 0; q + 1 < K; q++)
 #pragma unroll
             for (int r = 0; r < 6; r++) w[q][r] = w[q + 1][r];
+    }
+    st->x = x;
+    st->y = y;
+    st->used += K;
+}
+
+/* ---------------- on demand with the composed-step table ----------------
+ * For views with prng_walk_mode(v) == PRNG_WALK_L64 (the paper's generator):
+ *     __shared__ uint32_t tab[PRNG_TABLE_WORDS];        // 16 KB per block
+ *     prng_table_stage(&view, tab);  __syncthreads();   // every thread of the block
+ *     ... uint64_t r = prng_next_table(&st, &view, tab);
+ * Same numbers as prng_next; other views ignore the table (prng_next). */
+__device__ __forceinline__ void prng_table_stage(const prng_view *v, uint32_t *smem_tab)
+{
+    const uint4 *src = reinterpret_cast<const uint4 *>(v->tab);
+    uint4 *dst = reinterpret_cast<uint4 *>(smem_tab);
+    const uint32_t nthreads = blockDim.x * blockDim.y * blockDim.z;
+    const uint32_t tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
+    for (uint32_t i = tid; i < PRNG_TABLE_WORDS / 4; i += nthreads) dst[i] = __ldg(src + i);
+}
+
+__device__ __forceinline__ uint64_t prng_next_table(prng_state *st, const prng_view *v,
+                                                    const uint32_t *smem_tab)
+{
+    if (prng_walk_mode(v) != PRNG_WALK_L64) return prng_next(st, v);
+    if (st->used >= v->D || st->slot >= v->Wv) {
+        atomicOr(v->flags, PRNG_FLAG_OVERRUN);
+        return 0ull;
+    }
+    const uint32_t *rec = v->bits + (uint64_t)st->used * 6u * v->pitch + st->slot;
+    uint32_t w[6];
+#pragma unroll
+    for (int r = 0; r < 6; r++) w[r] = __ldg(rec + (uint64_t)r * v->pitch);
+    uint32_t x = st->x, y = st->y;
+    prng_walk64_table(smem_tab, w, x, y, prng_tab_shifts_load());
+    st->x = x;
+    st->y = y;
+    st->used++;
+    return gg_label(x, y, v->m, v->log2m, true);
+}
+
+/* K draws with the table, records loaded together (prng_next_n's contract);
+ * ROLL: one walk copy in a rolled loop. */
+template <int K, bool ROLL = false>
+__device__ __forceinline__ void prng_next_n_table(prng_state *st, const prng_view *v,
+                                                  const uint32_t *smem_tab, uint64_t (&out)[K])
+{
+    if (prng_walk_mode(v) != PRNG_WALK_L64 || st->used + K > v->D || st->slot >= v->Wv) {
+#pragma unroll
+        for (int k = 0; k < K; k++) out[k] = prng_next_table(st, v, smem_tab);
+        return;
+    }
+    uint32_t w[K][6];
+#pragma unroll
+    for (int k = 0; k < K; k++) {
+        const uint32_t *rec = v->bits + (uint64_t)(st->used + k) * 6u * v->pitch + st->slot;
+#pragma unroll
+        for (int r = 0; r < 6; r++) w[k][r] = __ldg(rec + (uint64_t)r * v->pitch);
+    }
+    const prng_tab_shifts ks = prng_tab_shifts_load();
+    uint32_t x = st->x, y = st->y;
+    if (!ROLL) {
+#pragma unroll
+        for (int k = 0; k < K; k++) {
+            prng_walk64_table(smem_tab, w[k], x, y, ks);
+            out[k] = gg_label(x, y, v->m, v->log2m, true);
+        }
+    } else {
+#pragma unroll 1
+        for (int k = 0; k < K; k++) {
+            prng_walk64_table(smem_tab, w[0], x, y, ks);
+            const uint64_t lab = gg_label(x, y, v->m, v->log2m, true);
+#pragma unroll
+            for (int q = 0; q < K; q++)
+                if (q == k) out[q] = lab;
+#pragma unroll
+            for (int q = 0; q + 1 < K; q++)
+#pragma unroll
+                for (int r = 0; r < 6; r++) w[q][r] = w[q + 1][r];
+        }
     }
     st->x = x;
     st->y = y;

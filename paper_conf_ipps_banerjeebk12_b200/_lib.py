@@ -83,7 +83,7 @@ class prng_view(ctypes.Structure):
     _fields_ = [("bits", vp), ("wmap", vp), ("x", vp), ("y", vp), ("j", vp), ("flags", vp), ("pitch", u64),
                 ("m", u64), ("J0", u32), ("D", u32), ("Wv", u32), ("R", u32), ("l", u32),
                 ("log2m", u32), ("pow2", u32), ("variant", u32), ("l0", u32),
-                ("_pad", u32)]
+                ("_pad", u32), ("tab", vp)]
 
 
 _SIGS = {

@@ -21,6 +21,13 @@ __global__ void __launch_bounds__(128) consume_kernel(const __grid_constant__ pr
                                                       const uint32_t *counts, uint32_t uniform,
                                                       uint64_t *out, const uint64_t *offsets,
                                                       uint64_t *xor_out) {
+    // the paper's generator (PRNG_WALK_L64): composed-step table in shared memory
+    constexpr bool TAB = MODE == PRNG_WALK_L64;
+    __shared__ __align__(16) uint32_t tab[TAB ? PRNG_TABLE_WORDS : 4];
+    if (TAB) {
+        prng_table_stage(&v, tab);
+        __syncthreads();
+    }
     const uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= threads) return;
     const uint32_t c = counts ? counts[t] : uniform;
@@ -34,7 +41,10 @@ __global__ void __launch_bounds__(128) consume_kernel(const __grid_constant__ pr
     uint32_t r = 0;
     for (; r + 4 <= c; r += 4) {  // four records' loads in flight together
         uint64_t z4[4];
-        prng_next_n<4, false, MODE>(&st, &v, z4);
+        if (TAB)
+            prng_next_n_table<4>(&st, &v, tab, z4);
+        else
+            prng_next_n<4, false, MODE>(&st, &v, z4);
 #pragma unroll
         for (int k = 0; k < 4; k++) {
             acc ^= z4[k];
@@ -42,7 +52,7 @@ __global__ void __launch_bounds__(128) consume_kernel(const __grid_constant__ pr
         }
     }
     for (; r < c; r++) {
-        const uint64_t z = prng_next<MODE>(&st, &v);
+        const uint64_t z = TAB ? prng_next_table(&st, &v, tab) : prng_next<MODE>(&st, &v);
         acc ^= z;
         if (out) out[base + r] = z;
     }

@@ -49,6 +49,10 @@ struct FillArgs {
 };
 cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count);
 
+// The composed-step walk table (PRNG_TABLE_WORDS entries, prng_device.cuh) in
+// global memory of the current device, built on first use; nullptr on error.
+const uint32_t *walk_table(int device);
+
 // Host feed: SplitMix64 counter-hash stream (R9), SoA rows.
 //   out[r*pitch + i] = word32(seed, tg0 + i, k0 + r),  r < nrows, i < count
 // nt: stream the stores past the CPU caches (bursty feeds; see feed.cpp).

@@ -14,6 +14,8 @@
 #include <cstdint>
 #include <cstdlib>
 #include <cstring>
+#include <map>
+#include <mutex>
 #include <type_traits>
 
 #include <cuda.h>
@@ -842,49 +844,28 @@ __device__ __forceinline__ void gg_build_table(uint32_t *tab) {
     __syncthreads();
 }
 
-// shared-memory byte offset of group G's entry: its 12 record bits times 4
-template <int G>
-__device__ __forceinline__ uint32_t gg_group_off(const uint32_t (&w)[6]) {
-    constexpr int bit = 12 * G, wi = bit >> 5, sh = bit & 31;
-    if (sh == 0) return (w[wi] << 2) & 0x3FFCu;
-    if (sh <= 20) return (w[wi] >> (sh - 2)) & 0x3FFCu;
-    return __funnelshift_r(w[wi], w[wi + 1], sh - 2) & 0x3FFCu;
+__global__ void gg_table_init_kernel(uint32_t *tab) {
+    const uint32_t p = blockIdx.x * blockDim.x + threadIdx.x;
+    if (p < kTabEntries) tab[p] = gg_compose4(p);
 }
 
-// Left shifts by multiplications with opaque powers of two (IMAD on the
-// FMA-heavy pipe), right shifts and masks on the ALU pipe: ptxas would
-// otherwise fuse each (t << s) >> r into SHF + LOP3 and put the whole unpack
-// on the ALU pipe.
-struct TabShifts {
-    uint32_t k22, k17, k12, k6;
-};
-__device__ __forceinline__ TabShifts gg_tab_shifts() {
-    TabShifts k{1u << 22, 1u << 17, 1u << 12, 1u << 6};
-    asm volatile("" : "+r"(k.k22), "+r"(k.k17), "+r"(k.k12), "+r"(k.k6));
-    return k;
-}
-
-__device__ __forceinline__ void gg_group_apply(const uint32_t *tab, uint32_t off, uint32_t &x,
-                                               uint32_t &y, const TabShifts &k) {
-    const uint32_t t = *reinterpret_cast<const uint32_t *>(reinterpret_cast<const char *>(tab) + off);
-    const uint32_t a = t & 31u, b = (t * k.k22) >> 27, c = (t * k.k17) >> 27, d = (t * k.k12) >> 27;
-    const uint32_t e = (t * k.k6) >> 26, f = t >> 26;
-    const uint32_t nx = b * y + (a * x + e);
-    const uint32_t ny = d * y + (c * x + f);
-    x = nx;
-    y = ny;
-}
-
-__device__ __forceinline__ void gg_walk64x2_table(const uint32_t *tab, const uint32_t (&wa)[6],
-                                                  const uint32_t (&wb)[6], uint32_t &xa,
-                                                  uint32_t &ya, uint32_t &xb, uint32_t &yb,
-                                                  const TabShifts &k) {
-#define GG_TG(G)                                           \
-    gg_group_apply(tab, gg_group_off<G>(wa), xa, ya, k);   \
-    gg_group_apply(tab, gg_group_off<G>(wb), xb, yb, k);
-    GG_TG(0) GG_TG(1) GG_TG(2) GG_TG(3) GG_TG(4) GG_TG(5) GG_TG(6) GG_TG(7)
-    GG_TG(8) GG_TG(9) GG_TG(10) GG_TG(11) GG_TG(12) GG_TG(13) GG_TG(14) GG_TG(15)
-#undef GG_TG
+// The table in global memory, once per device (prng_view::tab, staged into
+// shared memory by the on-demand consumers).
+const uint32_t *walk_table(int device) {
+    static std::mutex mu;
+    static std::map<int, uint32_t *> tabs;
+    std::lock_guard<std::mutex> lk(mu);
+    auto it = tabs.find(device);
+    if (it != tabs.end()) return it->second;
+    uint32_t *t = nullptr;
+    if (cudaMalloc(&t, kTabEntries * 4) != cudaSuccess) return nullptr;
+    gg_table_init_kernel<<<kTabEntries / 256, 256>>>(t);
+    if (cudaDeviceSynchronize() != cudaSuccess) {
+        cudaFree(t);
+        return nullptr;
+    }
+    tabs[device] = t;
+    return t;
 }
 
 // The pair kernel (adjacent walkers per lane, per-warp TMA, two stages) with
@@ -909,7 +890,7 @@ __global__ void __launch_bounds__(NW * 32) gg_fill64t_tma_kernel(const __grid_co
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     gg_build_table(tab);  // includes __syncthreads
-    const TabShifts ksh = gg_tab_shifts();
+    const prng_tab_shifts ksh = prng_tab_shifts_load();
     uint32_t ph0 = 0, ph1 = 0;
     const uint32_t kBytes = kTile * 4;
     for (uint32_t u = warp; u < units64; u += nwarps) {
@@ -967,7 +948,7 @@ __global__ void __launch_bounds__(NW * 32) gg_fill64t_tma_kernel(const __grid_co
             mbar_wait(bar, ph);
             uint32_t wa[6], wb[6];
             load(buf, wa, wb);
-            gg_walk64x2_table(tab, wa, wb, xa, ya, xb, yb, ksh);
+            prng_walk64x2_table(tab, wa, wb, xa, ya, xb, yb, ksh);
             const uint64_t idx = (uint64_t)j * a.W + ta - a.g_origin;
             if (EMIT == 0 && V4) {
                 *reinterpret_cast<uint4 *>(reinterpret_cast<uint2 *>(a.out) + idx) =
@@ -983,7 +964,7 @@ __global__ void __launch_bounds__(NW * 32) gg_fill64t_tma_kernel(const __grid_co
             uint32_t wa[6], wb[6];
             load(buf, wa, wb);
             uint32_t nxa = xa, nya = ya, nxb = xb, nyb = yb;
-            gg_walk64x2_table(tab, wa, wb, nxa, nya, nxb, nyb, ksh);
+            prng_walk64x2_table(tab, wa, wb, nxa, nya, nxb, nyb, ksh);
             if (j >= ja0 && j < ja1) {
                 xa = nxa;
                 ya = nya;

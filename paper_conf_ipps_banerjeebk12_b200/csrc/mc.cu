@@ -156,6 +156,10 @@ __global__ void __launch_bounds__(128, MINB) mc_epoch(const __grid_constant__ pr
                                                 unsigned long long *tallies,
                                                 long long *per_thread,
                                                 unsigned long long *counters) {
+    // the paper's generator (PRNG_WALK_L64): composed-step table in shared memory
+    constexpr bool TAB = MODE == PRNG_WALK_L64;
+    __shared__ __align__(16) uint32_t tab[TAB ? PRNG_TABLE_WORDS : 4];
+    if (TAB) prng_table_stage(&v, tab);  // made visible by the __syncthreads below
     const uint64_t slot = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const int nt = kFixed + P.nl;
     // block tallies in shared memory (int64 atomics: exact, order independent)
@@ -186,7 +190,10 @@ __global__ void __launch_bounds__(128, MINB) mc_epoch(const __grid_constant__ pr
             if (!alive && launched == budget) break;
             // three draws at a convergent point (R22), their loads in flight together
             uint64_t d3[3];
-            prng_next_n<3, true, MODE>(&st, &v, d3);
+            if (TAB)
+                prng_next_n_table<3, true>(&st, &v, tab, d3);
+            else
+                prng_next_n<3, true, MODE>(&st, &v, d3);
             const uint64_t la = d3[0], lb = d3[1], lc = d3[2];
             draws += 3;
             if (!alive) {

@@ -214,6 +214,7 @@ struct Timeline {
 
 struct prng_s {
     Timeline *tl = nullptr;
+    const uint32_t *walk_tab = nullptr;  // composed-step table of the device (gg::walk_table)
     prng_graph_params g{};
     prng_options o{};
     uint64_t W = 0, seed = 0;
@@ -681,6 +682,8 @@ int prng_create(prng_t **out, const prng_graph_params *g, uint64_t walkers, uint
             }
         }
         h->pool = new ThreadPool(nt, cpus);
+        h->walk_tab = gg::walk_table(o.device);
+        if (!h->walk_tab) CK(cudaErrorMemoryAllocation);
         if (const char *tp = getenv("GG_TIMELINE")) {
             h->tl = new Timeline();
             h->tl->path = tp;
@@ -1144,6 +1147,7 @@ int prng_device_view(prng_t *h, void *view, size_t view_bytes) {
     v.pow2 = h->pow2;
     v.variant = h->g.variant;
     v.l0 = h->g.burnin_len;
+    v.tab = h->walk_tab;
     memcpy(view, &v, sizeof(v));
     return PRNG_OK;
 }
