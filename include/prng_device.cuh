@@ -467,13 +467,16 @@ __device__ __forceinline__ void gg_walk64x2_r2p(const uint32_t a[6], const uint3
  * ------------------------------------------------------------------------ */
 #define PRNG_TABLE_WORDS 4096
 
-/* Shared-memory byte offset of group G's entry: its 12 record bits times 4. */
+/* Shared-space address of group G's entry: base | (its 12 record bits times
+ * 4).  The table is aligned to PRNG_TABLE_ALIGN bytes in shared memory, so
+ * the OR is an add and folds into the masking LOP3 (one instruction). */
+#define PRNG_TABLE_ALIGN 16384
 template <int G>
-__device__ __forceinline__ uint32_t prng_group_off(const uint32_t (&w)[6]) {
+__device__ __forceinline__ uint32_t prng_group_off(const uint32_t (&w)[6], uint32_t base) {
     constexpr int bit = 12 * G, wi = bit >> 5, sh = bit & 31;
-    if (sh == 0) return (w[wi] << 2) & 0x3FFCu;
-    if (sh <= 20) return (w[wi] >> (sh - 2)) & 0x3FFCu;
-    return __funnelshift_r(w[wi], w[wi + 1], sh - 2) & 0x3FFCu;
+    if constexpr (sh == 0) return ((w[wi] << 2) & 0x3FFCu) | base;
+    else if constexpr (sh <= 20) return ((w[wi] >> (sh - 2)) & 0x3FFCu) | base;
+    else return (__funnelshift_r(w[wi], w[wi + 1], sh - 2) & 0x3FFCu) | base;
 }
 
 // Left shifts by multiplications with opaque powers of two (IMAD on the
@@ -489,9 +492,10 @@ __device__ __forceinline__ prng_tab_shifts prng_tab_shifts_load() {
     return k;
 }
 
-__device__ __forceinline__ void prng_group_apply(const uint32_t *tab, uint32_t off, uint32_t &x,
-                                               uint32_t &y, const prng_tab_shifts &k) {
-    const uint32_t t = *reinterpret_cast<const uint32_t *>(reinterpret_cast<const char *>(tab) + off);
+__device__ __forceinline__ void prng_group_apply(uint32_t addr, uint32_t &x, uint32_t &y,
+                                                 const prng_tab_shifts &k) {
+    uint32_t t;
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(t) : "r"(addr));
     const uint32_t a = t & 31u, b = (t * k.k22) >> 27, c = (t * k.k17) >> 27, d = (t * k.k12) >> 27;
     const uint32_t e = (t * k.k6) >> 26, f = t >> 26;
     const uint32_t nx = b * y + (a * x + e);
@@ -500,13 +504,19 @@ __device__ __forceinline__ void prng_group_apply(const uint32_t *tab, uint32_t o
     y = ny;
 }
 
+/* Shared-space address (32-bit) of a PRNG_TABLE_ALIGN-aligned table. */
+__device__ __forceinline__ uint32_t prng_table_base(const uint32_t *smem_tab) {
+    return (uint32_t)__cvta_generic_to_shared(smem_tab);
+}
+
 __device__ __forceinline__ void prng_walk64x2_table(const uint32_t *tab, const uint32_t (&wa)[6],
                                                   const uint32_t (&wb)[6], uint32_t &xa,
                                                   uint32_t &ya, uint32_t &xb, uint32_t &yb,
                                                   const prng_tab_shifts &k) {
+    const uint32_t base = prng_table_base(tab);
 #define PRNG_TG(G)                                           \
-    prng_group_apply(tab, prng_group_off<G>(wa), xa, ya, k);   \
-    prng_group_apply(tab, prng_group_off<G>(wb), xb, yb, k);
+    prng_group_apply(prng_group_off<G>(wa, base), xa, ya, k);   \
+    prng_group_apply(prng_group_off<G>(wb, base), xb, yb, k);
     PRNG_TG(0) PRNG_TG(1) PRNG_TG(2) PRNG_TG(3) PRNG_TG(4) PRNG_TG(5) PRNG_TG(6) PRNG_TG(7)
     PRNG_TG(8) PRNG_TG(9) PRNG_TG(10) PRNG_TG(11) PRNG_TG(12) PRNG_TG(13) PRNG_TG(14) PRNG_TG(15)
 #undef PRNG_TG
@@ -517,7 +527,8 @@ __device__ __forceinline__ void prng_walk64_table(const uint32_t *tab, const uin
                                                   uint32_t &x, uint32_t &y,
                                                   const prng_tab_shifts &k)
 {
-#define PRNG_TG1(G) prng_group_apply(tab, prng_group_off<G>(w), x, y, k);
+    const uint32_t base = prng_table_base(tab);
+#define PRNG_TG1(G) prng_group_apply(prng_group_off<G>(w, base), x, y, k);
     PRNG_TG1(0) PRNG_TG1(1) PRNG_TG1(2) PRNG_TG1(3) PRNG_TG1(4) PRNG_TG1(5) PRNG_TG1(6) PRNG_TG1(7)
     PRNG_TG1(8) PRNG_TG1(9) PRNG_TG1(10) PRNG_TG1(11) PRNG_TG1(12) PRNG_TG1(13) PRNG_TG1(14) PRNG_TG1(15)
 #undef PRNG_TG1
@@ -802,12 +813,13 @@ __device__ __forceinline__ void prng_next_n(prng_state *st, const prng_view *v, 
 
 /* ---------------- on demand with the composed-step table ----------------
  * For views with prng_walk_mode(v) == PRNG_WALK_L64 (the paper's generator):
- *     __shared__ uint32_t tab[PRNG_TABLE_WORDS];        // 16 KB per block
+ *     __shared__ __align__(PRNG_TABLE_ALIGN) uint32_t tab[PRNG_TABLE_WORDS];  // 16 KB
  *     prng_table_stage(&view, tab);  __syncthreads();   // every thread of the block
  *     ... uint64_t r = prng_next_table(&st, &view, tab);
  * Same numbers as prng_next; other views ignore the table (prng_next). */
 __device__ __forceinline__ void prng_table_stage(const prng_view *v, uint32_t *smem_tab)
 {
+    if (prng_table_base(smem_tab) & (PRNG_TABLE_ALIGN - 1)) __trap();  /* see PRNG_TABLE_ALIGN */
     const uint4 *src = reinterpret_cast<const uint4 *>(v->tab);
     uint4 *dst = reinterpret_cast<uint4 *>(smem_tab);
     const uint32_t nthreads = blockDim.x * blockDim.y * blockDim.z;

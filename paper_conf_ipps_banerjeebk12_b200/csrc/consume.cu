@@ -23,7 +23,7 @@ __global__ void __launch_bounds__(128) consume_kernel(const __grid_constant__ pr
                                                       uint64_t *xor_out) {
     // the paper's generator (PRNG_WALK_L64): composed-step table in shared memory
     constexpr bool TAB = MODE == PRNG_WALK_L64;
-    __shared__ __align__(16) uint32_t tab[TAB ? PRNG_TABLE_WORDS : 4];
+    __shared__ __align__(PRNG_TABLE_ALIGN) uint32_t tab[TAB ? PRNG_TABLE_WORDS : 4];
     if (TAB) {
         prng_table_stage(&v, tab);
         __syncthreads();

@@ -876,9 +876,9 @@ template <int NW, int EMIT, bool V4>
 __global__ void __launch_bounds__(NW * 32) gg_fill64t_tma_kernel(const __grid_constant__ CUtensorMap tmap,
                                                                  FillArgs a, uint32_t units64) {
     constexpr int kTile = 6 * 64;
+    __shared__ __align__(PRNG_TABLE_ALIGN) uint32_t tab[kTabEntries];
     __shared__ __align__(128) uint32_t tiles[NW][2][kTile];
     __shared__ __align__(8) uint64_t bars[NW][2];
-    __shared__ __align__(16) uint32_t tab[kTabEntries];
     const uint32_t lane = threadIdx.x & 31u, wib = threadIdx.x >> 5;
     const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
@@ -889,6 +889,7 @@ __global__ void __launch_bounds__(NW * 32) gg_fill64t_tma_kernel(const __grid_co
         mbar_init(bar1, 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
+    if (prng_table_base(tab) & (PRNG_TABLE_ALIGN - 1)) __trap();  // the OR-addressing needs it
     gg_build_table(tab);  // includes __syncthreads
     const prng_tab_shifts ksh = prng_tab_shifts_load();
     uint32_t ph0 = 0, ph1 = 0;

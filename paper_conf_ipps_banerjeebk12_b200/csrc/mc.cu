@@ -158,7 +158,7 @@ __global__ void __launch_bounds__(128, MINB) mc_epoch(const __grid_constant__ pr
                                                 unsigned long long *counters) {
     // the paper's generator (PRNG_WALK_L64): composed-step table in shared memory
     constexpr bool TAB = MODE == PRNG_WALK_L64;
-    __shared__ __align__(16) uint32_t tab[TAB ? PRNG_TABLE_WORDS : 4];
+    __shared__ __align__(PRNG_TABLE_ALIGN) uint32_t tab[TAB ? PRNG_TABLE_WORDS : 4];
     if (TAB) prng_table_stage(&v, tab);  // made visible by the __syncthreads below
     const uint64_t slot = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const int nt = kFixed + P.nl;
