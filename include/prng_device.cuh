@@ -492,12 +492,24 @@ __device__ __forceinline__ prng_tab_shifts prng_tab_shifts_load() {
     return k;
 }
 
+/* SIGNED: the bipartite table's two's-complement fields (arithmetic shifts). */
+template <bool SIGNED = false>
 __device__ __forceinline__ void prng_group_apply(uint32_t addr, uint32_t &x, uint32_t &y,
                                                  const prng_tab_shifts &k) {
     uint32_t t;
     asm volatile("ld.shared.u32 %0, [%1];" : "=r"(t) : "r"(addr));
-    const uint32_t a = t & 31u, b = (t * k.k22) >> 27, c = (t * k.k17) >> 27, d = (t * k.k12) >> 27;
-    const uint32_t e = (t * k.k6) >> 26, f = t >> 26;
+    uint32_t a, b, c, d, e, f;
+    if (SIGNED) {
+        a = (uint32_t)((int32_t)(t << 27) >> 27);
+        b = (uint32_t)((int32_t)(t * k.k22) >> 27);
+        c = (uint32_t)((int32_t)(t * k.k17) >> 27);
+        d = (uint32_t)((int32_t)(t * k.k12) >> 27);
+        e = (uint32_t)((int32_t)(t * k.k6) >> 26);
+        f = (uint32_t)((int32_t)t >> 26);
+    } else {
+        a = t & 31u, b = (t * k.k22) >> 27, c = (t * k.k17) >> 27, d = (t * k.k12) >> 27;
+        e = (t * k.k6) >> 26, f = t >> 26;
+    }
     const uint32_t nx = b * y + (a * x + e);
     const uint32_t ny = d * y + (c * x + f);
     x = nx;
@@ -509,14 +521,15 @@ __device__ __forceinline__ uint32_t prng_table_base(const uint32_t *smem_tab) {
     return (uint32_t)__cvta_generic_to_shared(smem_tab);
 }
 
+template <bool SIGNED = false>
 __device__ __forceinline__ void prng_walk64x2_table(const uint32_t *tab, const uint32_t (&wa)[6],
                                                   const uint32_t (&wb)[6], uint32_t &xa,
                                                   uint32_t &ya, uint32_t &xb, uint32_t &yb,
                                                   const prng_tab_shifts &k) {
     const uint32_t base = prng_table_base(tab);
 #define PRNG_TG(G)                                           \
-    prng_group_apply(prng_group_off<G>(wa, base), xa, ya, k);   \
-    prng_group_apply(prng_group_off<G>(wb, base), xb, yb, k);
+    prng_group_apply<SIGNED>(prng_group_off<G>(wa, base), xa, ya, k);   \
+    prng_group_apply<SIGNED>(prng_group_off<G>(wb, base), xb, yb, k);
     PRNG_TG(0) PRNG_TG(1) PRNG_TG(2) PRNG_TG(3) PRNG_TG(4) PRNG_TG(5) PRNG_TG(6) PRNG_TG(7)
     PRNG_TG(8) PRNG_TG(9) PRNG_TG(10) PRNG_TG(11) PRNG_TG(12) PRNG_TG(13) PRNG_TG(14) PRNG_TG(15)
 #undef PRNG_TG

@@ -839,8 +839,35 @@ __device__ __forceinline__ uint32_t gg_compose4(uint32_t p) {
     return a | b << 5 | c << 10 | d << 15 | e << 20 | f << 26;
 }
 
+// Bipartite variant: a group starts at an even global step
+// (l0 even, l = 64), so its steps are sigma, sigma^-1, sigma, sigma^-1; the
+// inverse steps subtract (y -= 2x + c | x -= 2y + c) and the composed
+// coefficients lie in [-8, 8] (a..d) and [-12, 14] (e, f): the same
+// 5-5-5-5-6-6 fields, two's complement, unpacked with arithmetic shifts.
+__device__ __forceinline__ uint32_t gg_compose4_bip(uint32_t p) {
+    int32_t a = 1, b = 0, e = 0, c = 0, d = 1, f = 0;
+#pragma unroll
+    for (int i = 0; i < 4; i++) {
+        const int32_t k = (int32_t)(((p >> (3 * i)) & 7u) % 7u);
+        const int32_t sg = (i & 1) ? -1 : 1;
+        if (k >= 1 && k <= 3) {
+            c += sg * 2 * a;
+            d += sg * 2 * b;
+            f += sg * (2 * e + (k - 1));
+        } else if (k >= 4) {
+            a += sg * 2 * c;
+            b += sg * 2 * d;
+            e += sg * (2 * f + (k - 4));
+        }
+    }
+    return ((uint32_t)a & 31u) | ((uint32_t)b & 31u) << 5 | ((uint32_t)c & 31u) << 10 |
+           ((uint32_t)d & 31u) << 15 | ((uint32_t)e & 63u) << 20 | ((uint32_t)f & 63u) << 26;
+}
+
+template <bool BIP = false>
 __device__ __forceinline__ void gg_build_table(uint32_t *tab) {
-    for (uint32_t p = threadIdx.x; p < kTabEntries; p += blockDim.x) tab[p] = gg_compose4(p);
+    for (uint32_t p = threadIdx.x; p < kTabEntries; p += blockDim.x)
+        tab[p] = BIP ? gg_compose4_bip(p) : gg_compose4(p);
     __syncthreads();
 }
 
@@ -872,7 +899,7 @@ const uint32_t *walk_table(int device) {
 // the composed-step walk; NW warps per block share one table.  EMIT: 0 = u64
 // label for m = 2^32 ((y << 32) | x), 1 = u64 label for m = 2^k < 2^32,
 // 2 = low u32 word (m <= 2^16); V4: 16-byte stores of two m = 2^32 labels.
-template <int NW, int EMIT, bool V4>
+template <int NW, int EMIT, bool V4, bool BIP = false>
 __global__ void __launch_bounds__(NW * 32) gg_fill64t_tma_kernel(const __grid_constant__ CUtensorMap tmap,
                                                                  FillArgs a, uint32_t units64) {
     constexpr int kTile = 6 * 64;
@@ -890,7 +917,7 @@ __global__ void __launch_bounds__(NW * 32) gg_fill64t_tma_kernel(const __grid_co
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     if (prng_table_base(tab) & (PRNG_TABLE_ALIGN - 1)) __trap();  // the OR-addressing needs it
-    gg_build_table(tab);  // includes __syncthreads
+    gg_build_table<BIP>(tab);  // includes __syncthreads
     const prng_tab_shifts ksh = prng_tab_shifts_load();
     uint32_t ph0 = 0, ph1 = 0;
     const uint32_t kBytes = kTile * 4;
@@ -949,7 +976,7 @@ __global__ void __launch_bounds__(NW * 32) gg_fill64t_tma_kernel(const __grid_co
             mbar_wait(bar, ph);
             uint32_t wa[6], wb[6];
             load(buf, wa, wb);
-            prng_walk64x2_table(tab, wa, wb, xa, ya, xb, yb, ksh);
+            prng_walk64x2_table<BIP>(tab, wa, wb, xa, ya, xb, yb, ksh);
             const uint64_t idx = (uint64_t)j * a.W + ta - a.g_origin;
             if (EMIT == 0 && V4) {
                 *reinterpret_cast<uint4 *>(reinterpret_cast<uint2 *>(a.out) + idx) =
@@ -965,7 +992,7 @@ __global__ void __launch_bounds__(NW * 32) gg_fill64t_tma_kernel(const __grid_co
             uint32_t wa[6], wb[6];
             load(buf, wa, wb);
             uint32_t nxa = xa, nya = ya, nxb = xb, nyb = yb;
-            prng_walk64x2_table(tab, wa, wb, nxa, nya, nxb, nyb, ksh);
+            prng_walk64x2_table<BIP>(tab, wa, wb, nxa, nya, nxb, nyb, ksh);
             if (j >= ja0 && j < ja1) {
                 xa = nxa;
                 ya = nya;
@@ -1467,6 +1494,22 @@ cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count) {
     // = 28 warps per SM, shared memory bound; C2 A/B 4.78 / 5.01 / 5.22 ms for
     // 4 / 8 / 2, 5.08 ms for 8 warps at 48 registers), 0 = the R2P kernels
     static const int table_nw = getenv("GG_FILL_TABLE") ? atoi(getenv("GG_FILL_TABLE")) : 4;
+    if (a.l == 64 && a.pow2 && a.variant == 1 && (a.l0 & 1u) == 0 && table_nw > 0 && a.rows &&
+        getenv("GG_FILL_NO_BIP") == nullptr) {
+        // bipartite variant: the signed composed-step table (4 warps per block)
+        CUtensorMap map;
+        const uint32_t units64 = (a.W + 63u) / 64u;
+        if (make_window_map(&map, a.bits, a.pitch, a.rows, 64)) {
+            const uint32_t blocks = (units64 + 3) / 4;
+            if (a.out_u32)
+                gg_fill64t_tma_kernel<4, 2, false, true><<<blocks, 128, 0, s>>>(map, a, units64);
+            else if (a.log2m != 32)
+                gg_fill64t_tma_kernel<4, 1, false, true><<<blocks, 128, 0, s>>>(map, a, units64);
+            else
+                gg_fill64t_tma_kernel<4, 0, false, true><<<blocks, 128, 0, s>>>(map, a, units64);
+            return cudaGetLastError();
+        }
+    }
     if (a.l == 64 && a.pow2 && a.variant == 0 && table_nw > 0 && a.rows) {
         CUtensorMap map;
         const uint32_t units64 = (a.W + 63u) / 64u;

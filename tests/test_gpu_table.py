@@ -1,7 +1,8 @@
 """The composed-step table fill kernel (GG_FILL_TABLE = warps per block,
 csrc/gg_walk.cu gg_fill64t_tma_kernel) is bit-exact with the oracle for every
 m = 2^k output form it serves (u64 labels of m = 2^32 with and without the
-16-byte store path, u64 labels of m = 2^k < 2^32, u32 words of m <= 2^16), on
+16-byte store path, u64 labels of m = 2^k < 2^32, u32 words of m <= 2^16) and
+for the bipartite variant's signed table, on
 ragged walker counts and fills that stop mid-draw.  The hook is read once per
 process, so each configuration runs in a subprocess."""
 import json
@@ -23,9 +24,10 @@ import numpy as np, torch
 sys.path.insert(0, %(root)r)
 from paper_conf_ipps_banerjeebk12_b200 import Generator
 res = {}
-for m, W, fmt in ((1 << 32, 1000, "u64"), (1 << 32, 999, "u64"), (1 << 32, 4096, "u32"),
-                  (256, 1000, "u64"), (1 << 20, 777, "u64"), (1 << 16, 640, "u32")):
-    g = Generator(walkers=W, seed=0x7AB1E + W, m=m, epoch_draws=5)
+for m, W, fmt, var in ((1 << 32, 1000, "u64", 0), (1 << 32, 999, "u64", 0), (1 << 32, 4096, "u32", 0),
+                       (256, 1000, "u64", 0), (1 << 20, 777, "u64", 0), (1 << 16, 640, "u32", 0),
+                       (1 << 32, 1000, "u64", 1), (1 << 12, 333, "u64", 1)):
+    g = Generator(walkers=W, seed=0x7AB1E + W, m=m, epoch_draws=5, variant=var)
     outs = []
     for n in (7, 3 * W + 5, 2 * W + 2, 9 * W):
         if fmt == "u64":
@@ -41,7 +43,7 @@ for m, W, fmt in ((1 << 32, 1000, "u64"), (1 << 32, 999, "u64"), (1 << 32, 4096,
     o = torch.empty(12 * W, dtype=torch.int64, device="cuda")
     g.fill(o)
     outs.append(o.cpu().numpy().view(np.uint64))
-    res[f"{m}-{W}-{fmt}"] = [int(v) for v in np.concatenate(outs)]
+    res[f"{m}-{W}-{fmt}-{var}"] = [int(v) for v in np.concatenate(outs)]
 print(json.dumps(res))
 """
 
@@ -54,10 +56,10 @@ def test_table_kernel_bit_exact(nw):
     assert p.returncode == 0, p.stderr[-2000:]
     got = json.loads(p.stdout.strip().splitlines()[-1])
     for key, vals in got.items():
-        m, W, fmt = key.split("-")
-        m, W = int(m), int(W)
+        m, W, fmt, var = key.split("-")
+        m, W, var = int(m), int(W), int(var)
         total = 7 + (3 * W + 5) + (2 * W + 2) + 9 * W
         n_pref = 12 * W
         # fills continue from the running N (R11), the resident window included
-        want = O.bulk(m, 64, 64, 0x7AB1E + W, W, 0, total + n_pref)
+        want = O.bulk_v(m, 64, 64, var, 0x7AB1E + W, W, 0, total + n_pref)
         assert np.array_equal(np.array(vals, dtype=np.uint64), want), (nw, key)

@@ -101,3 +101,61 @@ def test_power_of_two_moduli_reduce_at_emission():
             x, y = walk64_table(w, x0, y0)
             assert (x & ((1 << k) - 1), y & ((1 << k) - 1)) == O.walk(
                 1 << k, x0, y0, np.array(w, np.uint32), 64)
+
+
+# ---------------------------------------------------------------------------
+# Bipartite variant: a group starts at an even global step,
+# so it applies sigma, sigma^-1, sigma, sigma^-1; signed 5-5-5-5-6-6 fields.
+
+def compose4_bip(p):
+    a, b, e, c, d, f = 1, 0, 0, 0, 1, 0
+    for i in range(4):
+        k = ((p >> (3 * i)) & 7) % 7
+        sg = -1 if i & 1 else 1
+        if 1 <= k <= 3:
+            c, d, f = c + sg * 2 * a, d + sg * 2 * b, f + sg * (2 * e + (k - 1))
+        elif k >= 4:
+            a, b, e = a + sg * 2 * c, b + sg * 2 * d, e + sg * (2 * f + (k - 4))
+    return a, b, c, d, e, f
+
+
+def pack_signed(co):
+    a, b, c, d, e, f = co
+    return (a & 31) | (b & 31) << 5 | (c & 31) << 10 | (d & 31) << 15 | (e & 63) << 20 | (f & 63) << 26
+
+
+def sx(v, bits):
+    return v - (1 << bits) if v >> (bits - 1) else v
+
+
+def unpack_signed(t):
+    return (sx(t & 31, 5), sx((t >> 5) & 31, 5), sx((t >> 10) & 31, 5), sx((t >> 15) & 31, 5),
+            sx((t >> 20) & 63, 6), sx(t >> 26, 6))
+
+
+TAB_BIP = [pack_signed(compose4_bip(p)) for p in range(4096)]
+
+
+def test_bipartite_coefficient_bounds_fit_signed_fields():
+    lo, hi = [0] * 6, [0] * 6
+    for p in range(4096):
+        for i, v in enumerate(compose4_bip(p)):
+            lo[i], hi[i] = min(lo[i], v), max(hi[i], v)
+    assert lo == [-7, -8, -8, -7, -12, -12] and hi == [5, 8, 8, 5, 14, 14]
+    assert all(unpack_signed(TAB_BIP[p]) == compose4_bip(p) for p in range(4096))
+
+
+def test_bipartite_table_walk_equals_definition():
+    rng = np.random.default_rng(80)
+    for _ in range(1000):
+        w = [int(v) for v in rng.integers(0, 2 ** 32, 6, dtype=np.uint64)]
+        x, y = (int(v) for v in rng.integers(0, 2 ** 32, 2, dtype=np.uint64))
+        x0, y0 = x, y
+        for g in range(16):
+            a, b, c, d, e, f = unpack_signed(TAB_BIP[group_off4(w, g) >> 2])
+            x, y = (b * y + a * x + e) & M, (d * y + c * x + f) & M
+        rec = np.array(w, np.uint32)
+        xs, ys = np.array([x0], np.uint64), np.array([y0], np.uint64)
+        s0 = 64 * int(rng.integers(1, 1000))  # l0 + 64 j: even
+        O.lib().or_walk_bipartite(1 << 32, xs.ctypes.data, ys.ctypes.data, rec.ctypes.data, 64, s0)
+        assert (x, y) == (int(xs[0]), int(ys[0]))
