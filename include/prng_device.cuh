@@ -467,16 +467,22 @@ __device__ __forceinline__ void gg_walk64x2_r2p(const uint32_t a[6], const uint3
  * ------------------------------------------------------------------------ */
 #define PRNG_TABLE_WORDS 4096
 
-/* Shared-space address of group G's entry: base | (its 12 record bits times
- * 4).  The table is aligned to PRNG_TABLE_ALIGN bytes in shared memory, so
- * the OR is an add and folds into the masking LOP3 (one instruction). */
-#define PRNG_TABLE_ALIGN 16384
-template <int G>
+/* Shared-space address of group G's entry: base + its 12 record bits times
+ * 4.  The base is warp-uniform, so ptxas folds the add into the LDS address
+ * ([R + UR]).  (An OR with a 16 KB-aligned base is not portable: the CTA's
+ * shared window begins with a reserved 1 KB, and ptxas does not honour
+ * larger alignments of __shared__ variables.) */
+#define PRNG_TABLE_ALIGN 16
+template <int G, bool ORB = false>
 __device__ __forceinline__ uint32_t prng_group_off(const uint32_t (&w)[6], uint32_t base) {
     constexpr int bit = 12 * G, wi = bit >> 5, sh = bit & 31;
-    if constexpr (sh == 0) return ((w[wi] << 2) & 0x3FFCu) | base;
-    else if constexpr (sh <= 20) return ((w[wi] >> (sh - 2)) & 0x3FFCu) | base;
-    else return (__funnelshift_r(w[wi], w[wi + 1], sh - 2) & 0x3FFCu) | base;
+    uint32_t v;
+    if constexpr (sh == 0) v = w[wi] << 2;
+    else if constexpr (sh <= 20) v = w[wi] >> (sh - 2);
+    else v = __funnelshift_r(w[wi], w[wi + 1], sh - 2);
+    /* ORB: base is a multiple of 16 KB (library kernels that place the table
+     * so), and the OR folds into the masking LOP3 */
+    return ORB ? ((v & 0x3FFCu) | base) : ((v & 0x3FFCu) + base);
 }
 
 // Left shifts by multiplications with opaque powers of two (IMAD on the
@@ -497,7 +503,7 @@ template <bool SIGNED = false>
 __device__ __forceinline__ void prng_group_apply(uint32_t addr, uint32_t &x, uint32_t &y,
                                                  const prng_tab_shifts &k) {
     uint32_t t;
-    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(t) : "r"(addr));
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(t) : "r"(addr) : "memory");
     uint32_t a, b, c, d, e, f;
     if (SIGNED) {
         a = (uint32_t)((int32_t)(t << 27) >> 27);
@@ -516,9 +522,23 @@ __device__ __forceinline__ void prng_group_apply(uint32_t addr, uint32_t &x, uin
     y = ny;
 }
 
-/* Shared-space address (32-bit) of a PRNG_TABLE_ALIGN-aligned table. */
+/* Shared-space address (32-bit) of the staged table. */
 __device__ __forceinline__ uint32_t prng_table_base(const uint32_t *smem_tab) {
     return (uint32_t)__cvta_generic_to_shared(smem_tab);
+}
+
+/* Two walkers, table at shared-space address `base`. */
+template <bool SIGNED = false, bool ORB = false>
+__device__ __forceinline__ void prng_walk64x2_table_at(uint32_t base, const uint32_t (&wa)[6],
+                                                       const uint32_t (&wb)[6], uint32_t &xa,
+                                                       uint32_t &ya, uint32_t &xb, uint32_t &yb,
+                                                       const prng_tab_shifts &k) {
+#define PRNG_TG(G)                                                                \
+    prng_group_apply<SIGNED>(prng_group_off<G, ORB>(wa, base), xa, ya, k);        \
+    prng_group_apply<SIGNED>(prng_group_off<G, ORB>(wb, base), xb, yb, k);
+    PRNG_TG(0) PRNG_TG(1) PRNG_TG(2) PRNG_TG(3) PRNG_TG(4) PRNG_TG(5) PRNG_TG(6) PRNG_TG(7)
+    PRNG_TG(8) PRNG_TG(9) PRNG_TG(10) PRNG_TG(11) PRNG_TG(12) PRNG_TG(13) PRNG_TG(14) PRNG_TG(15)
+#undef PRNG_TG
 }
 
 template <bool SIGNED = false>
@@ -526,13 +546,7 @@ __device__ __forceinline__ void prng_walk64x2_table(const uint32_t *tab, const u
                                                   const uint32_t (&wb)[6], uint32_t &xa,
                                                   uint32_t &ya, uint32_t &xb, uint32_t &yb,
                                                   const prng_tab_shifts &k) {
-    const uint32_t base = prng_table_base(tab);
-#define PRNG_TG(G)                                           \
-    prng_group_apply<SIGNED>(prng_group_off<G>(wa, base), xa, ya, k);   \
-    prng_group_apply<SIGNED>(prng_group_off<G>(wb, base), xb, yb, k);
-    PRNG_TG(0) PRNG_TG(1) PRNG_TG(2) PRNG_TG(3) PRNG_TG(4) PRNG_TG(5) PRNG_TG(6) PRNG_TG(7)
-    PRNG_TG(8) PRNG_TG(9) PRNG_TG(10) PRNG_TG(11) PRNG_TG(12) PRNG_TG(13) PRNG_TG(14) PRNG_TG(15)
-#undef PRNG_TG
+    prng_walk64x2_table_at<SIGNED, false>(prng_table_base(tab), wa, wb, xa, ya, xb, yb, k);
 }
 
 
@@ -832,7 +846,6 @@ __device__ __forceinline__ void prng_next_n(prng_state *st, const prng_view *v, 
  * Same numbers as prng_next; other views ignore the table (prng_next). */
 __device__ __forceinline__ void prng_table_stage(const prng_view *v, uint32_t *smem_tab)
 {
-    if (prng_table_base(smem_tab) & (PRNG_TABLE_ALIGN - 1)) __trap();  /* see PRNG_TABLE_ALIGN */
     const uint4 *src = reinterpret_cast<const uint4 *>(v->tab);
     uint4 *dst = reinterpret_cast<uint4 *>(smem_tab);
     const uint32_t nthreads = blockDim.x * blockDim.y * blockDim.z;

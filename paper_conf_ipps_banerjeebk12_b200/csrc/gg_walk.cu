@@ -899,13 +899,50 @@ const uint32_t *walk_table(int device) {
 // the composed-step walk; NW warps per block share one table.  EMIT: 0 = u64
 // label for m = 2^32 ((y << 32) | x), 1 = u64 label for m = 2^k < 2^32,
 // 2 = low u32 word (m <= 2^16); V4: 16-byte stores of two m = 2^32 labels.
-template <int NW, int EMIT, bool V4, bool BIP = false>
+// Shared-memory layout.  ORB (table at a 16 KB boundary of the shared
+// window, so the group offset ORs into the table base in the masking LOP3
+// instead of costing an add per lookup): one raw buffer, the record tiles and
+// barriers at its start and the table at the first 16 KB boundary after
+// them.  The CTA's shared window begins with a reserved 1 KB, so for the
+// buffer at window offset 1 KB the boundary is 15 KB in; the host probes the
+// buffer's address once (probe != nullptr: thread 0 reports it and the
+// kernel returns) and uses ORB only if the layout fits, else the plain
+// layout (table first, added base).
+template <int NW>
+struct FillTLayout {
+    static constexpr uint32_t kTile = 6 * 64;
+    static constexpr uint32_t kTileBytes = NW * 2 * kTile * 4;
+    static constexpr uint32_t kBarBytes = NW * 2 * 8;
+    static constexpr uint32_t kLead = kTileBytes + kBarBytes;   // bytes before the table (ORB)
+    static constexpr uint32_t kOrbRaw = 15 * 1024 + kTabEntries * 4;  // ORB buffer
+    static constexpr bool kOrbOk = kLead <= 15 * 1024;
+};
+
+template <int NW, int EMIT, bool V4, bool BIP = false, bool ORB = false>
 __global__ void __launch_bounds__(NW * 32) gg_fill64t_tma_kernel(const __grid_constant__ CUtensorMap tmap,
-                                                                 FillArgs a, uint32_t units64) {
-    constexpr int kTile = 6 * 64;
-    __shared__ __align__(PRNG_TABLE_ALIGN) uint32_t tab[kTabEntries];
-    __shared__ __align__(128) uint32_t tiles[NW][2][kTile];
-    __shared__ __align__(8) uint64_t bars[NW][2];
+                                                                 FillArgs a, uint32_t units64,
+                                                                 uint32_t *probe) {
+    using L = FillTLayout<NW>;
+    constexpr int kTile = L::kTile;
+    constexpr uint32_t kRaw = ORB ? L::kOrbRaw : kTabEntries * 4 + L::kTileBytes + L::kBarBytes;
+    __shared__ __align__(1024) unsigned char raw[kRaw];
+    const uint32_t raw_base = (uint32_t)__cvta_generic_to_shared(raw);
+    if (probe) {
+        if (threadIdx.x == 0 && blockIdx.x == 0) *probe = raw_base;
+        return;
+    }
+    uint32_t tab_off;  // byte offset of the table in raw
+    unsigned char *lead;
+    if (ORB) {
+        tab_off = ((raw_base + 0x3FFFu) & ~0x3FFFu) - raw_base;
+        lead = raw;
+    } else {
+        tab_off = 0;
+        lead = raw + kTabEntries * 4;
+    }
+    uint32_t *tab = reinterpret_cast<uint32_t *>(raw + tab_off);
+    auto tiles = reinterpret_cast<uint32_t (*)[2][kTile]>(lead);
+    auto bars = reinterpret_cast<uint64_t (*)[2]>(lead + L::kTileBytes);
     const uint32_t lane = threadIdx.x & 31u, wib = threadIdx.x >> 5;
     const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
@@ -916,8 +953,8 @@ __global__ void __launch_bounds__(NW * 32) gg_fill64t_tma_kernel(const __grid_co
         mbar_init(bar1, 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
-    if (prng_table_base(tab) & (PRNG_TABLE_ALIGN - 1)) __trap();  // the OR-addressing needs it
     gg_build_table<BIP>(tab);  // includes __syncthreads
+    const uint32_t tbase = raw_base + tab_off;
     const prng_tab_shifts ksh = prng_tab_shifts_load();
     uint32_t ph0 = 0, ph1 = 0;
     const uint32_t kBytes = kTile * 4;
@@ -976,7 +1013,7 @@ __global__ void __launch_bounds__(NW * 32) gg_fill64t_tma_kernel(const __grid_co
             mbar_wait(bar, ph);
             uint32_t wa[6], wb[6];
             load(buf, wa, wb);
-            prng_walk64x2_table<BIP>(tab, wa, wb, xa, ya, xb, yb, ksh);
+            prng_walk64x2_table_at<BIP, ORB>(tbase, wa, wb, xa, ya, xb, yb, ksh);
             const uint64_t idx = (uint64_t)j * a.W + ta - a.g_origin;
             if (EMIT == 0 && V4) {
                 *reinterpret_cast<uint4 *>(reinterpret_cast<uint2 *>(a.out) + idx) =
@@ -992,7 +1029,7 @@ __global__ void __launch_bounds__(NW * 32) gg_fill64t_tma_kernel(const __grid_co
             uint32_t wa[6], wb[6];
             load(buf, wa, wb);
             uint32_t nxa = xa, nya = ya, nxb = xb, nyb = yb;
-            prng_walk64x2_table<BIP>(tab, wa, wb, nxa, nya, nxb, nyb, ksh);
+            prng_walk64x2_table_at<BIP, ORB>(tbase, wa, wb, nxa, nya, nxb, nyb, ksh);
             if (j >= ja0 && j < ja1) {
                 xa = nxa;
                 ya = nya;
@@ -1494,6 +1531,27 @@ cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count) {
     // = 28 warps per SM, shared memory bound; C2 A/B 4.78 / 5.01 / 5.22 ms for
     // 4 / 8 / 2, 5.08 ms for 8 warps at 48 registers), 0 = the R2P kernels
     static const int table_nw = getenv("GG_FILL_TABLE") ? atoi(getenv("GG_FILL_TABLE")) : 4;
+    // ORB layout (table at a 16 KB boundary, FillTLayout): probed once per
+    // process; A/B hook GG_FILL_ORB=0 forces the plain layout
+    static int orb_state = -1;
+    if (orb_state < 0) {
+        orb_state = 0;
+        if (!(getenv("GG_FILL_ORB") && atoi(getenv("GG_FILL_ORB")) == 0)) {
+            uint32_t *d = nullptr, hbase = 0;
+            if (cudaMalloc(&d, 4) == cudaSuccess) {
+                CUtensorMap dummy{};
+                gg_fill64t_tma_kernel<4, 0, true, false, true><<<1, 128, 0, s>>>(dummy, a, 0, d);
+                if (cudaMemcpyAsync(&hbase, d, 4, cudaMemcpyDeviceToHost, s) == cudaSuccess &&
+                    cudaStreamSynchronize(s) == cudaSuccess) {
+                    const uint32_t off = ((hbase + 0x3FFFu) & ~0x3FFFu) - hbase;
+                    orb_state = (off >= FillTLayout<4>::kLead && off <= 15u * 1024u) ? 1 : 0;
+                }
+                cudaFree(d);
+            }
+        }
+        cudaGetLastError();  // a failed probe only disables the ORB layout
+    }
+    const bool orb = orb_state == 1;
     if (a.l == 64 && a.pow2 && a.variant == 1 && (a.l0 & 1u) == 0 && table_nw > 0 && a.rows &&
         getenv("GG_FILL_NO_BIP") == nullptr) {
         // bipartite variant: the signed composed-step table (4 warps per block)
@@ -1501,12 +1559,12 @@ cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count) {
         const uint32_t units64 = (a.W + 63u) / 64u;
         if (make_window_map(&map, a.bits, a.pitch, a.rows, 64)) {
             const uint32_t blocks = (units64 + 3) / 4;
-            if (a.out_u32)
-                gg_fill64t_tma_kernel<4, 2, false, true><<<blocks, 128, 0, s>>>(map, a, units64);
-            else if (a.log2m != 32)
-                gg_fill64t_tma_kernel<4, 1, false, true><<<blocks, 128, 0, s>>>(map, a, units64);
-            else
-                gg_fill64t_tma_kernel<4, 0, false, true><<<blocks, 128, 0, s>>>(map, a, units64);
+#define GG_LAUNCH_B(E, O)                                                                         \
+    gg_fill64t_tma_kernel<4, E, false, true, O><<<blocks, 128, 0, s>>>(map, a, units64, nullptr)
+            if (a.out_u32) { if (orb) GG_LAUNCH_B(2, true); else GG_LAUNCH_B(2, false); }
+            else if (a.log2m != 32) { if (orb) GG_LAUNCH_B(1, true); else GG_LAUNCH_B(1, false); }
+            else { if (orb) GG_LAUNCH_B(0, true); else GG_LAUNCH_B(0, false); }
+#undef GG_LAUNCH_B
             return cudaGetLastError();
         }
     }
@@ -1517,19 +1575,19 @@ cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count) {
             const bool v4 = (a.W % 2 == 0) && (a.g_origin % 2 == 0) && ((uintptr_t)a.out % 16 == 0);
             // one 64-walker unit per warp; A/B hook GG_FILL_KPW = units per warp
             static const int kpw_t = getenv("GG_FILL_KPW") ? std::max(1, atoi(getenv("GG_FILL_KPW"))) : 1;
-#define GG_LAUNCH_T(NW, E, V)                                                                    \
-    gg_fill64t_tma_kernel<NW, E, V><<<(units64 + NW * kpw_t - 1) / (NW * kpw_t), NW * 32, 0, s>>>( \
-        map, a, units64)
-#define GG_LAUNCH_TNW(NW)                                                                        \
-    do {                                                                                         \
-        if (a.out_u32) GG_LAUNCH_T(NW, 2, false);                                                \
-        else if (a.log2m != 32) GG_LAUNCH_T(NW, 1, false);                                       \
-        else if (v4) GG_LAUNCH_T(NW, 0, true);                                                   \
-        else GG_LAUNCH_T(NW, 0, false);                                                          \
+#define GG_LAUNCH_T(NW, E, V, O)                                                                  \
+    gg_fill64t_tma_kernel<NW, E, V, false, O>                                                     \
+        <<<(units64 + NW * kpw_t - 1) / (NW * kpw_t), NW * 32, 0, s>>>(map, a, units64, nullptr)
+#define GG_LAUNCH_TNW(NW, O)                                                                      \
+    do {                                                                                          \
+        if (a.out_u32) GG_LAUNCH_T(NW, 2, false, O);                                              \
+        else if (a.log2m != 32) GG_LAUNCH_T(NW, 1, false, O);                                     \
+        else if (v4) GG_LAUNCH_T(NW, 0, true, O);                                                 \
+        else GG_LAUNCH_T(NW, 0, false, O);                                                        \
     } while (0)
-            if (table_nw >= 8) GG_LAUNCH_TNW(8);
-            else if (table_nw >= 4) GG_LAUNCH_TNW(4);
-            else GG_LAUNCH_TNW(2);
+            if (table_nw >= 8) GG_LAUNCH_TNW(8, false);  // 8 warps' tiles exceed the ORB lead
+            else if (table_nw >= 4) { if (orb) GG_LAUNCH_TNW(4, true); else GG_LAUNCH_TNW(4, false); }
+            else { if (orb) GG_LAUNCH_TNW(2, true); else GG_LAUNCH_TNW(2, false); }
 #undef GG_LAUNCH_TNW
 #undef GG_LAUNCH_T
             return cudaGetLastError();

@@ -12,7 +12,7 @@ import subprocess
 
 LIB = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))),
                    "paper_conf_ipps_banerjeebk12_b200", "libggprng.so")
-KERNEL = "_ZN2gg21gg_fill64t_tma_kernelILi4ELi0ELb1EEEv14CUtensorMap_stNS_8FillArgsEj"
+KERNEL = "_ZN2gg21gg_fill64t_tma_kernelILi4ELi0ELb1ELb0ELb1EEEv14CUtensorMap_stNS_8FillArgsEjPj"
 ALU = ("LOP3", "SHF", "LEA", "IADD3", "R2P", "ISETP", "SEL", "PLOP3", "VIADD", "MOV", "LOP")
 
 out = subprocess.run(["cuobjdump", "-sass", LIB], capture_output=True, text=True, check=True).stdout
