@@ -1490,42 +1490,6 @@ cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count) {
             return cudaGetLastError();
         }
     }
-    if (a.l == 64 && a.pow2 && a.variant == 1 && (a.l0 & 1u) == 0 && a.rows &&
-        getenv("GG_FILL_NO_BIP") == nullptr) {
-        // bipartite variant (f1): every draw starts at an even global step
-        // (l0 + 64 j), so the fixed (sigma, sigma^-1) pairing of the R2P walk holds
-        CUtensorMap map;
-        const uint32_t units64 = (a.W + 63u) / 64u;
-        if (make_window_map(&map, a.bits, a.pitch, a.rows, 64)) {
-            if (a.out_u32) {
-                plan_grid(gg_fill64x2_tma_kernel<2, 1, 1, 1, true>, units64, sm_count, blocks, threads);
-                gg_fill64x2_tma_kernel<2, 1, 1, 1, true><<<blocks, threads, 0, s>>>(map, a, units64);
-            } else if (a.log2m == 32) {
-                plan_grid(gg_fill64x2_tma_kernel<0, 1, 1, 1, true>, units64, sm_count, blocks, threads);
-                gg_fill64x2_tma_kernel<0, 1, 1, 1, true><<<blocks, threads, 0, s>>>(map, a, units64);
-            } else {
-                plan_grid(gg_fill64x2_tma_kernel<1, 1, 1, 1, true>, units64, sm_count, blocks, threads);
-                gg_fill64x2_tma_kernel<1, 1, 1, 1, true><<<blocks, threads, 0, s>>>(map, a, units64);
-            }
-            return cudaGetLastError();
-        }
-    }
-    if (a.l == 64 && !a.pow2 && a.variant == 0 && a.m <= (1ull << 30) && a.rows &&
-        getenv("GG_FILL_NO_MOD") == nullptr) {
-        // other m <= 2^30: the R2P step with two conditional subtracts per step
-        CUtensorMap map;
-        const uint32_t units64 = (a.W + 63u) / 64u;
-        if (make_window_map(&map, a.bits, a.pitch, a.rows, 64)) {
-            if (a.out_u32) {
-                plan_grid(gg_fill64x2_tma_kernel<4, 1, 1, 1, false, true>, units64, sm_count, blocks, threads);
-                gg_fill64x2_tma_kernel<4, 1, 1, 1, false, true><<<blocks, threads, 0, s>>>(map, a, units64);
-            } else {
-                plan_grid(gg_fill64x2_tma_kernel<3, 1, 1, 1, false, true>, units64, sm_count, blocks, threads);
-                gg_fill64x2_tma_kernel<3, 1, 1, 1, false, true><<<blocks, threads, 0, s>>>(map, a, units64);
-            }
-            return cudaGetLastError();
-        }
-    }
     // composed-step table walk (the default for l = 64, m = 2^k, forward maps);
     // GG_FILL_TABLE = warps per block (2, 4, 8; default 4: 63 registers, 7 blocks
     // = 28 warps per SM, shared memory bound; C2 A/B 4.78 / 5.01 / 5.22 ms for
@@ -1590,6 +1554,42 @@ cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count) {
             else { if (orb) GG_LAUNCH_TNW(2, true); else GG_LAUNCH_TNW(2, false); }
 #undef GG_LAUNCH_TNW
 #undef GG_LAUNCH_T
+            return cudaGetLastError();
+        }
+    }
+    if (a.l == 64 && a.pow2 && a.variant == 1 && (a.l0 & 1u) == 0 && a.rows &&
+        getenv("GG_FILL_NO_BIP") == nullptr) {
+        // bipartite variant (f1): every draw starts at an even global step
+        // (l0 + 64 j), so the fixed (sigma, sigma^-1) pairing of the R2P walk holds
+        CUtensorMap map;
+        const uint32_t units64 = (a.W + 63u) / 64u;
+        if (make_window_map(&map, a.bits, a.pitch, a.rows, 64)) {
+            if (a.out_u32) {
+                plan_grid(gg_fill64x2_tma_kernel<2, 1, 1, 1, true>, units64, sm_count, blocks, threads);
+                gg_fill64x2_tma_kernel<2, 1, 1, 1, true><<<blocks, threads, 0, s>>>(map, a, units64);
+            } else if (a.log2m == 32) {
+                plan_grid(gg_fill64x2_tma_kernel<0, 1, 1, 1, true>, units64, sm_count, blocks, threads);
+                gg_fill64x2_tma_kernel<0, 1, 1, 1, true><<<blocks, threads, 0, s>>>(map, a, units64);
+            } else {
+                plan_grid(gg_fill64x2_tma_kernel<1, 1, 1, 1, true>, units64, sm_count, blocks, threads);
+                gg_fill64x2_tma_kernel<1, 1, 1, 1, true><<<blocks, threads, 0, s>>>(map, a, units64);
+            }
+            return cudaGetLastError();
+        }
+    }
+    if (a.l == 64 && !a.pow2 && a.variant == 0 && a.m <= (1ull << 30) && a.rows &&
+        getenv("GG_FILL_NO_MOD") == nullptr) {
+        // other m <= 2^30: the R2P step with two conditional subtracts per step
+        CUtensorMap map;
+        const uint32_t units64 = (a.W + 63u) / 64u;
+        if (make_window_map(&map, a.bits, a.pitch, a.rows, 64)) {
+            if (a.out_u32) {
+                plan_grid(gg_fill64x2_tma_kernel<4, 1, 1, 1, false, true>, units64, sm_count, blocks, threads);
+                gg_fill64x2_tma_kernel<4, 1, 1, 1, false, true><<<blocks, threads, 0, s>>>(map, a, units64);
+            } else {
+                plan_grid(gg_fill64x2_tma_kernel<3, 1, 1, 1, false, true>, units64, sm_count, blocks, threads);
+                gg_fill64x2_tma_kernel<3, 1, 1, 1, false, true><<<blocks, threads, 0, s>>>(map, a, units64);
+            }
             return cudaGetLastError();
         }
     }

@@ -48,7 +48,7 @@ print(json.dumps(res))
 """
 
 
-@pytest.mark.parametrize("nw", ["2", "4", "8"])
+@pytest.mark.parametrize("nw", ["2", "4", "8", "0"])  # 0: the R2P kernels (x2, bipartite pair)
 def test_table_kernel_bit_exact(nw):
     env = dict(os.environ, GG_FILL_TABLE=nw)
     p = subprocess.run([sys.executable, "-c", SNIPPET % {"root": ROOT}], env=env,
