@@ -49,6 +49,11 @@ struct FillArgs {
 };
 cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count);
 
+// Decide once per process whether the table fill kernel's shared window puts
+// its table at a 16 KB boundary (ORB layout, gg_walk.cu); called by
+// prng_create on a library stream (never inside a user's stream capture).
+void probe_fill_layout(cudaStream_t s);
+
 // The composed-step walk table (PRNG_TABLE_WORDS entries, prng_device.cuh) in
 // global memory of the current device, built on first use; nullptr on error.
 const uint32_t *walk_table(int device);

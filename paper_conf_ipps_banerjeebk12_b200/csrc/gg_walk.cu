@@ -1458,6 +1458,32 @@ static void plan_grid(K kernel, uint32_t units, int sm_count, uint32_t &blocks, 
     if (blocks == 0) blocks = 1;
 }
 
+// ORB layout state of the table fill kernel: -1 not probed, 0 plain, 1 ORB.
+static int g_orb_state = -1;
+
+void probe_fill_layout(cudaStream_t s) {
+    static std::mutex mu;
+    std::lock_guard<std::mutex> lk(mu);
+    if (g_orb_state >= 0) return;
+    g_orb_state = 0;
+    if (getenv("GG_FILL_ORB") && atoi(getenv("GG_FILL_ORB")) == 0) return;  // A/B hook
+    uint32_t *d = nullptr, hbase = 0;
+    if (cudaMalloc(&d, 4) != cudaSuccess) {
+        cudaGetLastError();
+        return;
+    }
+    CUtensorMap dummy{};
+    FillArgs a{};
+    gg_fill64t_tma_kernel<4, 0, true, false, true><<<1, 128, 0, s>>>(dummy, a, 0, d);
+    if (cudaMemcpyAsync(&hbase, d, 4, cudaMemcpyDeviceToHost, s) == cudaSuccess &&
+        cudaStreamSynchronize(s) == cudaSuccess) {
+        const uint32_t off = ((hbase + 0x3FFFu) & ~0x3FFFu) - hbase;
+        g_orb_state = (off >= FillTLayout<4>::kLead && off <= 15u * 1024u) ? 1 : 0;
+    }
+    cudaFree(d);
+    cudaGetLastError();  // a failed probe only leaves the plain layout
+}
+
 cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count) {
     if (a.jb <= a.ja || a.nl == 0) return cudaSuccess;
     const uint32_t units = (a.W + 31u) / 32u;
@@ -1495,27 +1521,9 @@ cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count) {
     // = 28 warps per SM, shared memory bound; C2 A/B 4.78 / 5.01 / 5.22 ms for
     // 4 / 8 / 2, 5.08 ms for 8 warps at 48 registers), 0 = the R2P kernels
     static const int table_nw = getenv("GG_FILL_TABLE") ? atoi(getenv("GG_FILL_TABLE")) : 4;
-    // ORB layout (table at a 16 KB boundary, FillTLayout): probed once per
-    // process; A/B hook GG_FILL_ORB=0 forces the plain layout
-    static int orb_state = -1;
-    if (orb_state < 0) {
-        orb_state = 0;
-        if (!(getenv("GG_FILL_ORB") && atoi(getenv("GG_FILL_ORB")) == 0)) {
-            uint32_t *d = nullptr, hbase = 0;
-            if (cudaMalloc(&d, 4) == cudaSuccess) {
-                CUtensorMap dummy{};
-                gg_fill64t_tma_kernel<4, 0, true, false, true><<<1, 128, 0, s>>>(dummy, a, 0, d);
-                if (cudaMemcpyAsync(&hbase, d, 4, cudaMemcpyDeviceToHost, s) == cudaSuccess &&
-                    cudaStreamSynchronize(s) == cudaSuccess) {
-                    const uint32_t off = ((hbase + 0x3FFFu) & ~0x3FFFu) - hbase;
-                    orb_state = (off >= FillTLayout<4>::kLead && off <= 15u * 1024u) ? 1 : 0;
-                }
-                cudaFree(d);
-            }
-        }
-        cudaGetLastError();  // a failed probe only disables the ORB layout
-    }
-    const bool orb = orb_state == 1;
+    // ORB layout (table at a 16 KB boundary, FillTLayout), probed by
+    // probe_fill_layout at handle creation; plain layout until then
+    const bool orb = g_orb_state == 1;
     if (a.l == 64 && a.pow2 && a.variant == 1 && (a.l0 & 1u) == 0 && table_nw > 0 && a.rows &&
         getenv("GG_FILL_NO_BIP") == nullptr) {
         // bipartite variant: the signed composed-step table (4 warps per block)

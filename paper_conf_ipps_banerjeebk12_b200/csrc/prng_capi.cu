@@ -695,6 +695,7 @@ int prng_create(prng_t **out, const prng_graph_params *g, uint64_t walkers, uint
         CK(cudaStreamCreateWithFlags(&h->copy_stream, cudaStreamNonBlocking));
         CK(cudaStreamCreateWithFlags(&h->d2h_stream, cudaStreamNonBlocking));
         CK(cudaStreamCreateWithFlags(&h->work_stream, cudaStreamNonBlocking));
+        gg::probe_fill_layout(h->work_stream);
         CK(cudaEventCreateWithFlags(&h->ev_tmp, cudaEventDisableTiming));
         static const int chunk_mb = getenv("GG_FEED_CHUNK_MB") ? atoi(getenv("GG_FEED_CHUNK_MB")) : 16;
         static const int nchunks = getenv("GG_FEED_CHUNKS") ? atoi(getenv("GG_FEED_CHUNKS")) : 4;
