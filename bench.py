@@ -261,6 +261,17 @@ def committed_traffic():
         return None
 
 
+def sass_per_label():
+    """Static SASS count per number of the fill kernel's interior draw
+    (tools/sass_hist.py -> profiles/r02_fill_table_sass.txt), or None."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "r02_fill_table_sass.txt")) as f:
+            head = f.readline()
+        return float(head.split("=")[1].split("per label")[0])
+    except (OSError, IndexError, ValueError):
+        return None
+
+
 def measured_int_peak():
     """Interleaved LOP3/IMAD lane-op rate measured by tools/int_peak.cu on this
     pool's B200 (profiles/r01_measured_box.json), T ops/s, or None."""
@@ -401,6 +412,14 @@ def run_ours(args, rank, world, local_rank):
         # 4 steps into one affine map needs fewer than 6 instructions per step)
         "frac_at_6_ops_per_step": (LABELS_PER_STEP * OPS_PER_LABEL_6 / (kern_ms / 1e3)) / peak_ops,
     }
+    spl = sass_per_label()
+    if spl:
+        # the kernel's own instruction stream against the issue peak (one warp
+        # instruction per SMSP per cycle = the same 128 lanes/clk/SM)
+        roofline["executed_sass_per_label"] = spl
+        roofline["executed_frac"] = LABELS_PER_STEP * spl / (kern_ms / 1e3) / peak_ops
+        roofline["executed_note"] = ("static SASS of the interior draw (profiles/r02_fill_table_sass.txt) "
+                                     "x labels / kernel time / peak")
     # (no oracle call here: the task reserves oracle/ for the cpu_baseline leg;
     # parity of this exact launch configuration is tests/test_gpu_generator.py's
     # full-size sampled check)
