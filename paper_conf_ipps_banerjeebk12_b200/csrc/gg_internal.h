@@ -46,6 +46,7 @@ struct FillArgs {
     uint64_t m;
     uint32_t log2m, pow2;
     uint32_t variant, l0;
+    const uint32_t *tab;  // composed-step tables (walk_table: forward, then bipartite)
 };
 cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count);
 
@@ -54,8 +55,9 @@ cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count);
 // prng_create on a library stream (never inside a user's stream capture).
 void probe_fill_layout(cudaStream_t s);
 
-// The composed-step walk table (PRNG_TABLE_WORDS entries, prng_device.cuh) in
-// global memory of the current device, built on first use; nullptr on error.
+// The composed-step walk tables in global memory of the current device, built
+// on first use: PRNG_TABLE_WORDS entries of the forward maps (prng_device.cuh),
+// then as many of the bipartite variant's; nullptr on error.
 const uint32_t *walk_table(int device);
 
 // Host feed: SplitMix64 counter-hash stream (R9), SoA rows.

@@ -814,7 +814,8 @@ __global__ void __launch_bounds__(64, 1) gg_fill64ps_tma_kernel(const __grid_con
 // patterns the coefficients are a, d <= 29, b, c <= 22, e, f <= 40 (checked by
 // enumeration in tests/test_table_formulation.py), so one 32-bit word holds
 // them (5-5-5-5-6-6 bits) and the 4096-entry table is 16 KB of shared memory,
-// built by each block at start.  Per group and walker: the 12 bits as a
+// copied by each block at start from the per-device table in global memory
+// (gg::walk_table: forward, then bipartite).  Per group and walker: the 12 bits as a
 // scaled table offset (2 ALU), one LDS, the six coefficients (balanced
 // between left shifts on the FMA pipe and right shifts on the ALU pipe), four
 // IMAD -- ~17 SASS per 4 steps instead of ~25 for four R2P steps.
@@ -864,16 +865,22 @@ __device__ __forceinline__ uint32_t gg_compose4_bip(uint32_t p) {
            ((uint32_t)d & 31u) << 15 | ((uint32_t)e & 63u) << 20 | ((uint32_t)f & 63u) << 26;
 }
 
-template <bool BIP = false>
-__device__ __forceinline__ void gg_build_table(uint32_t *tab) {
-    for (uint32_t p = threadIdx.x; p < kTabEntries; p += blockDim.x)
-        tab[p] = BIP ? gg_compose4_bip(p) : gg_compose4(p);
-    __syncthreads();
-}
 
 __global__ void gg_table_init_kernel(uint32_t *tab) {
     const uint32_t p = blockIdx.x * blockDim.x + threadIdx.x;
-    if (p < kTabEntries) tab[p] = gg_compose4(p);
+    if (p < kTabEntries) {
+        tab[p] = gg_compose4(p);                    // forward maps
+        tab[kTabEntries + p] = gg_compose4_bip(p);  // bipartite variant
+    }
+}
+
+// Copy a prebuilt table (global memory, 16 KB) into shared memory; the block
+// synchronises after.  1024 x 16-byte loads over the block.
+__device__ __forceinline__ void gg_stage_table(uint32_t *dst, const uint32_t *src) {
+    const uint4 *s4 = reinterpret_cast<const uint4 *>(src);
+    uint4 *d4 = reinterpret_cast<uint4 *>(dst);
+    for (uint32_t i = threadIdx.x; i < kTabEntries / 4; i += blockDim.x) d4[i] = __ldg(s4 + i);
+    __syncthreads();
 }
 
 // The table in global memory, once per device (prng_view::tab, staged into
@@ -885,7 +892,7 @@ const uint32_t *walk_table(int device) {
     auto it = tabs.find(device);
     if (it != tabs.end()) return it->second;
     uint32_t *t = nullptr;
-    if (cudaMalloc(&t, kTabEntries * 4) != cudaSuccess) return nullptr;
+    if (cudaMalloc(&t, 2 * kTabEntries * 4) != cudaSuccess) return nullptr;
     gg_table_init_kernel<<<kTabEntries / 256, 256>>>(t);
     if (cudaDeviceSynchronize() != cudaSuccess) {
         cudaFree(t);
@@ -953,7 +960,7 @@ __global__ void __launch_bounds__(NW * 32) gg_fill64t_tma_kernel(const __grid_co
         mbar_init(bar1, 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
-    gg_build_table<BIP>(tab);  // includes __syncthreads
+    gg_stage_table(tab, a.tab + (BIP ? kTabEntries : 0));  // includes __syncthreads
     const uint32_t tbase = raw_base + tab_off;
     const prng_tab_shifts ksh = prng_tab_shifts_load();
     uint32_t ph0 = 0, ph1 = 0;

@@ -521,6 +521,7 @@ gg::FillArgs fill_args(prng_s *h, const uint32_t *bits, uint64_t pitch, uint64_t
     a.pow2 = h->pow2;
     a.variant = h->g.variant;
     a.l0 = h->g.burnin_len;
+    a.tab = h->walk_tab;
     return a;
 }
 
