@@ -148,9 +148,6 @@ __device__ __forceinline__ void mbar_expect_tx(uint64_t *bar, uint32_t bytes) {
                  "r"(bytes)
                  : "memory");
 }
-__device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
-    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
-}
 
 __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
     asm volatile(
@@ -525,284 +522,6 @@ __global__ void __launch_bounds__(64, 1) gg_fill64p_tma_kernel(const __grid_cons
     }
 }
 
-// Two-stage form of the block-shared TMA pair kernel: the draw loop is
-// unrolled by two so both stages have fixed shared-memory addresses (as in
-// gg_fill64p_tma_kernel); after reading draw j every warp arrives on
-// empty[stage j]; thread 0 then waits for both warps' arrival on the stage of
-// draw j-1 and issues draw j+1 into it, one walk (~4 us) ahead of its use.
-template <bool V4>
-__global__ void __launch_bounds__(64, 1) gg_fill64ps2_tma_kernel(const __grid_constant__ CUtensorMap tmap,
-                                                                 FillArgs a, uint32_t units128) {
-    constexpr int kTile = 6 * 128;
-    __shared__ __align__(128) uint32_t tiles[2][kTile];
-    __shared__ __align__(8) uint64_t full[2], empty[2];
-    __shared__ uint32_t red[kFillWarps][4];
-    const uint32_t lane = threadIdx.x & 31u, wib = threadIdx.x >> 5;
-    if (threadIdx.x == 0) {
-        for (int q = 0; q < 2; q++) {
-            mbar_init(&full[q], 1);
-            mbar_init(&empty[q], kFillWarps);
-        }
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    }
-    __syncthreads();
-    const uint32_t kBytes = kTile * 4;
-    uint32_t fph0 = 0, fph1 = 0, eph0 = 0, eph1 = 0;
-    for (uint32_t u = blockIdx.x; u < units128; u += gridDim.x) {
-        const uint32_t ta = u * 128u + wib * 64u + 2u * lane, tb = ta + 1u;
-        uint32_t ja0 = 0xFFFFFFFFu, ja1 = 0, jb0 = 0xFFFFFFFFu, jb1 = 0;
-        if (ta < a.W) {
-            walker_draw_range(a.N, a.nl, a.W, ta, ja0, ja1);
-            ja0 = max(ja0, a.ja);
-            ja1 = min(ja1, a.jb);
-        }
-        if (tb < a.W) {
-            walker_draw_range(a.N, a.nl, a.W, tb, jb0, jb1);
-            jb0 = max(jb0, a.ja);
-            jb1 = min(jb1, a.jb);
-        }
-        {
-            const uint32_t v0 = __reduce_min_sync(0xFFFFFFFFu, min(ja0, jb0));
-            const uint32_t v1 = __reduce_max_sync(0xFFFFFFFFu, max(ja1, jb1));
-            const uint32_t v2 = __reduce_max_sync(0xFFFFFFFFu, max(ja0, jb0));
-            const uint32_t v3 = __reduce_min_sync(0xFFFFFFFFu, min(ja1, jb1));
-            if (lane == 0) {
-                red[wib][0] = v0;
-                red[wib][1] = v1;
-                red[wib][2] = v2;
-                red[wib][3] = v3;
-            }
-        }
-        __syncthreads();
-        const uint32_t jlo = min(red[0][0], red[1][0]), jhi = max(red[0][1], red[1][1]);
-        const uint32_t jin0 = max(red[0][2], red[1][2]), jin1 = min(red[0][3], red[1][3]);
-        __syncthreads();
-        if (jlo >= jhi) continue;  // block-uniform
-        uint32_t xa = 0, ya = 0, xb = 0, yb = 0;
-        if (tb < a.W) {
-            const uint2 px = *reinterpret_cast<const uint2 *>(a.x + ta);
-            const uint2 py = *reinterpret_cast<const uint2 *>(a.y + ta);
-            xa = px.x, xb = px.y, ya = py.x, yb = py.y;
-        } else if (ta < a.W) {
-            xa = a.x[ta];
-            ya = a.y[ta];
-        }
-        if (threadIdx.x == 0) {
-            mbar_expect_tx(&full[0], kBytes);
-            tma_load_tile(tiles[0], &tmap, &full[0], (int32_t)(u * 128u), (int32_t)((jlo - a.Jw) * 6u));
-        }
-        // draw j from stage S (0: j - jlo even), then refill stage 1-S with j+1
-        auto draw = [&](auto stage, uint32_t j) {
-            constexpr int S = decltype(stage)::value;
-            mbar_wait(&full[S], S ? fph1 : fph0);
-            if (S) fph1 ^= 1u; else fph0 ^= 1u;
-            uint32_t wa[6], wb[6];
-#pragma unroll
-            for (int r = 0; r < 6; r++) {
-                const uint2 v = *reinterpret_cast<const uint2 *>(tiles[S] + r * 128 + wib * 64 + 2 * lane);
-                wa[r] = v.x;
-                wb[r] = v.y;
-            }
-            __syncwarp();
-            if (lane == 0) mbar_arrive(&empty[S]);
-            if (threadIdx.x == 0 && j + 1 < jhi) {
-                if (j > jlo) {  // both warps have read draw j-1 from stage 1-S
-                    mbar_wait(&empty[1 - S], S ? eph0 : eph1);
-                    if (S) eph0 ^= 1u; else eph1 ^= 1u;
-                }
-                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-                mbar_expect_tx(&full[1 - S], kBytes);
-                tma_load_tile(tiles[1 - S], &tmap, &full[1 - S], (int32_t)(u * 128u),
-                              (int32_t)((j + 1 - a.Jw) * 6u));
-            }
-            if (j >= jin0 && j < jin1) {  // block-uniform: all 128 walkers active
-                gg_walk64x2_r2p(wa, wb, xa, ya, xb, yb);
-                const uint64_t idx = (uint64_t)j * a.W + ta - a.g_origin;
-                if (V4) {
-                    *reinterpret_cast<uint4 *>(reinterpret_cast<uint2 *>(a.out) + idx) =
-                        make_uint4(xa, ya, xb, yb);
-                } else {
-                    reinterpret_cast<uint2 *>(a.out)[idx] = make_uint2(xa, ya);
-                    reinterpret_cast<uint2 *>(a.out)[idx + 1] = make_uint2(xb, yb);
-                }
-            } else {
-                uint32_t nxa = xa, nya = ya, nxb = xb, nyb = yb;
-                gg_walk64x2_r2p(wa, wb, nxa, nya, nxb, nyb);
-                if (j >= ja0 && j < ja1) {
-                    xa = nxa;
-                    ya = nya;
-                    emit_label<0>(a, (uint64_t)j * a.W + ta - a.g_origin, xa, ya);
-                }
-                if (j >= jb0 && j < jb1) {
-                    xb = nxb;
-                    yb = nyb;
-                    emit_label<0>(a, (uint64_t)j * a.W + tb - a.g_origin, xb, yb);
-                }
-            }
-        };
-        for (uint32_t j = jlo; j < jhi; j += 2) {
-            draw(std::integral_constant<int, 0>(), j);
-            if (j + 1 < jhi) draw(std::integral_constant<int, 1>(), j + 1);
-        }
-        // the producer's empty-phase bookkeeping must see every consumption:
-        // the unit's last two draws were read but never waited for
-        if (threadIdx.x == 0) {
-            for (uint32_t d = (jhi - jlo >= 2 ? jhi - 2 : jlo); d < jhi; d++) {
-                const uint32_t sd = (d - jlo) & 1u;
-                mbar_wait(&empty[sd], sd ? eph1 : eph0);
-                if (sd) eph1 ^= 1u; else eph0 ^= 1u;
-            }
-        }
-        __syncthreads();  // stages free before the next unit's prologue
-        if (tb < a.W) {
-            *reinterpret_cast<uint2 *>(a.x + ta) = make_uint2(xa, xb);
-            *reinterpret_cast<uint2 *>(a.y + ta) = make_uint2(ya, yb);
-        } else if (ta < a.W) {
-            a.x[ta] = xa;
-            a.y[ta] = ya;
-        }
-    }
-}
-
-// Pair variant with ONE TMA per draw for the whole block (2 warps, 128
-// walkers, box 128 x 6 words) into a 3-stage ring: full barriers complete on
-// the copy's bytes, empty barriers on one arrival per warp; thread 0 is the
-// producer and refills the stage of draw j-1 with draw j+2 once both warps
-// have read it (lagging one draw so the warps are not held in lockstep).
-// The elected-copy overhead (~23 issue slots) is paid once per block per
-// draw instead of once per warp.  Stage and barrier phase of the block's
-// g-th draw (counted over its lifetime) are g % 3 and (g / 3) & 1, kept
-// incrementally.
-constexpr int kPsStages = 3;
-
-template <bool V4>
-__global__ void __launch_bounds__(64, 1) gg_fill64ps_tma_kernel(const __grid_constant__ CUtensorMap tmap,
-                                                                FillArgs a, uint32_t units128) {
-    constexpr int kTile = 6 * 128;
-    __shared__ __align__(128) uint32_t tiles[kPsStages][kTile];
-    __shared__ __align__(8) uint64_t full[kPsStages], empty[kPsStages];
-    __shared__ uint32_t red[kFillWarps][4];
-    const uint32_t lane = threadIdx.x & 31u, wib = threadIdx.x >> 5;
-    if (threadIdx.x == 0) {
-        for (int q = 0; q < kPsStages; q++) {
-            mbar_init(&full[q], 1);
-            mbar_init(&empty[q], kFillWarps);
-        }
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    }
-    __syncthreads();
-    const uint32_t kBytes = kTile * 4;
-    // stage / phase of the block's next draw, advanced incrementally
-    // (st cycles 0, 1, 2; ph flips when st wraps)
-    uint32_t st = 0, ph = 0;
-    for (uint32_t u = blockIdx.x; u < units128; u += gridDim.x) {
-        const uint32_t ta = u * 128u + wib * 64u + 2u * lane, tb = ta + 1u;
-        uint32_t ja0 = 0xFFFFFFFFu, ja1 = 0, jb0 = 0xFFFFFFFFu, jb1 = 0;
-        if (ta < a.W) {
-            walker_draw_range(a.N, a.nl, a.W, ta, ja0, ja1);
-            ja0 = max(ja0, a.ja);
-            ja1 = min(ja1, a.jb);
-        }
-        if (tb < a.W) {
-            walker_draw_range(a.N, a.nl, a.W, tb, jb0, jb1);
-            jb0 = max(jb0, a.ja);
-            jb1 = min(jb1, a.jb);
-        }
-        {
-            const uint32_t v0 = __reduce_min_sync(0xFFFFFFFFu, min(ja0, jb0));
-            const uint32_t v1 = __reduce_max_sync(0xFFFFFFFFu, max(ja1, jb1));
-            const uint32_t v2 = __reduce_max_sync(0xFFFFFFFFu, max(ja0, jb0));
-            const uint32_t v3 = __reduce_min_sync(0xFFFFFFFFu, min(ja1, jb1));
-            if (lane == 0) {
-                red[wib][0] = v0;
-                red[wib][1] = v1;
-                red[wib][2] = v2;
-                red[wib][3] = v3;
-            }
-        }
-        __syncthreads();
-        const uint32_t jlo = min(red[0][0], red[1][0]), jhi = max(red[0][1], red[1][1]);
-        const uint32_t jin0 = max(red[0][2], red[1][2]), jin1 = min(red[0][3], red[1][3]);
-        __syncthreads();  // red is rewritten by the next unit
-        if (jlo >= jhi) continue;  // block-uniform
-        uint32_t xa = 0, ya = 0, xb = 0, yb = 0;
-        if (tb < a.W) {
-            const uint2 px = *reinterpret_cast<const uint2 *>(a.x + ta);
-            const uint2 py = *reinterpret_cast<const uint2 *>(a.y + ta);
-            xa = px.x, xb = px.y, ya = py.x, yb = py.y;
-        } else if (ta < a.W) {
-            xa = a.x[ta];
-            ya = a.y[ta];
-        }
-        if (threadIdx.x == 0) {
-            for (uint32_t q = 0, sq = st; q < kPsStages && jlo + q < jhi; q++) {
-                mbar_expect_tx(&full[sq], kBytes);
-                tma_load_tile(tiles[sq], &tmap, &full[sq], (int32_t)(u * 128u),
-                              (int32_t)((jlo + q - a.Jw) * 6u));
-                sq = sq == kPsStages - 1 ? 0 : sq + 1;
-            }
-        }
-        uint32_t sp = 0, pp = 0;  // stage / phase of the previous draw
-        for (uint32_t j = jlo; j < jhi; j++) {
-            mbar_wait(&full[st], ph);
-            uint32_t wa[6], wb[6];
-#pragma unroll
-            for (int r = 0; r < 6; r++) {
-                const uint2 v = *reinterpret_cast<const uint2 *>(tiles[st] + r * 128 + wib * 64 + 2 * lane);
-                wa[r] = v.x;
-                wb[r] = v.y;
-            }
-            __syncwarp();
-            if (lane == 0) mbar_arrive(&empty[st]);
-            if (threadIdx.x == 0 && j > jlo && j + 2 < jhi) {
-                // refill the stage of draw j-1 with draw j+2 once both warps read it
-                mbar_wait(&empty[sp], pp);
-                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-                mbar_expect_tx(&full[sp], kBytes);
-                tma_load_tile(tiles[sp], &tmap, &full[sp], (int32_t)(u * 128u),
-                              (int32_t)((j + 2 - a.Jw) * 6u));
-            }
-            sp = st;
-            pp = ph;
-            if (++st == kPsStages) {
-                st = 0;
-                ph ^= 1u;
-            }
-            if (j >= jin0 && j < jin1) {  // block-uniform: all 128 walkers active
-                gg_walk64x2_r2p(wa, wb, xa, ya, xb, yb);
-                const uint64_t idx = (uint64_t)j * a.W + ta - a.g_origin;
-                if (V4) {
-                    *reinterpret_cast<uint4 *>(reinterpret_cast<uint2 *>(a.out) + idx) =
-                        make_uint4(xa, ya, xb, yb);
-                } else {
-                    reinterpret_cast<uint2 *>(a.out)[idx] = make_uint2(xa, ya);
-                    reinterpret_cast<uint2 *>(a.out)[idx + 1] = make_uint2(xb, yb);
-                }
-            } else {
-                uint32_t nxa = xa, nya = ya, nxb = xb, nyb = yb;
-                gg_walk64x2_r2p(wa, wb, nxa, nya, nxb, nyb);
-                if (j >= ja0 && j < ja1) {
-                    xa = nxa;
-                    ya = nya;
-                    emit_label<0>(a, (uint64_t)j * a.W + ta - a.g_origin, xa, ya);
-                }
-                if (j >= jb0 && j < jb1) {
-                    xb = nxb;
-                    yb = nyb;
-                    emit_label<0>(a, (uint64_t)j * a.W + tb - a.g_origin, xb, yb);
-                }
-            }
-        }
-        if (tb < a.W) {
-            *reinterpret_cast<uint2 *>(a.x + ta) = make_uint2(xa, xb);
-            *reinterpret_cast<uint2 *>(a.y + ta) = make_uint2(ya, yb);
-        } else if (ta < a.W) {
-            a.x[ta] = xa;
-            a.y[ta] = ya;
-        }
-    }
-}
-
 // ---------------------------------------------------------------------------
 // Composed-step ("table") walk, l = 64, m = 2^k, forward maps.  The 64 steps
 // of a draw are 16 groups of 4 steps; a group reads 12 consecutive record
@@ -1064,118 +783,6 @@ __global__ void __launch_bounds__(NW * 32) gg_fill64t_tma_kernel(const __grid_co
                 }
             }
         }
-        if (tb < a.W) {
-            *reinterpret_cast<uint2 *>(a.x + ta) = make_uint2(xa, xb);
-            *reinterpret_cast<uint2 *>(a.y + ta) = make_uint2(ya, yb);
-        } else if (ta < a.W) {
-            a.x[ta] = xa;
-            a.y[ta] = ya;
-        }
-    }
-}
-
-// Pair variant with per-lane cp.async staging instead of TMA: each lane
-// copies its own 8-byte slice of the 6 record rows (its two adjacent
-// walkers) into a lane-private column of a 3-stage shared-memory ring
-// (layout [stage][row][lane], conflict-free), so there is no cross-lane
-// hazard: no mbarrier, no __syncwarp, no elected issuer.  Per draw: 6
-// LDGSTS.64 + commit + wait + 6 LDS.64 (the TMA path spends ~23 issue slots
-// per draw on the elected copy alone).
-constexpr int kPcStages = 3;
-
-__device__ __forceinline__ void cp_async8(void *smem, const void *gmem, uint32_t src_bytes) {
-    asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;" ::"r"(smem_u32(smem)), "l"(gmem),
-                 "r"(src_bytes)
-                 : "memory");
-}
-
-template <bool V4>
-__global__ void __launch_bounds__(64, 1) gg_fill64pc_kernel(FillArgs a, uint32_t units64) {
-    __shared__ __align__(16) uint2 ring[kFillWarps][kPcStages][6][32];
-    const uint32_t lane = threadIdx.x & 31u, wib = threadIdx.x >> 5;
-    const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
-    const uint64_t rstride = a.pitch;  // words between rows
-    for (uint32_t u = warp; u < units64; u += nwarps) {
-        const uint32_t ta = u * 64u + 2u * lane, tb = ta + 1u;
-        uint32_t ja0 = 0xFFFFFFFFu, ja1 = 0, jb0 = 0xFFFFFFFFu, jb1 = 0;
-        if (ta < a.W) {
-            walker_draw_range(a.N, a.nl, a.W, ta, ja0, ja1);
-            ja0 = max(ja0, a.ja);
-            ja1 = min(ja1, a.jb);
-        }
-        if (tb < a.W) {
-            walker_draw_range(a.N, a.nl, a.W, tb, jb0, jb1);
-            jb0 = max(jb0, a.ja);
-            jb1 = min(jb1, a.jb);
-        }
-        const uint32_t jlo = __reduce_min_sync(0xFFFFFFFFu, min(ja0, jb0));
-        const uint32_t jhi = __reduce_max_sync(0xFFFFFFFFu, max(ja1, jb1));
-        if (jlo >= jhi) continue;
-        const uint32_t jin0 = __reduce_max_sync(0xFFFFFFFFu, max(ja0, jb0));
-        const uint32_t jin1 = __reduce_min_sync(0xFFFFFFFFu, min(ja1, jb1));
-        uint32_t xa = 0, ya = 0, xb = 0, yb = 0;
-        if (tb < a.W) {
-            const uint2 px = *reinterpret_cast<const uint2 *>(a.x + ta);
-            const uint2 py = *reinterpret_cast<const uint2 *>(a.y + ta);
-            xa = px.x, xb = px.y, ya = py.x, yb = py.y;
-        } else if (ta < a.W) {
-            xa = a.x[ta];
-            ya = a.y[ta];
-        }
-        // bytes of this lane's 8-byte slice that exist (the window's pitch is
-        // a multiple of 32 walkers, so the slice never straddles its end)
-        const uint32_t src_bytes = ta < a.W ? 8u : 0u;
-        const uint32_t *col = a.bits + ta;
-        auto issue = [&](uint32_t j, int stage) {
-            if (j < jhi) {
-                const uint32_t *rec = col + (uint64_t)(j - a.Jw) * 6u * rstride;
-#pragma unroll
-                for (int r = 0; r < 6; r++)
-                    cp_async8(&ring[wib][stage][r][lane], rec + r * rstride, src_bytes);
-            }
-            asm volatile("cp.async.commit_group;" ::: "memory");
-        };
-        issue(jlo, 0);
-        issue(jlo + 1, 1);
-        uint32_t stage = 0;
-        for (uint32_t j = jlo; j < jhi; j++) {
-            issue(j + 2, stage == 0 ? 2 : stage - 1);  // the stage read two draws ago
-            asm volatile("cp.async.wait_group 2;" ::: "memory");
-            uint32_t wa[6], wb[6];
-#pragma unroll
-            for (int r = 0; r < 6; r++) {
-                const uint2 v = ring[wib][stage][r][lane];
-                wa[r] = v.x;
-                wb[r] = v.y;
-            }
-            stage = stage == 2 ? 0 : stage + 1;
-            if (j >= jin0 && j < jin1) {  // warp-uniform: all 64 walkers active
-                gg_walk64x2_r2p(wa, wb, xa, ya, xb, yb);
-                const uint64_t idx = (uint64_t)j * a.W + ta - a.g_origin;
-                if (V4) {
-                    *reinterpret_cast<uint4 *>(reinterpret_cast<uint2 *>(a.out) + idx) =
-                        make_uint4(xa, ya, xb, yb);
-                } else {
-                    reinterpret_cast<uint2 *>(a.out)[idx] = make_uint2(xa, ya);
-                    reinterpret_cast<uint2 *>(a.out)[idx + 1] = make_uint2(xb, yb);
-                }
-            } else {
-                uint32_t nxa = xa, nya = ya, nxb = xb, nyb = yb;
-                gg_walk64x2_r2p(wa, wb, nxa, nya, nxb, nyb);
-                if (j >= ja0 && j < ja1) {
-                    xa = nxa;
-                    ya = nya;
-                    emit_label<0>(a, (uint64_t)j * a.W + ta - a.g_origin, xa, ya);
-                }
-                if (j >= jb0 && j < jb1) {
-                    xb = nxb;
-                    yb = nyb;
-                    emit_label<0>(a, (uint64_t)j * a.W + tb - a.g_origin, xb, yb);
-                }
-            }
-        }
-        asm volatile("cp.async.wait_group 0;" ::: "memory");
         if (tb < a.W) {
             *reinterpret_cast<uint2 *>(a.x + ta) = make_uint2(xa, xb);
             *reinterpret_cast<uint2 *>(a.y + ta) = make_uint2(ya, yb);
@@ -1627,44 +1234,6 @@ cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count) {
                 static const bool r2p = !(getenv("GG_FILL_STEP") && atoi(getenv("GG_FILL_STEP")) == 0);
                 static const bool u2 = !(getenv("GG_FILL_U2") && atoi(getenv("GG_FILL_U2")) == 0);
                 static const bool pair = getenv("GG_FILL_PAIR") && atoi(getenv("GG_FILL_PAIR")) == 1;
-                static const bool pair_cp = getenv("GG_FILL_PAIR") && atoi(getenv("GG_FILL_PAIR")) == 2;
-                static const bool pair_sh = getenv("GG_FILL_PAIR") && atoi(getenv("GG_FILL_PAIR")) == 3;
-                static const bool pair_sh2 = getenv("GG_FILL_PAIR") && atoi(getenv("GG_FILL_PAIR")) == 4;
-                CUtensorMap map128;
-                if (pair_sh2 && r2p && minb == 1 && u2 &&
-                    make_window_map(&map128, a.bits, a.pitch, a.rows, 128)) {
-                    const bool v4 = (a.W % 2 == 0) && (a.g_origin % 2 == 0) &&
-                                    ((uintptr_t)a.out % 16 == 0);
-                    const uint32_t units128 = (a.W + 127u) / 128u;
-                    if (v4)
-                        gg_fill64ps2_tma_kernel<true><<<units128, 64, 0, s>>>(map128, a, units128);
-                    else
-                        gg_fill64ps2_tma_kernel<false><<<units128, 64, 0, s>>>(map128, a, units128);
-                    return cudaGetLastError();
-                }
-                if (pair_sh && r2p && minb == 1 && u2 &&
-                    make_window_map(&map128, a.bits, a.pitch, a.rows, 128)) {
-                    const bool v4 = (a.W % 2 == 0) && (a.g_origin % 2 == 0) &&
-                                    ((uintptr_t)a.out % 16 == 0);
-                    const uint32_t units128 = (a.W + 127u) / 128u;
-                    if (v4)
-                        gg_fill64ps_tma_kernel<true><<<units128, 64, 0, s>>>(map128, a, units128);
-                    else
-                        gg_fill64ps_tma_kernel<false><<<units128, 64, 0, s>>>(map128, a, units128);
-                    return cudaGetLastError();
-                }
-                if (pair_cp && r2p && minb == 1 && u2) {
-                    const bool v4 = (a.W % 2 == 0) && (a.g_origin % 2 == 0) &&
-                                    ((uintptr_t)a.out % 16 == 0);
-                    if (v4) {
-                        plan_grid(gg_fill64pc_kernel<true>, units64, sm_count, blocks, threads);
-                        gg_fill64pc_kernel<true><<<blocks, threads, 0, s>>>(a, units64);
-                    } else {
-                        plan_grid(gg_fill64pc_kernel<false>, units64, sm_count, blocks, threads);
-                        gg_fill64pc_kernel<false><<<blocks, threads, 0, s>>>(a, units64);
-                    }
-                    return cudaGetLastError();
-                }
                 if (pair && r2p && minb == 1 && u2) {
                     // adjacent-walker lanes (LDS.64, 16-B stores when the output index parity allows)
                     const bool v4 = (a.W % 2 == 0) && (a.g_origin % 2 == 0) &&

@@ -2,7 +2,8 @@
 
     compute-sanitizer --tool memcheck|racecheck|synccheck python tools/sanitize_cases.py
 Covers: init, bulk fill (x2 TMA u64/u32, x1 TMA, LDG, generic m, bipartite,
-l = 1 TMA; the GG_FILL_PAIR variants when run under that hook), on-demand
+l = 1 TMA; the composed-step table kernel and, under the hooks, the R2P and
+pair kernels), on-demand
 consume in every walk mode, list ranking (Phase I-III, the compaction
 kernel over several tiles), Monte Carlo epoch.
 Sizes are tiny (the sanitizer slows kernels by orders of magnitude) but
