@@ -21,16 +21,24 @@ __global__ void __launch_bounds__(128) consume_kernel(const __grid_constant__ pr
                                                       const uint32_t *counts, uint32_t uniform,
                                                       uint64_t *out, const uint64_t *offsets,
                                                       uint64_t *xor_out) {
-    // the paper's generator (PRNG_WALK_L64): composed-step table in shared memory
-    constexpr bool TAB = MODE == PRNG_WALK_L64;
-    __shared__ __align__(PRNG_TABLE_ALIGN) uint32_t tab[TAB ? PRNG_TABLE_WORDS : 4];
-    if (TAB) {
-        prng_table_stage(&v, tab);
-        __syncthreads();
-    }
+    // the paper's generator (PRNG_WALK_L64): composed-step table in shared
+    // memory -- staged only by blocks where some thread makes >= kTabMin
+    // draws (16 KB of staging for a block of one-draw threads costs more
+    // than it saves: the list-ranking-shaped consumers)
+    constexpr bool TAB_MODE = MODE == PRNG_WALK_L64;
+    constexpr uint32_t kTabMin = 4;
+    __shared__ __align__(PRNG_TABLE_ALIGN) uint32_t tab[TAB_MODE ? PRNG_TABLE_WORDS : 4];
     const uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const uint32_t c = t < threads ? (counts ? counts[t] : uniform) : 0u;
+    bool TAB = false;
+    if (TAB_MODE) {
+        TAB = __syncthreads_or(c >= kTabMin) != 0;  // block-uniform
+        if (TAB) {
+            prng_table_stage(&v, tab);
+            __syncthreads();
+        }
+    }
     if (t >= threads) return;
-    const uint32_t c = counts ? counts[t] : uniform;
     if (c == 0) {  // idle this launch: the walker's state is untouched
         if (xor_out) xor_out[t] = 0;
         return;
