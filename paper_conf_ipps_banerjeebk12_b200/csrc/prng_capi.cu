@@ -5,7 +5,6 @@
 #include <algorithm>
 #include <cctype>
 #include <sched.h>
-#include <sys/mman.h>
 #include <pthread.h>
 #include <chrono>
 #include <condition_variable>
@@ -239,7 +238,6 @@ struct prng_s {
     int kChunks = 4;
     uint32_t *chunk[kMaxChunks] = {};
     size_t chunk_bytes = 0;
-    bool chunk_mmapped = false;  // GG_FEED_HUGE chunks (mmap + cudaHostRegister)
     cudaEvent_t chunk_done[kMaxChunks] = {};
     int chunk_next = 0;
 
@@ -298,12 +296,7 @@ void free_all(prng_s *h) {
     for (auto p : h->hout)
         if (p) cudaFree(p);
     for (int i = 0; i < h->kChunks; i++) {
-        if (h->chunk[i] && h->chunk_mmapped) {
-            cudaHostUnregister(h->chunk[i]);
-            munmap(h->chunk[i], h->chunk_bytes);
-        } else if (h->chunk[i]) {
-            cudaFreeHost(h->chunk[i]);
-        }
+        if (h->chunk[i]) cudaFreeHost(h->chunk[i]);
         if (h->chunk_done[i]) cudaEventDestroy(h->chunk_done[i]);
     }
     for (int i = 0; i < 2; i++) {
@@ -709,22 +702,8 @@ int prng_create(prng_t **out, const prng_graph_params *g, uint64_t walkers, uint
         static const int nchunks = getenv("GG_FEED_CHUNKS") ? atoi(getenv("GG_FEED_CHUNKS")) : 4;
         h->chunk_bytes = (size_t)(chunk_mb > 0 ? chunk_mb : 32) << 20;
         h->kChunks = std::min(prng_s::kMaxChunks, std::max(2, nchunks));
-        // A/B hook GG_FEED_HUGE=1: chunks in 2 MB transparent huge pages,
-        // registered with CUDA (fewer IOMMU/IOTLB translations for the DMA)
-        static const bool huge = getenv("GG_FEED_HUGE") && atoi(getenv("GG_FEED_HUGE")) == 1;
         for (int i = 0; i < h->kChunks; i++) {
-            if (huge) {
-                void *p = mmap(nullptr, h->chunk_bytes, PROT_READ | PROT_WRITE,
-                               MAP_PRIVATE | MAP_ANONYMOUS, -1, 0);
-                if (p == MAP_FAILED) throw std::bad_alloc();
-                madvise(p, h->chunk_bytes, MADV_HUGEPAGE);
-                memset(p, 0, h->chunk_bytes);
-                CK(cudaHostRegister(p, h->chunk_bytes, cudaHostRegisterPortable));
-                h->chunk[i] = (uint32_t *)p;
-                h->chunk_mmapped = true;
-            } else {
-                CK(cudaHostAlloc((void **)&h->chunk[i], h->chunk_bytes, cudaHostAllocPortable));
-            }
+            CK(cudaHostAlloc((void **)&h->chunk[i], h->chunk_bytes, cudaHostAllocPortable));
             CK(cudaEventCreateWithFlags(&h->chunk_done[i], cudaEventDisableTiming));
         }
         for (int i = 0; i < 2; i++) {
