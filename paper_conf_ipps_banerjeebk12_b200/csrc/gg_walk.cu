@@ -1043,6 +1043,58 @@ __global__ void __launch_bounds__(64) gg_fill_any_kernel(FillArgs a, uint32_t un
     }
 }
 
+// Any walk length with the composed-step table (l != 64, m = 2^k, forward
+// maps): the record's 12-bit groups are funnel-shifted out of a rolling pair
+// of words (each word loaded once); the last group of a walk whose l is not a
+// multiple of 4 masks its unused fields to 0 (sigma_0, stay), so the 4-step
+// table also covers 1..3 trailing steps.  4 warps per block share the table.
+constexpr int kAnyTW = 4;
+__global__ void __launch_bounds__(kAnyTW * 32) gg_fill_anyt_kernel(FillArgs a, uint32_t units) {
+    __shared__ __align__(16) uint32_t tab[kTabEntries];
+    gg_stage_table(tab, a.tab);
+    const uint32_t tbase = (uint32_t)__cvta_generic_to_shared(tab);
+    const prng_tab_shifts ksh = prng_tab_shifts_load();
+    const uint32_t lane = threadIdx.x & 31u;
+    const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+    const uint32_t ngroups = (a.l + 3u) / 4u;
+    const uint32_t tail = a.l - 4u * (ngroups - 1u);                 // steps in the last group
+    const uint32_t tail_mask = tail >= 4u ? 0xFFFu : ((1u << (3u * tail)) - 1u);
+    for (uint32_t u = warp; u < units; u += nwarps) {
+        const uint32_t t = u * 32u + lane;
+        if (t >= a.W) break;
+        uint32_t j0, j1;
+        walker_draw_range(a.N, a.nl, a.W, t, j0, j1);
+        j0 = max(j0, a.ja);
+        j1 = min(j1, a.jb);
+        if (j0 >= j1) continue;
+        uint32_t x = a.x[t], y = a.y[t];
+        for (uint32_t j = j0; j < j1; j++) {
+            const uint32_t *rec = a.bits + t + (uint64_t)(j - a.Jw) * a.R * a.pitch;
+            uint32_t lo = __ldg(rec), hi = a.R > 1 ? __ldg(rec + a.pitch) : 0u, wi = 0;
+            for (uint32_t g = 0; g < ngroups; g++) {
+                const uint32_t bit = 12u * g, i = bit >> 5, sh = bit & 31u;
+                if (i != wi) {  // 12-bit groups advance at most one word
+                    lo = hi;
+                    wi = i;
+                    hi = wi + 1 < a.R ? __ldg(rec + (uint64_t)(wi + 1) * a.pitch) : 0u;
+                }
+                uint32_t idx = __funnelshift_r(lo, hi, sh);
+                idx &= (g + 1 == ngroups) ? tail_mask : 0xFFFu;
+                prng_group_apply<false>(tbase + 4u * idx, x, y, ksh);
+            }
+            const uint64_t lab = gg_label(x, y, a.m, a.log2m, true);
+            const uint64_t gi = (uint64_t)j * a.W + t;
+            if (a.out_u32)
+                reinterpret_cast<uint32_t *>(a.out)[gi - a.g_origin] = (uint32_t)lab;
+            else
+                reinterpret_cast<uint64_t *>(a.out)[gi - a.g_origin] = lab;
+        }
+        a.x[t] = x;
+        a.y[t] = y;
+    }
+}
+
 // Grid of 64-thread blocks (2 warps each); `units` = work items a warp takes
 // round-robin (32 walkers; 64 for the x2 kernels).  One item per warp: the
 // block scheduler starts a new block wherever one finishes, so SMs stay busy to
@@ -1286,8 +1338,13 @@ cudaError_t launch_fill(const FillArgs &a, cudaStream_t s, int sm_count) {
             gg_fill64_kernel<0><<<blocks, threads, 0, s>>>(a, units);
         }
     } else if (a.pow2 && a.variant == 0 && a.l >= 2 && getenv("GG_FILL_NO_ANY") == nullptr) {
-        plan_grid(gg_fill_any_kernel, units, sm_count, blocks, threads);
-        gg_fill_any_kernel<<<blocks, threads, 0, s>>>(a, units);
+        if (table_nw > 0) {
+            // composed-step table; GG_FILL_TABLE=0: the R2P any-l kernel
+            gg_fill_anyt_kernel<<<(units + kAnyTW - 1) / kAnyTW, kAnyTW * 32, 0, s>>>(a, units);
+        } else {
+            plan_grid(gg_fill_any_kernel, units, sm_count, blocks, threads);
+            gg_fill_any_kernel<<<blocks, threads, 0, s>>>(a, units);
+        }
     } else {
         plan_grid(gg_fill_generic_kernel, units, sm_count, blocks, threads);
         gg_fill_generic_kernel<<<blocks, threads, 0, s>>>(a, units);

@@ -2,7 +2,8 @@
 csrc/gg_walk.cu gg_fill64t_tma_kernel) is bit-exact with the oracle for every
 m = 2^k output form it serves (u64 labels of m = 2^32 with and without the
 16-byte store path, u64 labels of m = 2^k < 2^32, u32 words of m <= 2^16) and
-for the bipartite variant's signed table, on
+for the bipartite variant's signed table, and the any-l table kernel (l = 16,
+13, 2, 101: whole and partial 4-step groups), on
 ragged walker counts and fills that stop mid-draw.  The hook is read once per
 process, so each configuration runs in a subprocess."""
 import json
@@ -24,10 +25,13 @@ import numpy as np, torch
 sys.path.insert(0, %(root)r)
 from paper_conf_ipps_banerjeebk12_b200 import Generator
 res = {}
-for m, W, fmt, var in ((1 << 32, 1000, "u64", 0), (1 << 32, 999, "u64", 0), (1 << 32, 4096, "u32", 0),
-                       (256, 1000, "u64", 0), (1 << 20, 777, "u64", 0), (1 << 16, 640, "u32", 0),
-                       (1 << 32, 1000, "u64", 1), (1 << 12, 333, "u64", 1)):
-    g = Generator(walkers=W, seed=0x7AB1E + W, m=m, epoch_draws=5, variant=var)
+for m, W, fmt, var, l in ((1 << 32, 1000, "u64", 0, 64), (1 << 32, 999, "u64", 0, 64),
+                          (1 << 32, 4096, "u32", 0, 64), (256, 1000, "u64", 0, 64),
+                          (1 << 20, 777, "u64", 0, 64), (1 << 16, 640, "u32", 0, 64),
+                          (1 << 32, 1000, "u64", 1, 64), (1 << 12, 333, "u64", 1, 64),
+                          (1 << 32, 1000, "u64", 0, 16), (1 << 32, 700, "u64", 0, 13),
+                          (1 << 20, 500, "u64", 0, 2), (1 << 32, 300, "u64", 0, 101)):
+    g = Generator(walkers=W, seed=0x7AB1E + W, m=m, epoch_draws=5, variant=var, walk_len=l)
     outs = []
     for n in (7, 3 * W + 5, 2 * W + 2, 9 * W):
         if fmt == "u64":
@@ -43,7 +47,7 @@ for m, W, fmt, var in ((1 << 32, 1000, "u64", 0), (1 << 32, 999, "u64", 0), (1 <
     o = torch.empty(12 * W, dtype=torch.int64, device="cuda")
     g.fill(o)
     outs.append(o.cpu().numpy().view(np.uint64))
-    res[f"{m}-{W}-{fmt}-{var}"] = [int(v) for v in np.concatenate(outs)]
+    res[f"{m}-{W}-{fmt}-{var}-{l}"] = [int(v) for v in np.concatenate(outs)]
 print(json.dumps(res))
 """
 
@@ -56,10 +60,10 @@ def test_table_kernel_bit_exact(nw):
     assert p.returncode == 0, p.stderr[-2000:]
     got = json.loads(p.stdout.strip().splitlines()[-1])
     for key, vals in got.items():
-        m, W, fmt, var = key.split("-")
-        m, W, var = int(m), int(W), int(var)
+        m, W, fmt, var, l = key.split("-")
+        m, W, var, l = int(m), int(W), int(var), int(l)
         total = 7 + (3 * W + 5) + (2 * W + 2) + 9 * W
         n_pref = 12 * W
         # fills continue from the running N (R11), the resident window included
-        want = O.bulk_v(m, 64, 64, var, 0x7AB1E + W, W, 0, total + n_pref)
+        want = O.bulk_v(m, l, 64, var, 0x7AB1E + W, W, 0, total + n_pref)
         assert np.array_equal(np.array(vals, dtype=np.uint64), want), (nw, key)
