@@ -21,7 +21,9 @@ KEYS = [
     "sm__pipe_fmaheavy_cycles_active.avg.pct_of_peak_sustained_elapsed",
     "sm__inst_executed_pipe_lsu.avg.pct_of_peak_sustained_active",
     "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum", "lts__t_sector_hit_rate.pct",
-    "smsp__inst_executed.sum",
+    "smsp__inst_executed.sum", "sm__cycles_elapsed.avg", "smsp__inst_executed_op_shared_ld.sum",
+    "l1tex__data_pipe_lsu_wavefronts_mem_shared_op_ld.sum",
+    "l1tex__data_bank_conflicts_pipe_lsu_mem_shared_op_ld.sum",
 ]
 STALLS = "smsp__pcsamp_warps_issue_stalled_"
 

@@ -2,7 +2,7 @@
 
     compute-sanitizer --tool memcheck|racecheck|synccheck python tools/sanitize_cases.py
 Covers: init, bulk fill (x2 TMA u64/u32, x1 TMA, LDG, generic m, bipartite,
-l = 1 TMA; the composed-step table kernel and, under the hooks, the R2P and
+l = 1 TMA; the composed-step table kernels (l = 64 and any l) and, under the hooks, the R2P and
 pair kernels), on-demand
 consume in every walk mode, list ranking (Phase I-III, the compaction
 kernel over several tiles), Monte Carlo epoch.
@@ -22,7 +22,7 @@ from paper_conf_ipps_banerjeebk12_b200 import Generator  # noqa: E402
 dev = "cuda:0"
 W = 200  # 3 full 64-walker units + a ragged one
 for kw in ({}, {"m": 256}, {"m": 1000}, {"walk_len": 1}, {"walk_len": 17, "m": 12345},
-           {"variant": 1}):
+           {"walk_len": 13}, {"walk_len": 16, "m": 1 << 20}, {"variant": 1}):
     g = Generator(walkers=W, seed=11, **kw)
     o = torch.empty(W * 5 + 7, dtype=torch.int64, device=dev)
     g.fill(o)
