@@ -30,7 +30,8 @@ for m, W, fmt, var, l in ((1 << 32, 1000, "u64", 0, 64), (1 << 32, 999, "u64", 0
                           (1 << 20, 777, "u64", 0, 64), (1 << 16, 640, "u32", 0, 64),
                           (1 << 32, 1000, "u64", 1, 64), (1 << 12, 333, "u64", 1, 64),
                           (1 << 32, 1000, "u64", 0, 16), (1 << 32, 700, "u64", 0, 13),
-                          (1 << 20, 500, "u64", 0, 2), (1 << 32, 300, "u64", 0, 101)):
+                          (1 << 20, 500, "u64", 0, 2), (1 << 32, 300, "u64", 0, 101),
+                          (1 << 16, 333, "u32", 0, 10)):
     g = Generator(walkers=W, seed=0x7AB1E + W, m=m, epoch_draws=5, variant=var, walk_len=l)
     outs = []
     for n in (7, 3 * W + 5, 2 * W + 2, 9 * W):
