@@ -326,8 +326,7 @@ def run_ours(args, rank, world, local_rank):
     props = torch.cuda.get_device_properties(dev)
     stream = torch.cuda.current_stream()
     # the ranks of one node share the host cores for their FEED threads
-    local_world = int(os.environ.get("LOCAL_WORLD_SIZE", str(world)))
-    feed_threads = max(1, (os.cpu_count() or 1) // max(1, local_world))
+    feed_threads = _feed_threads(world)
 
     def barrier():
         if world > 1:
@@ -526,6 +525,7 @@ def run_ours(args, rank, world, local_rank):
             "feed_s_per_step": (s1["feed_seconds"] - s0["feed_seconds"]) / e2e_steps,
             "api": "prng_fill_host (host FEED threads -> pinned -> H2D -> walk -> D2H to pinned)",
             "host_threads": feed_threads,
+            "feed_pace_mbs": s1["feed_pace_mbs"],
         }
         b = pcie_bound(res["e2e"]["h2d_bytes_per_step"], res["e2e"]["d2h_bytes_per_step"],
                        LABELS_PER_STEP)
@@ -564,8 +564,7 @@ def run_c5(args, rank, world, local_rank):
     dev = torch.device("cuda", local_rank)
     props = torch.cuda.get_device_properties(dev)
     stream = torch.cuda.current_stream()
-    local_world = int(os.environ.get("LOCAL_WORLD_SIZE", str(world)))
-    feed_threads = max(1, (os.cpu_count() or 1) // max(1, local_world))
+    feed_threads = _feed_threads(world)
     Wr = C5_WALKERS // world
     base = rank * Wr
     Lr = C5_LABELS // world
@@ -682,7 +681,10 @@ def host_info():
 
 
 def _feed_threads(world):
-    """Host FEED threads per rank: the ranks of a node share its cores."""
+    """Host FEED threads per rank: the ranks of a node share its cores
+    (GG_BENCH_FEED_THREADS overrides, for A/B runs)."""
+    if os.environ.get("GG_BENCH_FEED_THREADS"):
+        return int(os.environ["GG_BENCH_FEED_THREADS"])
     local_world = int(os.environ.get("LOCAL_WORLD_SIZE", str(world)))
     return max(1, (os.cpu_count() or 1) // max(1, local_world))
 
@@ -824,7 +826,7 @@ def run_apps(args, rank, world, local_rank, max_over_ranks, feed_threads=0):
         "ms_wall_runs": [w * 1e3 for w in walls], "timing": "median of 3 after 1 untimed call",
         "phase_ms": [info["phase1_us"] / 1e3, info["phase2_us"] / 1e3, info["phase3_us"] / 1e3],
         "draws_per_s_e2e": info["draws"] / wall / 1e9, "unit": "GNumbers/s",
-        "ranks_ok": ok,
+        "ranks_ok": ok, "feed_pace_mbs": g.stats()["feed_pace_mbs"],
         "note": "on-demand: the host feeds exactly the draws of each round after learning the "
                 "active count (FEED + H2D inside the measured time)"}
     h2d = _measured_h2d_gbs()

@@ -54,7 +54,8 @@ class prng_options(ctypes.Structure):
 
 class prng_stats(ctypes.Structure):
     _fields_ = [("labels_generated", u64), ("bits_bytes_fed", u64), ("h2d_bytes", u64),
-                ("d2h_bytes", u64), ("kernel_launches", u64), ("feed_seconds", ctypes.c_double)]
+                ("d2h_bytes", u64), ("kernel_launches", u64), ("feed_seconds", ctypes.c_double),
+                ("feed_pace_mbs", u32), ("_reserved", u32)]
 
 
 class gg_mc_layer(ctypes.Structure):

@@ -62,13 +62,15 @@ const uint32_t *walk_table(int device);
 
 // Host feed: SplitMix64 counter-hash stream (R9), SoA rows.
 //   out[r*pitch + i] = word32(seed, tg0 + i, k0 + r),  r < nrows, i < count
-// nt: stream the stores past the CPU caches (bursty feeds; see feed.cpp).
+// nt: stream the stores past the CPU caches (see feed.cpp).  pace_bps > 0:
+// the calling thread writes at most that many bytes per second (feed.cpp Pacer).
 void feed_splitmix_rows(uint64_t seed, uint64_t tg0, uint64_t count, uint64_t k0,
-                        uint32_t nrows, uint32_t *out, uint64_t pitch, bool nt = false);
+                        uint32_t nrows, uint32_t *out, uint64_t pitch, bool nt = false,
+                        double pace_bps = 0);
 // Same for an explicit walker list: column i = global walker base + ids[i].
 void feed_splitmix_rows_ids(uint64_t seed, uint64_t base, const uint32_t *ids, uint64_t count,
                             uint64_t k0, uint32_t nrows, uint32_t *out, uint64_t pitch,
-                            bool nt = false);
+                            bool nt = false, double pace_bps = 0);
 
 // Paper-faithful glibc rand_r seed bits (bit_source 1): see feed.cpp.
 void feed_randr_rows(uint64_t seed, uint64_t tg0, uint64_t count, uint64_t k0, uint32_t nrows,

@@ -32,8 +32,10 @@ namespace {
 class ThreadPool {
   public:
     // cpus: if non-empty, worker i (i >= 1; index 0 is the calling thread,
-    // never pinned) is pinned to cpus[i % cpus.size()].
-    explicit ThreadPool(unsigned n, std::vector<int> cpus = {}) : n_(n ? n : 1) {
+    // never pinned) is pinned to cpus[i % cpus.size()].  Each worker sleeps
+    // on its own condition variable, so a job for the first k threads wakes
+    // only those (the SplitMix feed uses a few writers of a larger pool).
+    explicit ThreadPool(unsigned n, std::vector<int> cpus = {}) : n_(n ? n : 1), slots_(n_) {
         for (unsigned i = 1; i < n_; i++)
             workers_.emplace_back([this, i, cpus] {
                 if (!cpus.empty()) {
@@ -46,60 +48,67 @@ class ThreadPool {
             });
     }
     ~ThreadPool() {
-        {
-            std::lock_guard<std::mutex> g(mu_);
-            stop_ = true;
+        for (unsigned i = 1; i < n_; i++) {
+            std::lock_guard<std::mutex> g(slots_[i].mu);
+            slots_[i].stop = true;
+            slots_[i].cv.notify_one();
         }
-        cv_.notify_all();
         for (auto &t : workers_) t.join();
     }
     unsigned size() const { return n_; }
-    // fn(thread_index) on every thread (the caller is thread 0); returns when all done.
-    void run(const std::function<void(unsigned)> &fn) {
-        if (n_ == 1) {
+    // fn(thread_index) on threads 0 .. k-1 (k = 0: all; the caller is thread
+    // 0); returns when they are done.
+    void run(const std::function<void(unsigned)> &fn, unsigned k = 0) {
+        k = (k == 0 || k > n_) ? n_ : k;
+        if (k == 1) {
             fn(0);
             return;
         }
         {
-            std::lock_guard<std::mutex> g(mu_);
-            job_ = &fn;
-            pending_ = n_ - 1;
-            gen_++;
+            std::lock_guard<std::mutex> g(done_mu_);
+            pending_ = k - 1;
         }
-        cv_.notify_all();
+        for (unsigned i = 1; i < k; i++) {
+            std::lock_guard<std::mutex> g(slots_[i].mu);
+            slots_[i].job = &fn;
+            slots_[i].cv.notify_one();
+        }
         fn(0);
-        std::unique_lock<std::mutex> lk(mu_);
+        std::unique_lock<std::mutex> lk(done_mu_);
         done_cv_.wait(lk, [this] { return pending_ == 0; });
-        job_ = nullptr;
     }
 
   private:
+    struct Slot {
+        std::mutex mu;
+        std::condition_variable cv;
+        const std::function<void(unsigned)> *job = nullptr;
+        bool stop = false;
+    };
     void loop(unsigned idx) {
-        uint64_t seen = 0;
+        Slot &sl = slots_[idx];
         for (;;) {
             const std::function<void(unsigned)> *job;
             {
-                std::unique_lock<std::mutex> lk(mu_);
-                cv_.wait(lk, [&] { return stop_ || gen_ != seen; });
-                if (stop_) return;
-                seen = gen_;
-                job = job_;
+                std::unique_lock<std::mutex> lk(sl.mu);
+                sl.cv.wait(lk, [&] { return sl.stop || sl.job != nullptr; });
+                if (sl.stop) return;
+                job = sl.job;
+                sl.job = nullptr;
             }
             (*job)(idx);
             {
-                std::lock_guard<std::mutex> g(mu_);
+                std::lock_guard<std::mutex> g(done_mu_);
                 if (--pending_ == 0) done_cv_.notify_one();
             }
         }
     }
     unsigned n_;
+    std::vector<Slot> slots_;
     std::vector<std::thread> workers_;
-    std::mutex mu_;
-    std::condition_variable cv_, done_cv_;
-    const std::function<void(unsigned)> *job_ = nullptr;
+    std::mutex done_mu_;
+    std::condition_variable done_cv_;
     unsigned pending_ = 0;
-    uint64_t gen_ = 0;
-    bool stop_ = false;
 };
 
 // CPUs of the GPU's own NUMA node (feed threads next to
@@ -212,6 +221,51 @@ struct Timeline {
     }
 };
 
+// Host FEED pace (SplitMix64 source).  A chunk is written by the pool's
+// threads together, then the copy engine reads it while the next chunks are
+// written.  Streaming stores from every core at once saturate host memory
+// (~180 GB/s on the GPU box) and starve that DMA (55 -> 21 GB/s,
+// tools/host_contention.cu, profiles/r02_host_contention.json); writers
+// at ~66 GB/s leave it at 55.  So the feed threads pace themselves to an
+// aggregate 1.25 x the pinned H2D rate, measured once per device per
+// process (GG_FEED_RATE=<GB/s> forces a cap, 0 = unpaced).  Returns bytes/s.
+double feed_rate_for(int device) {
+    if (const char *e = getenv("GG_FEED_RATE")) return std::max(0.0, atof(e)) * 1e9;
+    static std::mutex mu;
+    static std::vector<std::pair<int, double>> cache;  // device -> bytes/s
+    std::lock_guard<std::mutex> g(mu);
+    for (auto &c : cache)
+        if (c.first == device) return c.second;
+    double h2d_gbs = 55.0;  // pinned 4 x 16 MB after one warm-up copy
+    void *hp = nullptr, *dp = nullptr;
+    cudaStream_t st = nullptr;
+    cudaEvent_t a = nullptr, b = nullptr;
+    const size_t bytes = 16u << 20;
+    if (cudaHostAlloc(&hp, bytes, cudaHostAllocPortable) == cudaSuccess &&
+        cudaMalloc(&dp, bytes) == cudaSuccess &&
+        cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking) == cudaSuccess &&
+        cudaEventCreate(&a) == cudaSuccess && cudaEventCreate(&b) == cudaSuccess) {
+        memset(hp, 0, bytes);
+        cudaMemcpyAsync(dp, hp, bytes, cudaMemcpyHostToDevice, st);
+        cudaEventRecord(a, st);
+        for (int i = 0; i < 4; i++) cudaMemcpyAsync(dp, hp, bytes, cudaMemcpyHostToDevice, st);
+        cudaEventRecord(b, st);
+        float ms = 0;
+        if (cudaEventSynchronize(b) == cudaSuccess && cudaEventElapsedTime(&ms, a, b) == cudaSuccess &&
+            ms > 0)
+            h2d_gbs = 4.0 * bytes / (ms / 1e3) / 1e9;
+    }
+    if (a) cudaEventDestroy(a);
+    if (b) cudaEventDestroy(b);
+    if (st) cudaStreamDestroy(st);
+    if (dp) cudaFree(dp);
+    if (hp) cudaFreeHost(hp);
+    cudaGetLastError();  // a failed probe keeps the default above
+    const double rate = 1.25 * h2d_gbs * 1e9;
+    cache.emplace_back(device, rate);
+    return rate;
+}
+
 struct prng_s {
     Timeline *tl = nullptr;
     const uint32_t *walk_tab = nullptr;  // composed-step table of the device (gg::walk_table)
@@ -225,6 +279,7 @@ struct prng_s {
     cudaStream_t d2h_stream = nullptr;   // D2H of results (prng_fill_host)
     cudaStream_t work_stream = nullptr;  // kernels of prng_fill_host
     ThreadPool *pool = nullptr;
+    double feed_rate = 0;  // aggregate SplitMix feed pace, bytes/s (feed_rate_for; 0 = unpaced)
 
     // walker state (device) and checkpoint copies
     uint32_t *x = nullptr, *y = nullptr, *j = nullptr, *flags = nullptr;
@@ -319,6 +374,7 @@ void feed_chunk(prng_s *h, uint64_t wa, uint64_t wb, uint64_t k0, uint32_t nrows
     const uint64_t cw = wb - wa;
     const bool nt_st = streaming_stores;
     const unsigned nt = h->pool->size();
+    const double pace = h->feed_rate / nt;  // bytes/s per thread (0: unpaced)
     auto t0 = std::chrono::steady_clock::now();
     const double tl0 = h->tl ? h->tl->now_us() : 0.0;
     nvtxRangePushA("gg.feed");
@@ -344,7 +400,7 @@ void feed_chunk(prng_s *h, uint64_t wa, uint64_t wb, uint64_t k0, uint32_t nrows
                                  buf + i, bpitch);
             } else {
                 gg::feed_splitmix_rows_ids(h->seed, h->o.walker_base, ids + wa + lo, hi - lo, k0,
-                                           nrows, buf + lo, bpitch, nt_st);
+                                           nrows, buf + lo, bpitch, nt_st, pace);
             }
             return;
         }
@@ -354,7 +410,7 @@ void feed_chunk(prng_s *h, uint64_t wa, uint64_t wb, uint64_t k0, uint32_t nrows
         else if (h->o.bit_source == PRNG_BITS_CALLBACK)
             h->o.bits_fn(h->o.bits_ctx, tg0, hi - lo, k0, nrows, buf + lo, bpitch);
         else
-            gg::feed_splitmix_rows(h->seed, tg0, hi - lo, k0, nrows, buf + lo, bpitch, nt_st);
+            gg::feed_splitmix_rows(h->seed, tg0, hi - lo, k0, nrows, buf + lo, bpitch, nt_st, pace);
     });
     nvtxRangePop();
     if (h->tl) h->tl->host_span("feed", tl0, h->tl->now_us());
@@ -378,8 +434,10 @@ void stage_rows(prng_s *h, uint64_t k0, uint64_t nrows, uint64_t Wv, uint32_t *d
                 uint64_t dpitch, const uint32_t *ids = nullptr, bool bursty = false,
                 bool row_segments = false) {
     if (nrows == 0 || Wv == 0) return;
-    static const bool nt_all = getenv("GG_FEED_NT_ALL") != nullptr;  // A/B hook
-    bursty = bursty || nt_all;
+    // streaming stores on every window (paced, feed_rate_for; A/B hook
+    // GG_FEED_CACHED=1 restores cached stores for windows >= 1 GB)
+    static const bool cached_bulk = getenv("GG_FEED_CACHED") != nullptr;
+    bursty = bursty || !cached_bulk;
     const uint64_t chunk_words = h->chunk_bytes / 4;
     // Chunks hold an even number of rows (>= 2) so each 64-bit SplitMix word
     // feeds two rows (k even, k+1) with one hash.  Full-width chunks are
@@ -683,6 +741,8 @@ int prng_create(prng_t **out, const prng_graph_params *g, uint64_t walkers, uint
             }
         }
         h->pool = new ThreadPool(nt, cpus);
+        h->feed_rate = h->o.bit_source == PRNG_BITS_SPLITMIX ? feed_rate_for(o.device) : 0.0;
+        h->stats.feed_pace_mbs = (uint32_t)(h->feed_rate / 1e6);
         h->walk_tab = gg::walk_table(o.device);
         if (!h->walk_tab) CK(cudaErrorMemoryAllocation);
         if (const char *tp = getenv("GG_TIMELINE")) {

@@ -19,15 +19,18 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 SHIM = r'''
 #include <cstdint>
 namespace gg {
-void feed_splitmix_rows(uint64_t, uint64_t, uint64_t, uint64_t, uint32_t, uint32_t *, uint64_t, bool);
+void feed_splitmix_rows(uint64_t, uint64_t, uint64_t, uint64_t, uint32_t, uint32_t *, uint64_t, bool,
+                        double);
 void feed_splitmix_rows_ids(uint64_t, uint64_t, const uint32_t *, uint64_t, uint64_t, uint32_t,
-                            uint32_t *, uint64_t, bool);
+                            uint32_t *, uint64_t, bool, double);
 }
 extern "C" void run(uint64_t s, uint64_t t0, uint64_t n, uint64_t k0, uint32_t r, uint32_t *o,
-                    uint64_t p, int nt) { gg::feed_splitmix_rows(s, t0, n, k0, r, o, p, nt != 0); }
+                    uint64_t p, int nt, double pace) {
+    gg::feed_splitmix_rows(s, t0, n, k0, r, o, p, nt != 0, pace);
+}
 extern "C" void run_ids(uint64_t s, uint64_t b, const uint32_t *ids, uint64_t n, uint64_t k0,
-                        uint32_t r, uint32_t *o, uint64_t p, int nt) {
-    gg::feed_splitmix_rows_ids(s, b, ids, n, k0, r, o, p, nt != 0);
+                        uint32_t r, uint32_t *o, uint64_t p, int nt, double pace) {
+    gg::feed_splitmix_rows_ids(s, b, ids, n, k0, r, o, p, nt != 0, pace);
 }
 '''
 
@@ -50,28 +53,45 @@ def aligned(n_words):
     return buf, off
 
 
+@pytest.mark.parametrize("pace", [0.0, 2e8])  # paced feed threads (bytes/s): same words
 @pytest.mark.parametrize("nt", [0, 1])
 @pytest.mark.parametrize("n,pitch,k0,rows", [(1000, 1024, 8, 6), (37, 64, 3, 6), (4096, 4096, 0, 12),
-                                             (13, 32, 2, 1), (1 << 16, 1 << 16, 7, 4)])
-def test_contiguous_rows(feed, n, pitch, k0, rows, nt):
+                                             (13, 32, 2, 1), (1 << 16, 1 << 16, 7, 4),
+                                             (8192 + 37, 8192 + 64, 1, 3)])
+def test_contiguous_rows(feed, n, pitch, k0, rows, nt, pace):
     buf, off = aligned(rows * pitch)
     seed, t0 = 0x5EED0002, 77
     ptr = buf.ctypes.data + off * 4
     feed.run(ctypes.c_uint64(seed), ctypes.c_uint64(t0), ctypes.c_uint64(n), ctypes.c_uint64(k0),
-             ctypes.c_uint32(rows), ctypes.c_void_p(ptr), ctypes.c_uint64(pitch), ctypes.c_int(nt))
+             ctypes.c_uint32(rows), ctypes.c_void_p(ptr), ctypes.c_uint64(pitch), ctypes.c_int(nt),
+             ctypes.c_double(pace))
     got = buf[off:off + rows * pitch].reshape(rows, pitch)[:, :n]
     assert np.array_equal(got, O.stream_block(seed, t0, n, k0, rows))
 
 
+def test_pacer_caps_the_store_rate(feed):
+    """A paced feed thread writes no faster than its cap (prng_capi.cu
+    feed_rate_for: the DMA of earlier chunks keeps its share of host memory)."""
+    import time
+    n, rows, pace = 1 << 16, 16, 4e8          # 4 MiB at 0.4 GB/s: >= 10.5 ms
+    buf, off = aligned(rows * n)
+    t = time.perf_counter()
+    feed.run(ctypes.c_uint64(3), ctypes.c_uint64(0), ctypes.c_uint64(n), ctypes.c_uint64(0),
+             ctypes.c_uint32(rows), ctypes.c_void_p(buf.ctypes.data + off * 4), ctypes.c_uint64(n),
+             ctypes.c_int(1), ctypes.c_double(pace))
+    assert time.perf_counter() - t >= rows * n * 4 / pace * 0.99
+
+
 @pytest.mark.parametrize("nt", [0, 1])
-@pytest.mark.parametrize("n,k0", [(1000, 8), (9, 5), (64, 0)])
+@pytest.mark.parametrize("n,k0", [(1000, 8), (9, 5), (64, 0), (8192 + 9, 3)])
 def test_walker_list_rows(feed, n, k0, nt):
-    rows, pitch = 6, 1024
+    rows, pitch = 6, max(1024, (n + 63) // 64 * 64)
     buf, off = aligned(rows * pitch)
     ids = np.random.default_rng(n).permutation(20000)[:n].astype(np.uint32)
     feed.run_ids(ctypes.c_uint64(11), ctypes.c_uint64(500), ctypes.c_void_p(ids.ctypes.data),
                  ctypes.c_uint64(n), ctypes.c_uint64(k0), ctypes.c_uint32(rows),
-                 ctypes.c_void_p(buf.ctypes.data + off * 4), ctypes.c_uint64(pitch), ctypes.c_int(nt))
+                 ctypes.c_void_p(buf.ctypes.data + off * 4), ctypes.c_uint64(pitch), ctypes.c_int(nt),
+                 ctypes.c_double(1e9 if nt else 0.0))
     got = buf[off:off + rows * pitch].reshape(rows, pitch)[:, :n]
     want = np.stack([O.stream_block(11, 500 + int(t), 1, k0, rows)[:, 0] for t in ids], axis=1)
     assert np.array_equal(got, want)
