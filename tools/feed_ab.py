@@ -5,8 +5,9 @@
 Host-side rates on the GPU box drift between runs by 10-30%, so configs are
 run round-robin (A B C A B C ...), each in a fresh process, and medians are
 reported.  Each process measures, for its env settings:
-  e2e   -- prng_fill_host of 2^20 walkers x 64 draws (the C2 generator,
-           1.6 GB of seed bits, labels to pinned host memory), wall time;
+  e2e   -- prng_fill_host of 2^20 walkers x 512 draws (the bench's C2 e2e
+           step: 12.9 GB of seed bits, labels to pinned host memory; AB_E2E_DRAWS
+           changes the draws), best wall time of 2;
   lr    -- C3's FEED pipeline: C3's per-round active counts (computed once
            by the parent) replayed through prng_epoch_begin / prng_epoch_end
            (bits generated and copied, no kernels), wall time.
@@ -30,7 +31,8 @@ act = json.load(open(sys.argv[1]))
 ht = int(os.environ.get("HOST_THREADS", "0"))
 W = 1 << 20
 g = Generator(walkers=W, seed=0x5EED0002, epoch_draws=16, host_threads=ht)
-host = torch.empty(W * 64, dtype=torch.int64).pin_memory()
+D = int(os.environ.get("AB_E2E_DRAWS", "512"))  # 512: the bench e2e step (2^29 labels)
+host = torch.empty(W * D, dtype=torch.int64).pin_memory()
 g.fill_host(host, n=W * 8)
 g.mark()
 e2e = []
@@ -56,7 +58,7 @@ for _ in range(3):
     torch.cuda.synchronize()
     lr.append(time.perf_counter() - t)
 g.close()
-print(json.dumps({"e2e_gnum_s": W * 64 / min(e2e) / 1e9, "lr_ms": min(lr) * 1e3, "pace_mbs": writers}))
+print(json.dumps({"e2e_gnum_s": W * D / min(e2e) / 1e9, "lr_ms": min(lr) * 1e3, "pace_mbs": writers}))
 """
 
 
