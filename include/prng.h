@@ -241,7 +241,7 @@ typedef struct {
     uint64_t d2h_bytes;          /* bytes copied device -> host */
     uint64_t kernel_launches;    /* launches of the library's kernels */
     double feed_seconds;         /* wall time host threads spent generating */
-    uint32_t feed_pace_mbs;      /* SplitMix64 feed threads' aggregate store-rate cap, MB/s:
+    uint32_t feed_pace_mbs;      /* SplitMix64 feed threads' aggregate streaming-store cap, MB/s:
                                     1.25 x the pinned H2D rate measured at the first create
                                     on a device (0 = unpaced; GG_FEED_RATE overrides) */
     uint32_t _reserved;

@@ -221,9 +221,10 @@ struct Timeline {
     }
 };
 
-// Host FEED pace (SplitMix64 source).  A chunk is written by the pool's
-// threads together, then the copy engine reads it while the next chunks are
-// written.  Streaming stores from every core at once saturate host memory
+// Host FEED pace (SplitMix64 source, streaming-store windows: on-demand
+// epochs < 1 GB).  A chunk is written by the pool's threads together, then
+// the copy engine reads it while the next chunks are written.  Streaming
+// stores from every core at once saturate host memory
 // (~180 GB/s on the GPU box) and starve that DMA (55 -> 21 GB/s,
 // tools/host_contention.cu, profiles/r02_host_contention.json); writers
 // at ~66 GB/s leave it at 55.  So the feed threads pace themselves to an
@@ -374,7 +375,10 @@ void feed_chunk(prng_s *h, uint64_t wa, uint64_t wb, uint64_t k0, uint32_t nrows
     const uint64_t cw = wb - wa;
     const bool nt_st = streaming_stores;
     const unsigned nt = h->pool->size();
-    const double pace = h->feed_rate / nt;  // bytes/s per thread (0: unpaced)
+    // streaming stores are paced (feed_rate_for); cached stores (long bulk
+    // streams) are not: they measured faster unpaced (C2 E-mode 2.04 vs 1.74
+    // G/s streaming unpaced, 1.90 streaming paced, tools/feed_ab.py)
+    const double pace = nt_st ? h->feed_rate / nt : 0.0;  // bytes/s per thread
     auto t0 = std::chrono::steady_clock::now();
     const double tl0 = h->tl ? h->tl->now_us() : 0.0;
     nvtxRangePushA("gg.feed");
@@ -434,10 +438,8 @@ void stage_rows(prng_s *h, uint64_t k0, uint64_t nrows, uint64_t Wv, uint32_t *d
                 uint64_t dpitch, const uint32_t *ids = nullptr, bool bursty = false,
                 bool row_segments = false) {
     if (nrows == 0 || Wv == 0) return;
-    // streaming stores on every window (paced, feed_rate_for; A/B hook
-    // GG_FEED_CACHED=1 restores cached stores for windows >= 1 GB)
-    static const bool cached_bulk = getenv("GG_FEED_CACHED") != nullptr;
-    bursty = bursty || !cached_bulk;
+    static const bool nt_all = getenv("GG_FEED_NT_ALL") != nullptr;  // A/B hook
+    bursty = bursty || nt_all;
     const uint64_t chunk_words = h->chunk_bytes / 4;
     // Chunks hold an even number of rows (>= 2) so each 64-bit SplitMix word
     // feeds two rows (k even, k+1) with one hash.  Full-width chunks are

@@ -48,7 +48,7 @@ VARIANTS = ["GG_FILL_TABLE=0", _R2P + "GG_FILL_NO_TMA=1", _R2P + "GG_FILL_X1=1",
             _R2P + "GG_FILL_MINB=24", _R2P + "GG_FILL_STEP=0", _R2P + "GG_FILL_U2=0",
             _R2P + "GG_FILL_MINB=24 GG_FILL_U2=0",
             _R2P + "GG_FILL_ONEWAVE=1", _R2P + "GG_FILL_KPW=2", "GG_FILL_KPW=3", "GG_FILL_TABLE=2 GG_FILL_KPW=2", "GG_FILL_TABLE=8", "GG_FILL_ORB=0",
-            "GG_FEED_CACHED=1", "GG_FEED_NO_NT=1", "GG_FEED_RATE=0", "GG_FEED_RATE=5",
+            "GG_FEED_NT_ALL=1", "GG_FEED_NO_NT=1", "GG_FEED_RATE=0", "GG_FEED_RATE=5",
             "GG_FEED_CHUNK_MB=1", "GG_FEED_CHUNKS=2", "GG_MC_MINB=4", _R2P + "GG_FILL_PAIR=1"]
 
 

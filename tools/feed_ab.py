@@ -1,6 +1,6 @@
 """Interleaved A/B of host FEED settings (tool; §IV-A Fig.4-5).
 
-    python tools/feed_ab.py [--reps 3] "" "GG_FEED_RATE=0 GG_FEED_CACHED=1" "GG_FEED_RATE=70" ...
+    python tools/feed_ab.py [--reps 3] "" "GG_FEED_RATE=0" "GG_FEED_RATE=70" ...
 
 Host-side rates on the GPU box drift between runs by 10-30%, so configs are
 run round-robin (A B C A B C ...), each in a fresh process, and medians are
