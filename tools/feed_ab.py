@@ -10,7 +10,8 @@ reported.  Each process measures, for its env settings:
            changes the draws), best wall time of 2;
   lr    -- C3's FEED pipeline: C3's per-round active counts (computed once
            by the parent) replayed through prng_epoch_begin / prng_epoch_end
-           (bits generated and copied, no kernels), wall time.
+           (bits generated and copied, no kernels), wall time;
+  c3    -- the full C3 list ranking (median of 3 after one untimed call).
 HOST_THREADS=n sets the pool size (host_threads); the library's other
 knobs are read from the environment.
 """
@@ -58,7 +59,21 @@ for _ in range(3):
     torch.cuda.synchronize()
     lr.append(time.perf_counter() - t)
 g.close()
-print(json.dumps({"e2e_gnum_s": W * D / min(e2e) / 1e9, "lr_ms": min(lr) * 1e3, "pace_mbs": writers}))
+# the full C3 list ranking (kernels + on-demand FEED), median of 3 after one untimed call
+import inputs
+succ, pred, head = inputs.random_list(n, 0x5EED0003)
+g = Generator(walkers=n, seed=0x5EED0003, host_threads=ht)
+s_t, p_t = torch.from_numpy(succ).cuda(), torch.from_numpy(pred).cuda()
+g.list_rank(s_t, p_t, head)
+c3 = []
+for _ in range(3):
+    torch.cuda.synchronize()
+    t = time.perf_counter()
+    g.list_rank(s_t, p_t, head)
+    torch.cuda.synchronize()
+    c3.append(time.perf_counter() - t)
+g.close()
+print(json.dumps({"c3_ms": sorted(c3)[1] * 1e3, "e2e_gnum_s": W * D / min(e2e) / 1e9, "lr_ms": min(lr) * 1e3, "pace_mbs": writers}))
 """
 
 
@@ -97,6 +112,7 @@ def main():
         out["configs"][c] = {
             "e2e_gnum_s_median": statistics.median(r["e2e_gnum_s"] for r in ok),
             "lr_ms_median": statistics.median(r["lr_ms"] for r in ok),
+            "c3_ms_median": statistics.median(r["c3_ms"] for r in ok),
             "pace_mbs": ok[0]["pace_mbs"], "runs": ok}
     print(json.dumps(out, indent=1))
 
