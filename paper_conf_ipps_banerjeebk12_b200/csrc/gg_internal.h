@@ -94,6 +94,15 @@ void feed_ggcpu_rows(uint64_t seed, uint64_t base, uint64_t l0, const uint32_t *
 // pitch `pitch`) ahead of prng_epoch_begin (prng_capi.cu); list ranking.
 int epoch_prefeed(prng_s *h, uint64_t hi, uint64_t pitch);
 
+// Timeline recorder of the handle (GG_TIMELINE, diagnostic; prng_capi.cu):
+// host clock in us (< 0 when the recorder is off), a host interval, and a
+// device interval as an event pair on stream s (tl_dev_begin returns null
+// when off; tl_dev_end(h, kind, null, s) is a no-op).
+double tl_now_us(prng_s *h);
+void tl_host_span(prng_s *h, const char *kind, double a_us, double b_us);
+cudaEvent_t tl_dev_begin(prng_s *h, cudaStream_t s);
+void tl_dev_end(prng_s *h, const char *kind, cudaEvent_t a, cudaStream_t s);
+
 // Stable single-pass compaction (compact.cu): items i < n with flags[i] != 0
 // go, in order, to kept_out (the item is in[i], or i when in is null); the
 // others, in order, to removed_out (if not null).  The kept count is written

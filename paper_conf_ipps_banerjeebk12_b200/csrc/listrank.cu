@@ -369,7 +369,10 @@ extern "C" int gg_list_rank(prng_t *h, int64_t n, const int32_t *succ, const int
         static const bool trace = getenv("GG_LR_TRACE") != nullptr;
         while (A > target && rounds < 1000) {
             auto tr0 = std::chrono::steady_clock::now();
+            const double tb0 = gg::tl_now_us(h);
             LRC(prng_epoch_begin(h, (uint64_t)A, 1, s));
+            gg::tl_host_span(h, "lr.begin", tb0, gg::tl_now_us(h));
+            cudaEvent_t tk0 = gg::tl_dev_begin(h, s);
             auto tr1 = std::chrono::steady_clock::now();
             static const bool fine = trace && atoi(getenv("GG_LR_TRACE")) >= 2;
             auto sync_t = [&](const char *what, std::chrono::steady_clock::time_point &t) {
@@ -398,19 +401,32 @@ extern "C" int gg_list_rank(prng_t *h, int64_t n, const int32_t *succ, const int
             LCK(gg::compact_flagged(act, keep, A, act2, rem_log + log_off, d_num, slot.p, tag, tmp,
                                     s));
             sync_t("partition", tq);
+            gg::tl_dev_end(h, "lr.kernels", tk0, s);
             // While this round's kernels run, stage the next round's bits for the
-            // slots that certainly stay active: an interior node is removed with
-            // probability 1/8 (Alg.3 l.8-9), so the survivors are ~7/8 A with a
-            // standard deviation of sqrt(7A)/8; slots below 7/8 A - 8 sd (and the
-            // window pitch of this round, an upper bound) are safe.  Off with
-            // GG_LR_PREFEED=0.
-            static const bool prefeed = !(getenv("GG_LR_PREFEED") && atoi(getenv("GG_LR_PREFEED")) == 0);
-            if (prefeed && A > 4096) {
+            // slots that will most likely stay active: an interior node is removed
+            // with probability 1/8 (Alg.3 l.8-9), so the survivors are ~7/8 A with
+            // a standard deviation of sqrt(7A)/8.  Staging up to 7/8 A + 3 sd
+            // (capped at this round's pitch, an upper bound) leaves no remainder
+            // to stage after the count is known in all but ~0.1% of rounds, at
+            // ~3 sd x 24 B of unused bits (~40 KB at A = 2^24); a remainder, when
+            // there is one, is staged by the next prng_epoch_begin.  Bits are a
+            // pure function of (seed, slot, round), so the numbers do not depend
+            // on this bound.  GG_LR_PREFEED=0: off; =2: the round-1 bound 7/8 A -
+            // 8 sd (never more than the survivors; one remainder every round).
+            static const int prefeed_mode =
+                getenv("GG_LR_PREFEED") ? atoi(getenv("GG_LR_PREFEED")) : 1;
+            if (prefeed_mode != 0 && A > 4096) {
                 const double sd = std::sqrt(7.0 * (double)A) / 8.0;
-                const int64_t lo = (int64_t)(0.875 * (double)A - 8.0 * sd);
+                const int64_t lo = prefeed_mode == 2
+                                       ? (int64_t)(0.875 * (double)A - 8.0 * sd)
+                                       : std::min<int64_t>(A, (int64_t)(0.875 * (double)A + 3.0 * sd));
+                const double tp0 = gg::tl_now_us(h);
                 if (lo > 0) LRC(gg::epoch_prefeed(h, (uint64_t)lo, ((uint64_t)A + 31) / 32 * 32));
+                gg::tl_host_span(h, "lr.prefeed", tp0, gg::tl_now_us(h));
             }
+            const double tw0 = gg::tl_now_us(h);
             const int32_t kept = wait_count(slot.p, tag, s);
+            gg::tl_host_span(h, "lr.wait", tw0, gg::tl_now_us(h));
             if (trace) {
                 auto tr2 = std::chrono::steady_clock::now();
                 fprintf(stderr, "[lr] round %ld A=%ld feed+enqueue %.3f ms, kernels+sync %.3f ms\n",

@@ -3,6 +3,7 @@
 // staging pipeline (FEED -> TRANSFER, §IV-A Fig.4), resident and
 // streamed bit windows, on-demand epochs (R10), checkpoints.
 #include <algorithm>
+#include <atomic>
 #include <cctype>
 #include <sched.h>
 #include <pthread.h>
@@ -382,6 +383,41 @@ void feed_chunk(prng_s *h, uint64_t wa, uint64_t wb, uint64_t k0, uint32_t nrows
     auto t0 = std::chrono::steady_clock::now();
     const double tl0 = h->tl ? h->tl->now_us() : 0.0;
     nvtxRangePushA("gg.feed");
+    static const bool static_slices = getenv("GG_FEED_STATIC") != nullptr;  // A/B hook
+    if (nt_st && h->o.bit_source == PRNG_BITS_SPLITMIX && !static_slices) {
+        // Streaming-store windows: blocks of kBlk walkers claimed in order
+        // from a shared counter, block b released at t0 + (bytes before b) /
+        // feed_rate.  One clock for the whole pool: a worker that wakes late
+        // or is descheduled leaves its blocks to the others instead of
+        // finishing the chunk late (per-thread slices with per-thread pacing
+        // made each chunk as slow as its slowest writer).
+        constexpr uint64_t kBlk = 4096;  // 16 KB per row, 64 B aligned
+        const uint64_t nblk = (cw + kBlk - 1) / kBlk;
+        const double blk_s = h->feed_rate > 0 ? (double)kBlk * nrows * 4 / h->feed_rate : 0.0;
+        std::atomic<uint64_t> next{0};
+        h->pool->run([&](unsigned) {
+            for (;;) {
+                const uint64_t b = next.fetch_add(1, std::memory_order_relaxed);
+                if (b >= nblk) return;
+                if (blk_s > 0) {
+                    const double due = (double)b * blk_s;
+                    while (std::chrono::duration<double>(std::chrono::steady_clock::now() - t0)
+                               .count() < due) {
+#if defined(__x86_64__)
+                        __builtin_ia32_pause();
+#endif
+                    }
+                }
+                const uint64_t lo = b * kBlk, hi = std::min(cw, lo + kBlk);
+                if (ids)
+                    gg::feed_splitmix_rows_ids(h->seed, h->o.walker_base, ids + wa + lo, hi - lo,
+                                               k0, nrows, buf + lo, bpitch, true, 0.0);
+                else
+                    gg::feed_splitmix_rows(h->seed, h->o.walker_base + wa + lo, hi - lo, k0, nrows,
+                                           buf + lo, bpitch, true, 0.0);
+            }
+        });
+    } else
     h->pool->run([&](unsigned ti) {
         // contiguous, 16-walker aligned slices
         uint64_t per = round_up((cw + nt - 1) / nt, 16);
@@ -485,7 +521,11 @@ void stage_rows(prng_s *h, uint64_t k0, uint64_t nrows, uint64_t Wv, uint32_t *d
             if (((k0 + r) & 1) && nr > 1) nr -= 1;  // keep later chunks pair-aligned
             const int b = h->chunk_next;
             h->chunk_next = (b + 1) % h->kChunks;
-            CK(cudaEventSynchronize(h->chunk_done[b]));  // pinned chunk free again
+            {  // pinned chunk free again
+                const double w0 = h->tl ? h->tl->now_us() : 0.0;
+                CK(cudaEventSynchronize(h->chunk_done[b]));
+                if (h->tl) h->tl->host_span("ring_wait", w0, h->tl->now_us());
+            }
             feed_chunk(h, 0, Wv, k0 + r, (uint32_t)nr, h->chunk[b], ids, dpitch, bursty);
             h2d_copy(h, dst + r * dpitch, h->chunk[b], nr * dpitch * 4);
             CK(cudaEventRecord(h->chunk_done[b], h->copy_stream));
@@ -502,7 +542,11 @@ void stage_rows(prng_s *h, uint64_t k0, uint64_t nrows, uint64_t Wv, uint32_t *d
             const uint64_t wb = std::min<uint64_t>(Wv, wa + walkers_per);
             const int b = h->chunk_next;
             h->chunk_next = (b + 1) % h->kChunks;
-            CK(cudaEventSynchronize(h->chunk_done[b]));
+            {
+                const double w0 = h->tl ? h->tl->now_us() : 0.0;
+                CK(cudaEventSynchronize(h->chunk_done[b]));
+                if (h->tl) h->tl->host_span("ring_wait", w0, h->tl->now_us());
+            }
             const uint64_t cw = wb - wa;
             // rows start 32-B aligned in the chunk, so the streaming-store path
             // (feed.cpp nt_ok) covers the ragged last segment too: cached
@@ -1120,6 +1164,15 @@ namespace gg {
 // next prng_epoch_begin with draws = 1 and active <= pitch stages only the
 // walkers above hi.  No effect on the numbers: a walker's bits at a draw are
 // a pure function of (seed, walker, draw) (R9).
+double tl_now_us(prng_s *h) { return h && h->tl ? h->tl->now_us() : -1.0; }
+void tl_host_span(prng_s *h, const char *kind, double a_us, double b_us) {
+    if (h && h->tl && a_us >= 0.0) h->tl->host_span(kind, a_us, b_us);
+}
+cudaEvent_t tl_dev_begin(prng_s *h, cudaStream_t s) { return h && h->tl ? h->tl->begin(s) : nullptr; }
+void tl_dev_end(prng_s *h, const char *kind, cudaEvent_t a, cudaStream_t s) {
+    if (h && h->tl && a) h->tl->end(kind, a, s);
+}
+
 int epoch_prefeed(prng_t *h, uint64_t hi, uint64_t pitch) {
     if (!h || h->od_open || !h->od_started || hi == 0 || hi > pitch || pitch > round_up(h->W, 32))
         return PRNG_E_INVALID;

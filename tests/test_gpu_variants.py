@@ -49,7 +49,8 @@ VARIANTS = ["GG_FILL_TABLE=0", _R2P + "GG_FILL_NO_TMA=1", _R2P + "GG_FILL_X1=1",
             _R2P + "GG_FILL_MINB=24 GG_FILL_U2=0",
             _R2P + "GG_FILL_ONEWAVE=1", _R2P + "GG_FILL_KPW=2", "GG_FILL_KPW=3", "GG_FILL_TABLE=2 GG_FILL_KPW=2", "GG_FILL_TABLE=8", "GG_FILL_ORB=0",
             "GG_FEED_NT_ALL=1", "GG_FEED_NO_NT=1", "GG_FEED_RATE=0", "GG_FEED_RATE=5",
-            "GG_FEED_CHUNK_MB=1", "GG_FEED_CHUNKS=2", "GG_MC_MINB=4", _R2P + "GG_FILL_PAIR=1"]
+            "GG_FEED_CHUNK_MB=1", "GG_FEED_CHUNKS=2", "GG_MC_MINB=4", _R2P + "GG_FILL_PAIR=1",
+            "GG_FEED_STATIC=1", "GG_FEED_STATIC=1 GG_FEED_RATE=0"]
 
 
 @pytest.fixture(scope="module")
@@ -120,3 +121,45 @@ def test_l1_tma_store_several_units_per_warp(var, tmp_path):
     got = np.load(f)
     W = 32 * 700 + 5
     assert np.array_equal(got, O.bulk(M32, 1, 64, 0x5EED00F1, W, 0, W * 70 - 3)), var
+
+
+LR_SNIPPET = r"""
+import json, sys
+import numpy as np, torch
+sys.path.insert(0, %(root)r)
+import inputs
+from paper_conf_ipps_banerjeebk12_b200 import Generator
+n = 1 << 16
+succ, pred, head = inputs.random_list(n, 100 + n)
+g = Generator(walkers=n, seed=0x5EED0003)
+rr = torch.empty(n, dtype=torch.int32, device="cuda")
+sp = torch.empty(n, dtype=torch.int32, device="cuda")
+rank, info = g.list_rank(torch.from_numpy(succ).cuda(), torch.from_numpy(pred).cuda(), head,
+                         removed_round=rr, is_splitter=sp)
+print(json.dumps({"rank": rank.cpu().tolist(), "rr": rr.cpu().tolist(), "sp": sp.cpu().tolist(),
+                  "draws": info["draws"]}))
+"""
+
+
+@pytest.mark.parametrize("var", ["GG_LR_PREFEED=0", "GG_LR_PREFEED=2", "GG_FEED_STATIC=1",
+                                 "GG_FEED_CHUNK_MB=1"])
+def test_list_ranking_feed_variants_bit_exact(var):
+    """List-ranking prefeed bounds (none / the survivors' lower bound / the
+    default 7/8 A + 3 sd) and feed schedules give the oracle replica's FIS and
+    splitter sets (2^16 nodes: every round but the last few is prefed)."""
+    import inputs
+    env = dict(os.environ)
+    for kv in var.split():
+        k, v = kv.split("=")
+        env[k] = v
+    out = subprocess.run([sys.executable, "-c", LR_SNIPPET % {"root": ROOT}], env=env,
+                         capture_output=True, text=True, timeout=300)
+    assert out.returncode == 0, out.stderr[-2000:]
+    got = json.loads(out.stdout.strip().splitlines()[-1])
+    n = 1 << 16
+    succ, pred, head = inputs.random_list(n, 100 + n)
+    want = O.lr_run(succ, pred, head, seed=0x5EED0003)
+    assert np.array_equal(np.array(got["rank"], dtype=np.int32), O.lr_rank_seq(succ, head))
+    assert np.array_equal(np.array(got["rr"], dtype=np.int32), want["removed_round"]), var
+    assert np.array_equal(np.array(got["sp"], dtype=np.int32).astype(bool), want["is_splitter"]), var
+    assert got["draws"] == want["draws"], var
