@@ -1,7 +1,7 @@
 """Crush-scale battery on GPU output (tool; §IV-B,
 Table III: SmallCrush 15/15, Crush 14/15, BigCrush 13/15).
 
-    python tools/battery_big.py [--log2-words 33] > profiles/r02_battery.json
+    python tools/battery_big.py [--log2-words 33] [--streams 0,1] > profiles/r02_battery.json
 
 Streams 2^log2-words u32 words (default 2^33 = 2^32 labels) of the generator
 through the 15 streaming statistics of tests/battery_gpu.py (computed with
@@ -105,6 +105,7 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--log2-words", type=int, default=33)
     ap.add_argument("--log2-words-controls", type=int, default=28)
+    ap.add_argument("--streams", default="", help="comma-separated stream indices (default: all)")
     args = ap.parse_args()
     L = 1 << (args.log2_words - 1)
     Lc = 1 << (args.log2_words_controls - 1)
@@ -121,6 +122,8 @@ def main():
         ("control: walker-major l=16", lambda: gen_chunks(Lc, 4096, walk_len=16, walker_major=True)),
         ("control: 32-bit LCG", lambda: lcg_chunks(Lc)),
     ]
+    if args.streams:
+        runs = [runs[int(i)] for i in args.streams.split(",")]
     for name, mk in runs:
         t = time.perf_counter()
         r = run_stream(mk(), G.crush_scale_tests())
