@@ -1129,9 +1129,13 @@ static int epoch_begin_impl(prng_t *h, uint64_t active_walkers, const uint32_t *
             h->od_wmap = h->od_wmap_buf[slot];
             h->stats.h2d_bytes += active_walkers * 4;
         }
-        // small windows are bursty (the consumer waits for the last chunk):
-        // stream them past the CPU caches; large windows pipeline like bulk
-        const bool bursty = bytes < (1ull << 30);
+        // on-demand windows go past the CPU caches with paced streaming
+        // stores (the consumer waits for the last chunk).  Windows >= 1 GB
+        // (C4's 1.2 GB Monte Carlo epochs) used cached stores like bulk
+        // streams until the shared-clock feed blocks; A/B hook
+        // GG_FEED_EPOCH_CACHED=1 restores that.
+        static const bool epoch_cached = getenv("GG_FEED_EPOCH_CACHED") != nullptr;
+        const bool bursty = !epoch_cached || bytes < (1ull << 30);
         if (pf) {
             if (active_walkers > h->pf_hi) {  // the rest: walkers [pf_hi, active)
                 const uint64_t lo = h->pf_hi, saved = h->o.walker_base;
