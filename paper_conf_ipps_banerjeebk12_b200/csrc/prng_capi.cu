@@ -420,7 +420,7 @@ void feed_chunk(prng_s *h, uint64_t wa, uint64_t wb, uint64_t k0, uint32_t nrows
                                            buf + lo, bpitch, nt_st, 0.0);
             }
         });
-    } else
+    } else {
     h->pool->run([&](unsigned ti) {
         // contiguous, 16-walker aligned slices
         uint64_t per = round_up((cw + nt - 1) / nt, 16);
@@ -455,6 +455,7 @@ void feed_chunk(prng_s *h, uint64_t wa, uint64_t wb, uint64_t k0, uint32_t nrows
         else
             gg::feed_splitmix_rows(h->seed, tg0, hi - lo, k0, nrows, buf + lo, bpitch, nt_st, pace);
     });
+    }
     nvtxRangePop();
     if (h->tl) h->tl->host_span("feed", tl0, h->tl->now_us());
     auto t1 = std::chrono::steady_clock::now();
@@ -1164,13 +1165,6 @@ static int epoch_begin_impl(prng_t *h, uint64_t active_walkers, const uint32_t *
 
 extern "C++" {
 namespace gg {
-// Stage the next epoch's window ahead (one draw, walkers [0, hi), pitch
-// `pitch` >= the next epoch's active count) while the current epoch's
-// kernels run: list ranking knows the next round's active count only after
-// its kernels, but not fewer than ~7/8 of this round's nodes survive.  The
-// next prng_epoch_begin with draws = 1 and active <= pitch stages only the
-// walkers above hi.  No effect on the numbers: a walker's bits at a draw are
-// a pure function of (seed, walker, draw) (R9).
 double tl_now_us(prng_s *h) { return h && h->tl ? h->tl->now_us() : -1.0; }
 void tl_host_span(prng_s *h, const char *kind, double a_us, double b_us) {
     if (h && h->tl && a_us >= 0.0) h->tl->host_span(kind, a_us, b_us);
@@ -1180,6 +1174,13 @@ void tl_dev_end(prng_s *h, const char *kind, cudaEvent_t a, cudaStream_t s) {
     if (h && h->tl && a) h->tl->end(kind, a, s);
 }
 
+// Stage the next epoch's window ahead (one draw, walkers [0, hi), pitch
+// `pitch` >= the next epoch's active count) while the current epoch's
+// kernels run: list ranking knows the next round's active count only after
+// its kernels, but not fewer than ~7/8 of this round's nodes survive.  The
+// next prng_epoch_begin with draws = 1 and active <= pitch stages only the
+// walkers above hi.  No effect on the numbers: a walker's bits at a draw are
+// a pure function of (seed, walker, draw) (R9).
 int epoch_prefeed(prng_t *h, uint64_t hi, uint64_t pitch) {
     if (!h || h->od_open || !h->od_started || hi == 0 || hi > pitch || pitch > round_up(h->W, 32))
         return PRNG_E_INVALID;
