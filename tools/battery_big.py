@@ -31,10 +31,12 @@ CHUNK = 1 << 28   # labels per fill (2 GiB)
 SUB = 1 << 26     # labels per feed() call
 
 
-def gen_chunks(total_labels, walkers, walk_len=64, seed=0x5EED00B1, walker_major=False):
+def gen_chunks(total_labels, walkers, walk_len=64, seed=0x5EED00B1, walker_major=False,
+               variant=0, bit_source=0):
     # few walkers: deep ring slots, so each streamed window is ~100 MB of bits
     g = Generator(walkers=walkers, seed=seed, walk_len=walk_len,
-                  epoch_draws=16 if walkers >= (1 << 18) else 1024)
+                  epoch_draws=16 if walkers >= (1 << 18) else 1024, variant=variant,
+                  bit_source=bit_source)
     out = torch.empty(min(CHUNK, total_labels), dtype=torch.int64, device="cuda")
     done = 0
     while done < total_labels:
@@ -105,9 +107,12 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--log2-words", type=int, default=33)
     ap.add_argument("--log2-words-controls", type=int, default=28)
-    ap.add_argument("--streams", default="", help="comma-separated stream indices (default: all)")
+    ap.add_argument("--streams", default="", help="comma-separated stream indices (default: 0-4)")
+    ap.add_argument("--log2-words-extra", type=int, default=33,
+                    help="size of streams 5 (bipartite walk) and 6 (glibc rand_r seed bits)")
     args = ap.parse_args()
     L = 1 << (args.log2_words - 1)
+    Lx = 1 << (args.log2_words_extra - 1)
     Lc = 1 << (args.log2_words_controls - 1)
     rep = {"what": "15 streaming Crush-style statistics (tests/battery_gpu.py) computed with torch "
                    "on the GPU; fail = one-sided p outside [1e-4, 1-1e-4] or two-sided p < 1e-4",
@@ -121,9 +126,12 @@ def main():
         ("control: bulk l=1", lambda: gen_chunks(Lc, 1 << 20, walk_len=1)),
         ("control: walker-major l=16", lambda: gen_chunks(Lc, 4096, walk_len=16, walker_major=True)),
         ("control: 32-bit LCG", lambda: lcg_chunks(Lc)),
+        # f1: the bipartite sigma / sigma^-1 walk; f3: the paper's glibc rand_r
+        # LCG as the seed-bit source (§III-B), both C2-shaped, bulk order
+        ("bipartite l=64", lambda: gen_chunks(Lx, 1 << 20, variant=1)),
+        ("rand_r seed bits l=64", lambda: gen_chunks(Lx, 1 << 20, bit_source=1)),
     ]
-    if args.streams:
-        runs = [runs[int(i)] for i in args.streams.split(",")]
+    runs = [runs[int(i)] for i in args.streams.split(",")] if args.streams else runs[:5]
     for name, mk in runs:
         t = time.perf_counter()
         r = run_stream(mk(), G.crush_scale_tests())
